@@ -1,0 +1,356 @@
+#!/usr/bin/env python
+"""bench.py -- TagMatch B200 throughput (driver contract).
+
+A step = one tm_match_batch over one batch of queries = the whole hot path
+(encode, route, batch, pre-filter, subset scan, compaction,
+key expansion, sort/merge).  Default workload: BASELINE config C2 (1M tag
+sets, 100k-query stream, MAX_P = 200K), `match` (Table 1).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C2] [--unique]
+
+value  : queries/s over all ranks, inputs resident in HBM (tm_match_batch_device),
+         per-step CUDA events on the launching stream, L2 flushed between steps.
+e2e    : queries/s through tm_match_batch with pinned host queries (H2D inside
+         the timed region) and the sorted pairs copied back to host (D2H).
+N > 1  : one process per GPU (torchrun); every rank holds a replica of the
+         database and matches its own query batch (replicated mode, PAPER.md:110,
+         228: no data-path collective) -> "scaling": "weak"; time = max over ranks.
+--impl reference : the oracle (oracle/o2.c, the paper's CPU method) on the
+         host cores, on a bounded sample of the same workload per step.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "queries/sec vs DB size at 1/2/4/8 B200; subset-scan HBM GB/s vs roofline"
+ALU_LANES_PER_SM_CLK = 64     # LOP3/IADD3 ALU pipe: 16 lanes/clk/SMSP x 4 SMSP (B300_MICROARCH.md)
+SM_COUNT = 148
+# algorithmic INT ops: ~4 per (tile, query) prefix test, 7 per (set, query) check
+OPS_PER_TILE_TEST = 4
+OPS_PER_PAIR_CHECK = 7
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons with NVML during the timed region."""
+
+    def __init__(self, device_index: int):
+        self.samples, self.reasons, self.max_mhz = [], set(), None
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(device_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            pass
+        self._stop = threading.Event()
+        self._t = None
+
+    _REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown",
+                0x4: "sw_power_cap", 0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks_setting",
+                0x1: "gpu_idle", 0x100: "display_clock_setting", 0x10: "sync_boost"}
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for bit, name in self._REASONS.items():
+                    if r & bit and name != "gpu_idle":
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            time.sleep(0.02)
+
+    def __enter__(self):
+        if self.ok:
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons), "samples": 0}
+        return {"sm_mhz": statistics.median(self.samples), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def load_workload(name: str, rank: int = 0):
+    """BASELINE config `name`; rank r > 0 matches its own query batch (query seed + 7919 r)."""
+    import tmgen
+    c = dict(tmgen.CONFIGS[name])
+    wl = tmgen.generate(c["n_sets"], c["n_queries"], c["seed"], total_tags=c["total_tags"],
+                        max_partition=c["max_partition"], name=name,
+                        query_seed=c["seed"] + (1 << 32) + 7919 * rank)
+    return wl, c
+
+
+# ------------------------------------------------------------------ oracle --
+def oracle_rate(wl, c, unique: bool, target_s: float = 8.0, max_q: int | None = None):
+    """O2 (the paper's CPU method: Alg. 1 + Alg. 2 + linear scan, std threads)
+    on a bounded query sample sized for ~target_s seconds."""
+    from oracle import o2
+    db_sig = o2.encode(wl.db)
+    q_sig = o2.encode(wl.queries)
+    t0 = time.perf_counter()
+    ix = o2.Index(db_sig, c["max_partition"])
+    build_s = time.perf_counter() - t0
+    nq = q_sig.shape[0]
+    n = min(nq, 256)
+    t0 = time.perf_counter()
+    ix.match(wl.key_off, wl.keys, q_sig[:n], unique)
+    dt = max(time.perf_counter() - t0, 1e-6)
+    per_q = dt / n
+    size = int(min(nq, max(256, target_s / per_q)))
+    if max_q:
+        size = min(size, max_q)
+    return ix, q_sig, size, build_s
+
+
+def run_reference(args):
+    """--impl reference: the oracle as it stands, rank 0 only."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle import o2
+    wl, c = load_workload(args.config)
+    unique = bool(args.unique)
+    ix, q_sig, size, build_s = oracle_rate(wl, c, unique, target_s=args.ref_step_s)
+    rng = np.random.default_rng(0)
+    times = []
+    for step in range(args.warmup + args.steps):
+        sel = np.sort(rng.choice(q_sig.shape[0], size, replace=False))
+        t0 = time.perf_counter()
+        ix.match(wl.key_off, wl.keys, q_sig[sel], unique, qid=sel.astype(np.uint32))
+        dt = time.perf_counter() - t0
+        if step >= args.warmup:
+            times.append(dt)
+    tot = sum(times)
+    value = size * len(times) / tot
+    cores = o2.threads(0)
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * tot / len(times),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)",
+            "config": config_block(c, args, wl),
+            "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
+                             "sample": f"{size} of {q_sig.shape[0]} queries per step (O2: Alg.1 MAX_P="
+                                       f"{c['max_partition']} + Alg.2 + linear scan; Alg.1 build {build_s:.1f} s "
+                                       f"excluded)"},
+            "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def config_block(c, args, wl):
+    return {"workload": args.config, "n_sets": c["n_sets"], "n_queries": c["n_queries"],
+            "query_tags": "base set + 2..4 extra" if not c["total_tags"] else f"total {c['total_tags']}",
+            "max_partition": c["max_partition"], "mode": "match-unique" if args.unique else "match",
+            "tile_filter": ["alg4-prefix", "tile-and", "none"][args.tile_filter],
+            "parallelism": f"replicated-dp{args.gpus}" if args.gpus > 1 else "single",
+            "l2": "flushed between timed steps (512 MiB write)", "bloom": "192 bits, k=7 (PAPER.md:106)"}
+
+
+# --------------------------------------------------------------------- ours --
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    dev = torch.cuda.current_device()
+
+    import __graft_entry__
+    __graft_entry__.build() if rank == 0 or world == 1 else None
+    if world > 1:
+        dist.barrier()
+    import paper_conf_eurosys_rogorapkmcc17_b200 as tmb
+
+    wl, c = load_workload(args.config, rank)
+    unique = bool(args.unique)
+    Q = wl.queries.n_sets
+    t0 = time.perf_counter()
+    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], device=dev,
+                      tile_filter=args.tile_filter)
+    build_s = time.perf_counter() - t0
+
+    # device-resident query batch (value) and pinned host copy (e2e)
+    qarr = [np.ascontiguousarray(a) for a in (wl.queries.vocab_bytes, wl.queries.vocab_off.view(np.int64),
+                                              wl.queries.tag_idx.view(np.int32), wl.queries.set_off.view(np.int64))]
+    dt_ = [torch.from_numpy(a).to(f"cuda:{dev}") for a in qarr]
+    dq = tmb.device_tagsets(dt_[0].data_ptr(), dt_[1].data_ptr(), dt_[2].data_ptr(), dt_[3].data_ptr(),
+                            qarr[0].size, qarr[1].size - 1, qarr[2].size, Q)
+    pinned = [torch.from_numpy(a).pin_memory() for a in qarr]
+    hq = tmb.HostTagSets(pinned[0].numpy(), pinned[1].numpy().view(np.uint64), pinned[2].numpy().view(np.uint32),
+                         pinned[3].numpy().view(np.uint64))
+    h2d_bytes = sum(a.nbytes for a in qarr)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=f"cuda:{dev}")
+    stream = torch.cuda.current_stream()
+
+    def step_device():
+        return db.match_batch_device(dq, unique, stream.cuda_stream)
+
+    for _ in range(args.warmup):
+        step_device()
+        p = db.match_batch_raw(hq, unique)
+        db.free_pairs(p)
+    torch.cuda.synchronize()
+
+    # ---- value: device-resident inputs, per-step CUDA events, L2 flushed between steps
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    launches, scan_ms, stats = 0, [], []
+    sampler = ClockSampler(dev)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    with sampler:
+        for i in range(args.steps):
+            flush.zero_()
+            ev[i][0].record(stream)
+            out = step_device()
+            ev[i][1].record(stream)
+            st = db.stats()
+            launches += st["kernel_launches"]
+            scan_ms.append(st["scan_ms"])
+            stats.append(st)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    t_local = sum(step_ms) / 1000.0
+    t_max = t_local
+    if world > 1:
+        t = torch.tensor([t_local], device=f"cuda:{dev}", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t_max = float(t.item())
+    value = world * Q * args.steps / t_max
+
+    # ---- e2e: host API, pinned inputs, H2D + D2H inside the timed region
+    e2e_t, d2h = [], 0
+    for i in range(args.steps):
+        flush.zero_()
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        p = db.match_batch_raw(hq, unique)
+        e2e_t.append(time.perf_counter() - t0)
+        d2h = p.n * 8 + 8 * 2
+        db.free_pairs(p)
+    e2e_local = sum(e2e_t)
+    if world > 1:
+        t = torch.tensor([e2e_local], device=f"cuda:{dev}", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_local = float(t.item())
+    e2e_value = world * Q * args.steps / e2e_local
+
+    if rank == 0:
+        peaks, peak_src = measured_peaks()
+        last = stats[-1]
+        ops = OPS_PER_TILE_TEST * last["tile_tests"] + OPS_PER_PAIR_CHECK * last["pair_checks"]
+        scan_s = statistics.mean(scan_ms) / 1000.0
+        peak_tops = SM_COUNT * ALU_LANES_PER_SM_CLK * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+        achieved = ops / scan_s / 1e12
+        traffic = None
+        try:
+            with open(os.path.join(ROOT, "profiles", "ncu_scan_traffic.json")) as f:
+                tr = json.load(f)
+                if tr.get("config") == args.config:
+                    traffic = tr.get("dram_bytes_per_launch")
+        except Exception:
+            pass
+        line = {
+            "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": statistics.mean(step_ms), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)",
+            "config": config_block(c, args, wl),
+            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
+                         "frac": achieved / peak_tops, "traffic": traffic,
+                         "kernel": "k_scan", "kernel_ms": statistics.mean(scan_ms),
+                         "kernel_share_of_step": statistics.mean(scan_ms) / statistics.mean(step_ms),
+                         "ops_per_launch": ops,
+                         "peak_src": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM_CLK} ALU lanes/clk x "
+                                     f"{peaks.get('sm_max_mhz', 1965.0)} MHz ({peak_src} sm_max_mhz)"},
+            "e2e": {"value": e2e_value, "unit": "queries/s", "h2d_bytes_per_step": h2d_bytes,
+                    "d2h_bytes_per_step": d2h},
+            "gpu_launches": launches,
+            "clocks": sampler.summary(),
+            "stages_ms": {k: statistics.mean(s[k] for s in stats) for k in
+                          ("encode_ms", "route_ms", "scan_ms", "merge_ms", "total_ms")},
+            "path_stats": {k: last[k] for k in ("n_partitions", "routed", "candidate_pairs", "tile_tests",
+                                                "pair_checks", "matched_sets", "emitted_pairs", "result_pairs",
+                                                "work_items")},
+            "build_s": build_s,
+        }
+        if not args.no_cpu_baseline and world == 1:
+            from oracle import o2
+            ix, q_sig, size, obuild = oracle_rate(wl, c, unique, target_s=args.cpu_s)
+            sel = np.sort(np.random.default_rng(1).choice(q_sig.shape[0], size, replace=False))
+            t0 = time.perf_counter()
+            ix.match(wl.key_off, wl.keys, q_sig[sel], unique, qid=sel.astype(np.uint32))
+            dt = time.perf_counter() - t0
+            line["cpu_baseline"] = {"value": size / dt, "unit": "queries/s", "cores": o2.threads(0),
+                                    "kind": "oracle",
+                                    "sample": f"{size} of {Q} queries (O2: Alg.1 MAX_P={c['max_partition']} + "
+                                              f"Alg.2 + linear scan, {o2.threads(0)} threads; Alg.1 build "
+                                              f"{obuild:.1f} s excluded)"}
+        print(json.dumps(line), flush=True)
+    db.close()
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--unique", action="store_true", help="match-unique instead of match")
+    ap.add_argument("--tile-filter", type=int, default=0, choices=[0, 1, 2])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-s", type=float, default=10.0, help="seconds of oracle work for cpu_baseline")
+    ap.add_argument("--ref-step-s", type=float, default=8.0, help="seconds per --impl reference step")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

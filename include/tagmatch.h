@@ -1,0 +1,215 @@
+/*
+ * tagmatch.h -- C ABI of the B200-native TagMatch subset-matching library.
+ *
+ * The library implements the data-parallel hot path of TagMatch (Rogora et al.,
+ * "High-Throughput Subset Matching on Commodity GPU-Based Systems", EuroSys'17;
+ * cited as PAPER.md:<line>):
+ *
+ *   tm_build        add-set(set, key)* followed by consolidate()  (Table 2)
+ *                   = Bloom encoding + Algorithm 1 balanced
+ *                   partitioning + lexicographic order
+ *                   inside partitions + key table.
+ *   tm_match_batch  match / match-unique of a batch of query sets
+ *                   (Table 2): encode, route to
+ *                   every partition whose mask is a subset of the query
+ *                   (Algorithm 2), per-partition batches
+ *                   (PAPER.md:144), tile prefix pre-filter (Algorithm 4,
+ *                   PAPER.md:164-198), subset check sig(s) & ~sig(q) == 0
+ *                   (Algorithm 3), compaction,
+ *                   set-id -> key lookup and merge
+ *                   (PAPER.md:236).  Every step runs in the library's CUDA
+ *                   kernels on one B200 (sm_100a); there is no CPU fallback.
+ *   tm_free         release a database.
+ *
+ * Result semantics (readings R10-R13): entry i of the
+ * database is (set i, key) for every key in set i's key list.  For query j the
+ * result holds (j, key) for every entry whose Bloom signature is a bitwise
+ * subset of sig(q_j) -- Bloom false positives included --
+ * once per matching entry (match) or once per distinct key (match-unique).
+ * Pairs are returned sorted ascending by (query, key).
+ *
+ * Conventions for every call:
+ *   - return TM_OK (0) on success or a negative tm_status; no exception or
+ *     longjmp crosses the ABI; tm_last_error() gives a human-readable detail
+ *     for the calling thread's last failure;
+ *   - input arrays are borrowed for the duration of the call only, never
+ *     retained and never written;
+ *   - outputs are written only on TM_OK;
+ *   - a tm_db handle is not re-entrant: serialize calls per handle (different
+ *     handles may be used concurrently from different threads).
+ */
+#ifndef TAGMATCH_H
+#define TAGMATCH_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define TM_ABI_VERSION 1u
+/* Bloom filter width and number of hash functions. */
+#define TM_SIG_BITS 192u
+#define TM_SIG_WORDS 3u
+#define TM_NUM_HASHES 7u
+/* Default MAX_P (best throughput around 200K sets per partition). */
+#define TM_DEFAULT_MAX_PARTITION 200000u
+/* max_partition value meaning "no partitioning": one partition with the empty
+ * mask, routed to every query (reading R8; BASELINE config C1). */
+#define TM_NO_PARTITIONING 0xFFFFFFFFu
+
+typedef struct tm_db tm_db; /* opaque, owned by the library */
+
+typedef enum {
+    TM_OK = 0,
+    TM_EINVAL = -1, /* NULL pointer, non-monotone / out-of-range offsets, bad flag   */
+    TM_ENOMEM = -2, /* host or device allocation failed                            */
+    TM_ECUDA = -3,  /* CUDA runtime error (also: no CUDA device / no sm_100 device)  */
+    TM_ENCCL = -4,  /* NCCL error (sharded mode)                                    */
+    TM_ERANGE = -5, /* more than 2^32-1 sets, keys, tags or queries                 */
+    TM_ESTATE = -6  /* call not valid in the handle's state                        */
+} tm_status;
+
+/*
+ * A batch of tag sets in interned CSR form (tags are byte strings,
+ * PAPER.md:80 "sets of string tags"; case-sensitive, any bytes, no NUL needed).
+ *
+ *   vocabulary string v = vocab_bytes[vocab_off[v] .. vocab_off[v+1])
+ *   set i               = { string tag_idx[t] : set_off[i] <= t < set_off[i+1] }
+ *
+ * If tag_idx is NULL, tag t is vocabulary string t (n_tags == n_vocab).
+ * Repeated tags in a set are allowed (a set is a set: they do not change its
+ * signature).  Sizes are given explicitly so the same struct can describe
+ * device-resident arrays (tm_match_batch_device):
+ *   n_bytes = vocab_off[n_vocab], n_tags = set_off[n_sets], set_off[0] = 0,
+ * offsets non-decreasing, tag_idx[t] < n_vocab.  Host calls validate all of
+ * this (TM_EINVAL); device calls validate only what is checkable on the host.
+ */
+typedef struct {
+    const uint8_t *vocab_bytes; /* n_bytes bytes (may be NULL if n_bytes == 0)  */
+    const uint64_t *vocab_off;  /* n_vocab + 1 byte offsets                      */
+    const uint32_t *tag_idx;    /* n_tags vocabulary indices, or NULL (identity) */
+    const uint64_t *set_off;    /* n_sets + 1 offsets into the tag list          */
+    uint64_t n_bytes;
+    uint64_t n_vocab;
+    uint64_t n_tags;
+    uint64_t n_sets;
+} tm_tagsets;
+
+typedef struct {
+    uint32_t max_partition; /* MAX_P; 0 -> TM_DEFAULT_MAX_PARTITION;
+                               TM_NO_PARTITIONING -> one empty-mask partition        */
+    int32_t device;         /* CUDA device ordinal; -1 -> the calling thread's current */
+    uint32_t n_shards;      /* 0/1: this handle holds every partition; k > 1: it holds
+                               only the partitions assigned to `shard` (sec. "Shards") */
+    uint32_t shard;         /* 0 <= shard < n_shards                                   */
+    uint32_t tile_filter;   /* 0 = Alg. 4 common prefix of each 32-set tile (default);
+                               1 = AND of the tile's signatures (lossless strengthening);
+                               2 = no pre-filter (plain Alg. 3 scan)                   */
+    uint32_t reserved[3];   /* must be 0                                               */
+} tm_config;
+
+/* Result pairs in host memory, allocated by the library (pinned), released by
+ * tm_pairs_free().  query[i] is a 0-based index into the call's query batch. */
+typedef struct {
+    uint64_t n;
+    uint32_t *query;
+    uint32_t *key;
+    void *priv_; /* library bookkeeping; do not touch */
+} tm_pairs;
+
+/* Result pairs in device memory owned by the tm_db; valid until the next call
+ * on the same handle or tm_free. */
+typedef struct {
+    uint64_t n;
+    uint32_t *query; /* device pointer */
+    uint32_t *key;   /* device pointer */
+} tm_dev_pairs;
+
+/* Build the database from n_sets tag sets with their keys (add-set* +
+ * consolidate).
+ *   sets    : host arrays, see tm_tagsets.
+ *   key_off : host, n_sets + 1 non-decreasing offsets into keys (key_off[0] = 0)
+ *             -- set i's keys are keys[key_off[i] .. key_off[i+1]) -- or NULL,
+ *             meaning exactly one key per set, keys[i] (add-set semantics).
+ *   keys    : host, uint32 keys ("a link to application data").
+ *   cfg     : may be NULL (all defaults).
+ *   out     : receives the new handle on TM_OK.
+ * Sets with identical signatures share one row of the tagset table; their key
+ * lists are concatenated (multiplicity kept; reading R10).
+ * Errors: TM_EINVAL (NULL / inconsistent arrays, bad cfg), TM_ERANGE (more than
+ * 2^32-1 sets, keys or queries), TM_ECUDA, TM_ENOMEM. */
+tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys, const tm_config *cfg,
+                   tm_db **out);
+
+/* match (unique = 0) or match-unique (unique = 1) of a batch of queries
+ * (PAPER.md:94).  queries: host arrays.  On TM_OK *out owns the sorted pairs
+ * (release with tm_pairs_free).  The call copies the queries to the GPU, runs
+ * the whole path on the handle's stream, and copies the pairs back.
+ * Errors: TM_EINVAL, TM_ERANGE, TM_ECUDA, TM_ENOMEM. */
+tm_status tm_match_batch(tm_db *db, const tm_tagsets *queries, int unique, tm_pairs *out);
+
+/* Same as tm_match_batch with the query arrays already resident in device
+ * memory of the handle's device (pointers in *queries are device pointers;
+ * the struct itself is host memory) and the result left in device memory.
+ * stream: a cudaStream_t to run on, or NULL for the handle's own stream.
+ * The call returns after the pair count is known (it synchronizes the stream). */
+tm_status tm_match_batch_device(tm_db *db, const tm_tagsets *queries, int unique, tm_dev_pairs *out,
+                                void *stream);
+
+void tm_pairs_free(tm_pairs *p); /* NULL-safe; resets *p */
+void tm_free(tm_db *db);         /* NULL-safe */
+const char *tm_strerror(tm_status s);
+const char *tm_last_error(void); /* thread-local detail of the last failure ("" if none) */
+uint32_t tm_abi_version(void);
+
+/* ---------------------------------------------------------- test hooks --- */
+
+/* Bloom signatures of host tag sets computed on `device` (-1 = current):
+ * sig_out (host) receives n_sets * 3 uint64 words, set i at [3i, 3i+3), with
+ * position p (0..191) in word p>>6 at bit 63-(p&63) (reading R3).
+ * The hash is DESIGN.md reading R1: FNV-1a-64 of the tag bytes, then the
+ * first 7 SplitMix64 outputs seeded with it, each mapped to floor(z*192/2^64). */
+tm_status tm_encode(const tm_tagsets *sets, uint64_t *sig_out, int device);
+
+typedef struct {
+    /* database (tm_build) */
+    uint64_t n_sets;       /* input sets                                    */
+    uint64_t n_entries;    /* (set, key) entries = keys                      */
+    uint64_t n_unique;     /* distinct signatures = rows holding a set       */
+    uint64_t n_rows;       /* rows incl. padding (each partition padded to 32) */
+    uint64_t n_partitions; /* partitions held by this handle                 */
+    uint64_t n_partitions_total; /* partitions of the whole database (all shards) */
+    double build_ms;
+    /* last match call */
+    uint64_t n_queries;
+    uint64_t routed;           /* (query, partition) pairs forwarded by Alg. 2       */
+    uint64_t candidate_pairs;  /* sum over routed (q, p) of |P| (pairs Alg. 3 covers) */
+    uint64_t tile_tests;       /* (32-set tile, query) pre-filter tests (Alg. 4)     */
+    uint64_t pair_checks;      /* (set, query) subset checks after the pre-filter    */
+    uint64_t matched_sets;     /* (set, query) matches                               */
+    uint64_t emitted_pairs;    /* (query, key) pairs before merge                    */
+    uint64_t result_pairs;     /* pairs returned                                     */
+    uint64_t work_items;       /* (partition, set range, query chunk) items          */
+    uint64_t retries;          /* capacity-overflow re-runs in the last call          */
+    double encode_ms, route_ms, scan_ms, merge_ms, total_ms; /* CUDA-event stage times */
+    uint32_t scan_launches;    /* scan-kernel launches in the last call               */
+    uint32_t kernel_launches;  /* all library kernel launches in the last call (incl. CUB) */
+} tm_stats_t;
+
+tm_status tm_stats(const tm_db *db, tm_stats_t *out);
+
+/* Partition table of the handle in Algorithm 1's acceptance order
+ * (FIFO work queue).  masks: n_partitions*3 words (layout as
+ * tm_encode); sizes: n_partitions set counts (distinct signatures); either
+ * may be NULL.  n_partitions via tm_stats. */
+tm_status tm_partitions(const tm_db *db, uint64_t *masks, uint64_t *sizes);
+
+/* Signatures (layout as tm_encode) of the distinct sets of partition p in
+ * the tagset table's order (lexicographic). sig_out: sizes[p]*3. */
+tm_status tm_partition_sigs(const tm_db *db, uint64_t p, uint64_t *sig_out);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* TAGMATCH_H */

@@ -1,0 +1,880 @@
+// tm_api.cu -- the C ABI (include/tagmatch.h): tm_build, tm_match_batch, tm_free, hooks.
+//
+// Host code only orchestrates: it validates arguments, owns device buffers and
+// the stream, launches the stage kernels (tm_kernels.cu) and reads back one
+// small counter block per call.  Every step of the matching path runs on the GPU.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstddef>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <mutex>
+#include <new>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "tm_internal.h"
+
+namespace tmb {
+
+static thread_local std::string g_err;
+void set_error(const std::string &msg) { g_err = msg; }
+
+namespace {
+
+struct CudaFail {
+    cudaError_t e;
+    const char *what;
+    int line;
+};
+
+#define TMCK(call)                                                       \
+    do {                                                                 \
+        cudaError_t _e = (call);                                         \
+        if (_e != cudaSuccess) throw ::tmb::CudaFail{_e, #call, __LINE__}; \
+    } while (0)
+
+struct StatusFail {
+    tm_status s;
+    std::string msg;
+};
+
+[[noreturn]] void fail(tm_status s, const std::string &m) { throw StatusFail{s, m}; }
+
+struct DevBuf {
+    void *p = nullptr;
+    size_t cap = 0;
+    template <class T>
+    T *as() const { return static_cast<T *>(p); }
+    // grows (never shrinks); the caller guarantees the stream is idle w.r.t. the old contents
+    void ensure(size_t bytes) {
+        if (bytes <= cap) return;
+        if (p) TMCK(cudaFree(p));
+        p = nullptr;
+        cap = 0;
+        size_t want = std::max<size_t>(bytes + bytes / 4, 256);
+        cudaError_t e = cudaMalloc(&p, want);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            p = nullptr;
+            if (e == cudaErrorMemoryAllocation) fail(TM_ENOMEM, "device allocation of " + std::to_string(want) + " bytes failed");
+            throw CudaFail{e, "cudaMalloc", __LINE__};
+        }
+        cap = want;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        cap = 0;
+    }
+};
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        cudaGetDevice(&prev);
+        if (dev >= 0 && dev != prev) TMCK(cudaSetDevice(dev));
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+// -------------------------------------------- pinned host result blocks --
+struct PinnedBlock {
+    void *p;
+    size_t cap;
+};
+std::mutex g_pin_mu;
+std::multimap<size_t, void *> g_pin_cache;
+size_t g_pin_cached = 0;
+
+PinnedBlock *pinned_get(size_t bytes) {
+    {
+        std::lock_guard<std::mutex> lk(g_pin_mu);
+        auto it = g_pin_cache.lower_bound(bytes);
+        if (it != g_pin_cache.end() && it->first <= 2 * bytes + (1 << 20)) {
+            PinnedBlock *b = new PinnedBlock{it->second, it->first};
+            g_pin_cached -= it->first;
+            g_pin_cache.erase(it);
+            return b;
+        }
+    }
+    void *p = nullptr;
+    size_t cap = std::max<size_t>(bytes, 4096);
+    cudaError_t e = cudaMallocHost(&p, cap);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        fail(TM_ENOMEM, "pinned host allocation failed");
+    }
+    return new PinnedBlock{p, cap};
+}
+
+void pinned_put(PinnedBlock *b) {
+    if (!b) return;
+    {
+        std::lock_guard<std::mutex> lk(g_pin_mu);
+        if (g_pin_cached + b->cap <= (size_t(4) << 30)) {
+            g_pin_cache.emplace(b->cap, b->p);
+            g_pin_cached += b->cap;
+            delete b;
+            return;
+        }
+    }
+    cudaFreeHost(b->p);
+    delete b;
+}
+
+// ------------------------------------------------------------ validation --
+void check_tagsets_host(const tm_tagsets *t, const char *what) {
+    const std::string w(what);
+    if (!t) fail(TM_EINVAL, w + ": NULL tagsets");
+    if (t->n_sets > 0xFFFFFFFFull) fail(TM_ERANGE, w + ": more than 2^32-1 sets");
+    if (!t->set_off) fail(TM_EINVAL, w + ": set_off is NULL");
+    if (t->n_vocab > 0 && !t->vocab_off) fail(TM_EINVAL, w + ": vocab_off is NULL");
+    if (t->n_bytes > 0 && !t->vocab_bytes) fail(TM_EINVAL, w + ": vocab_bytes is NULL");
+    if (t->n_tags > 0 && t->tag_idx == nullptr && t->n_tags != t->n_vocab)
+        fail(TM_EINVAL, w + ": tag_idx NULL requires n_tags == n_vocab");
+    if (t->n_vocab > 0xFFFFFFFFull) fail(TM_ERANGE, w + ": more than 2^32-1 vocabulary strings");
+    if (t->set_off[0] != 0 || t->set_off[t->n_sets] != t->n_tags) fail(TM_EINVAL, w + ": set_off[0] != 0 or set_off[n_sets] != n_tags");
+    for (uint64_t i = 0; i < t->n_sets; ++i)
+        if (t->set_off[i + 1] < t->set_off[i]) fail(TM_EINVAL, w + ": set_off not non-decreasing");
+    if (t->n_vocab > 0) {
+        if (t->vocab_off[0] != 0 || t->vocab_off[t->n_vocab] != t->n_bytes)
+            fail(TM_EINVAL, w + ": vocab_off[0] != 0 or vocab_off[n_vocab] != n_bytes");
+        for (uint64_t i = 0; i < t->n_vocab; ++i)
+            if (t->vocab_off[i + 1] < t->vocab_off[i]) fail(TM_EINVAL, w + ": vocab_off not non-decreasing");
+    } else if (t->n_tags > 0) {
+        fail(TM_EINVAL, w + ": tags without a vocabulary");
+    }
+    if (t->tag_idx)
+        for (uint64_t i = 0; i < t->n_tags; ++i)
+            if (t->tag_idx[i] >= t->n_vocab) fail(TM_EINVAL, w + ": tag_idx out of range");
+}
+
+void check_tagsets_device(const tm_tagsets *t) {
+    if (!t) fail(TM_EINVAL, "queries: NULL tagsets");
+    if (t->n_sets > 0xFFFFFFFFull) fail(TM_ERANGE, "queries: more than 2^32-1 sets");
+    if (t->n_sets > 0 && !t->set_off) fail(TM_EINVAL, "queries: set_off is NULL");
+    if (t->n_vocab > 0 && !t->vocab_off) fail(TM_EINVAL, "queries: vocab_off is NULL");
+    if (t->n_bytes > 0 && !t->vocab_bytes) fail(TM_EINVAL, "queries: vocab_bytes is NULL");
+    if (t->n_tags > 0 && t->tag_idx == nullptr && t->n_tags != t->n_vocab)
+        fail(TM_EINVAL, "queries: tag_idx NULL requires n_tags == n_vocab");
+    if (t->n_tags > 0 && t->n_vocab == 0) fail(TM_EINVAL, "queries: tags without a vocabulary");
+}
+
+int bits_for(uint64_t n) {  // bits needed to represent values < n
+    int b = 0;
+    while (b < 64 && (1ULL << b) < n) ++b;
+    return b;
+}
+
+}  // namespace
+}  // namespace tmb
+
+using namespace tmb;
+
+// ================================================================== tm_db ==
+struct tm_db {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    cudaEvent_t ev[6] = {};
+    tm_config cfg{};
+    int scan_grid = 0;
+    // database (device)
+    uint64_t n_sets = 0, n_entries = 0, n_unique = 0, n_rows = 0, n_parts = 0, n_parts_total = 0;
+    DevBuf planes;   // 3 x rows u64
+    DevBuf key_off;  // rows + 1 u32
+    DevBuf keys;     // K u32
+    DevBuf masks;    // P x 3 u64
+    DevBuf part_row; // P + 1 u32
+    DevBuf part_n;   // P u32
+    std::vector<uint64_t> h_masks, h_sizes;
+    std::vector<uint32_t> h_part_row;
+    double build_ms = 0;
+    // per-call workspace
+    DevBuf in_bytes, in_voff, in_tidx, in_soff;  // host-API staging of the queries
+    DevBuf vsig, qplanes, bm, word_off, qidx, qoff, item_cnt, item_off, out, out_alt, res_q, res_k, tmp, ctr;
+    DevCounters *h_ctr = nullptr;  // pinned
+    unsigned long long *h_nuniq = nullptr;
+    unsigned long long cap_qidx = 0, cap_out = 0;
+    tm_stats_t st{};
+};
+
+namespace tmb {
+namespace {
+
+void *cub_tmp(tm_db *db, size_t bytes) {
+    db->tmp.ensure(bytes);
+    return db->tmp.p;
+}
+
+// Run the whole path for device-resident queries; leaves n results in db->res_q/res_k.
+uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) {
+    tm_stats_t &st = db->st;
+    const uint64_t Q = q->n_sets;
+    const uint32_t P = (uint32_t)db->n_parts;
+    std::memset(&st.n_queries, 0, sizeof(tm_stats_t) - offsetof(tm_stats_t, n_queries));
+    st.n_queries = Q;
+    if (Q == 0 || P == 0) return 0;
+    const uint64_t QW = (Q + 31) / 32;
+    const uint64_t n_words = (uint64_t)P * QW;
+    uint32_t launches = 0, cub_calls = 0;
+
+    db->ctr.ensure(sizeof(DevCounters));
+    DevCounters *ctr = db->ctr.as<DevCounters>();
+    TMCK(cudaEventRecord(db->ev[0], s));
+
+    // S1: encode
+    db->vsig.ensure(std::max<uint64_t>(q->n_vocab, 1) * 24);
+    db->qplanes.ensure(Q * 24);
+    uint64_t *q0 = db->qplanes.as<uint64_t>(), *q1 = q0 + Q, *q2 = q1 + Q;
+    TMCK(launch_hash_vocab(q->vocab_bytes, q->vocab_off, q->n_vocab, db->vsig.as<uint64_t>(), s));
+    TMCK(launch_encode_sets(db->vsig.as<uint64_t>(), q->tag_idx, q->set_off, Q, q0, q1, q2, s));
+    launches += 2;
+    TMCK(cudaEventRecord(db->ev[1], s));
+
+    // S2: route (bitmap of mask_p subset-of q, scanned to a partition-major CSR)
+    db->bm.ensure(n_words * 4);
+    db->word_off.ensure((n_words + 1) * 8);
+    TMCK(launch_route_bitmap(db->masks.as<uint64_t>(), P, q0, q1, q2, Q, db->bm.as<uint32_t>(), s));
+    launches++;
+    size_t tb = 0;
+    TMCK(cub_exclusive_popc_scan(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words, nullptr, &tb, s));
+    TMCK(cub_exclusive_popc_scan(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words,
+                                 cub_tmp(db, tb), &tb, s));
+    cub_calls++;
+    db->qoff.ensure((uint64_t)(P + 1) * 8);
+    db->item_cnt.ensure((uint64_t)(P + 1) * 8);
+    db->item_off.ensure((uint64_t)(P + 1) * 8);
+    if (db->cap_qidx == 0) db->cap_qidx = std::max<unsigned long long>(Q * 32, 1 << 16);
+    if (db->cap_out == 0) db->cap_out = std::max<unsigned long long>(Q * 32, 1 << 16);
+
+    for (int attempt = 0;; ++attempt) {
+        db->qidx.ensure(db->cap_qidx * 4);
+        db->out.ensure(db->cap_out * 8);
+        TMCK(cudaMemsetAsync(ctr, 0, sizeof(DevCounters), s));
+        TMCK(launch_route_scatter(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words,
+                                  (uint32_t)QW, db->qidx.as<uint32_t>(), db->cap_qidx, s));
+        // S3: per-partition batches -> work items
+        TMCK(launch_items(db->word_off.as<unsigned long long>(), (uint32_t)QW, db->part_row.as<uint32_t>(),
+                          db->part_n.as<uint32_t>(), P, db->qoff.as<unsigned long long>(),
+                          db->item_cnt.as<unsigned long long>(), ctr, s));
+        launches += 2;
+        tb = 0;
+        TMCK(cub_exclusive_scan_u64(db->item_cnt.as<unsigned long long>(), db->item_off.as<unsigned long long>(),
+                                    P + 1, nullptr, &tb, s));
+        TMCK(cub_exclusive_scan_u64(db->item_cnt.as<unsigned long long>(), db->item_off.as<unsigned long long>(),
+                                    P + 1, cub_tmp(db, tb), &tb, s));
+        cub_calls++;
+        TMCK(cudaEventRecord(db->ev[2], s));
+        // S4-S7: subset scan
+        ScanParams sp;
+        sp.w0 = db->planes.as<uint64_t>();
+        sp.w1 = sp.w0 + db->n_rows;
+        sp.w2 = sp.w1 + db->n_rows;
+        sp.key_off = db->key_off.as<uint32_t>();
+        sp.keys = db->keys.as<uint32_t>();
+        sp.part_row = db->part_row.as<uint32_t>();
+        sp.part_n = db->part_n.as<uint32_t>();
+        sp.q0 = q0;
+        sp.q1 = q1;
+        sp.q2 = q2;
+        sp.qidx = db->qidx.as<uint32_t>();
+        sp.qcap = db->cap_qidx;
+        sp.qoff = db->qoff.as<unsigned long long>();
+        sp.item_off = db->item_off.as<unsigned long long>();
+        sp.n_parts = P;
+        sp.out = db->out.as<uint64_t>();
+        sp.cap = db->cap_out;
+        sp.ctr = ctr;
+        sp.filter = db->cfg.tile_filter;
+        TMCK(launch_scan(sp, db->scan_grid, s));
+        launches++;
+        st.scan_launches++;
+        TMCK(cudaEventRecord(db->ev[3], s));
+        TMCK(cudaMemcpyAsync(db->h_ctr, ctr, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+        TMCK(cudaStreamSynchronize(s));
+        const DevCounters c = *db->h_ctr;
+        bool retry = false;
+        if (c.routed > db->cap_qidx) {
+            db->cap_qidx = c.routed + c.routed / 4;
+            retry = true;
+        }
+        if (!retry && c.n_out > db->cap_out) {
+            db->cap_out = c.n_out + c.n_out / 8;
+            retry = true;
+        }
+        if (retry) {
+            st.retries++;
+            if (attempt > 4) fail(TM_ESTATE, "capacity retry loop did not converge");
+            continue;
+        }
+        st.routed = c.routed;
+        st.candidate_pairs = c.candidates;
+        st.tile_tests = c.tile_tests;
+        st.pair_checks = c.pair_checks;
+        st.matched_sets = c.matched_sets;
+        st.emitted_pairs = c.n_out;
+        st.work_items = c.n_items;
+        break;
+    }
+    uint64_t n = st.emitted_pairs;
+    // S8: canonical order (sort by (query, key)), merge (unique for match-unique)
+    db->out_alt.ensure(std::max<uint64_t>(n, 1) * 8);
+    uint64_t *sorted = db->out.as<uint64_t>();
+    if (n > 1) {
+        int sel = 0;
+        const int end_bit = 32 + bits_for(Q);
+        tb = 0;
+        TMCK(cub_sort_keys_u64(db->out.as<uint64_t>(), db->out_alt.as<uint64_t>(), n, end_bit, &sel, nullptr, &tb, s));
+        TMCK(cub_sort_keys_u64(db->out.as<uint64_t>(), db->out_alt.as<uint64_t>(), n, end_bit, &sel,
+                               cub_tmp(db, tb), &tb, s));
+        cub_calls++;
+        sorted = sel ? db->out_alt.as<uint64_t>() : db->out.as<uint64_t>();
+    }
+    if (unique && n > 1) {
+        uint64_t *dst = (sorted == db->out.as<uint64_t>()) ? db->out_alt.as<uint64_t>() : db->out.as<uint64_t>();
+        unsigned long long *d_n = &ctr->item_ctr;  // reuse a counter slot
+        tb = 0;
+        TMCK(cub_unique_u64(sorted, dst, d_n, n, nullptr, &tb, s));
+        TMCK(cub_unique_u64(sorted, dst, d_n, n, cub_tmp(db, tb), &tb, s));
+        cub_calls++;
+        TMCK(cudaMemcpyAsync(db->h_nuniq, d_n, 8, cudaMemcpyDeviceToHost, s));
+        TMCK(cudaStreamSynchronize(s));
+        n = *db->h_nuniq;
+        sorted = dst;
+    }
+    db->res_q.ensure(std::max<uint64_t>(n, 1) * 4);
+    db->res_k.ensure(std::max<uint64_t>(n, 1) * 4);
+    TMCK(launch_split(sorted, n, db->res_q.as<uint32_t>(), db->res_k.as<uint32_t>(), s));
+    launches++;
+    TMCK(cudaEventRecord(db->ev[4], s));
+    st.result_pairs = n;
+    st.kernel_launches = launches;
+    (void)cub_calls;
+    return n;
+}
+
+void finish_timing(tm_db *db, cudaStream_t s) {
+    TMCK(cudaStreamSynchronize(s));
+    float ms = 0;
+    tm_stats_t &st = db->st;
+    if (st.n_queries == 0 || db->n_parts == 0) return;
+    TMCK(cudaEventElapsedTime(&ms, db->ev[0], db->ev[1]));
+    st.encode_ms = ms;
+    TMCK(cudaEventElapsedTime(&ms, db->ev[1], db->ev[2]));
+    st.route_ms = ms;
+    TMCK(cudaEventElapsedTime(&ms, db->ev[2], db->ev[3]));
+    st.scan_ms = ms;
+    TMCK(cudaEventElapsedTime(&ms, db->ev[3], db->ev[4]));
+    st.merge_ms = ms;
+    TMCK(cudaEventElapsedTime(&ms, db->ev[0], db->ev[4]));
+    st.total_ms = ms;
+}
+
+tm_status translate(const CudaFail &f) {
+    char buf[512];
+    snprintf(buf, sizeof buf, "CUDA error %d (%s) at tm_api.cu:%d in %s", (int)f.e, cudaGetErrorString(f.e), f.line,
+             f.what);
+    set_error(buf);
+    cudaGetLastError();
+    if (f.e == cudaErrorMemoryAllocation) return TM_ENOMEM;
+    return TM_ECUDA;
+}
+
+// Partition -> shard assignment (n_shards > 1): greedy longest-processing-time
+// over the estimated work |P| * 4^-|mask| (routing probability of a mask of
+// |mask| bits for queries with one-bit density ~1/4), ties by partition id.
+std::vector<uint32_t> assign_shards(const std::vector<Partition> &parts, uint32_t n_shards) {
+    std::vector<uint32_t> owner(parts.size(), 0);
+    if (n_shards <= 1) return owner;
+    std::vector<double> w(parts.size());
+    for (size_t i = 0; i < parts.size(); ++i) {
+        int pc = __builtin_popcountll(parts[i].mask.w[0]) + __builtin_popcountll(parts[i].mask.w[1]) +
+                 __builtin_popcountll(parts[i].mask.w[2]);
+        w[i] = (double)(parts[i].end - parts[i].begin) * std::pow(0.25, pc);
+    }
+    std::vector<uint32_t> ord(parts.size());
+    std::iota(ord.begin(), ord.end(), 0u);
+    std::stable_sort(ord.begin(), ord.end(), [&](uint32_t a, uint32_t b) { return w[a] > w[b]; });
+    std::vector<double> load(n_shards, 0.0);
+    for (uint32_t i : ord) {
+        uint32_t best = 0;
+        for (uint32_t s = 1; s < n_shards; ++s)
+            if (load[s] < load[best]) best = s;
+        owner[i] = best;
+        load[best] += w[i];
+    }
+    return owner;
+}
+
+void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys) {
+    auto t0 = std::chrono::steady_clock::now();
+    cudaStream_t s = db->stream;
+    const uint64_t N = sets->n_sets;
+    // keys
+    std::vector<uint64_t> koff_default;
+    if (!key_off) {
+        koff_default.resize(N + 1);
+        for (uint64_t i = 0; i <= N; ++i) koff_default[i] = i;
+        key_off = koff_default.data();
+    } else {
+        if (key_off[0] != 0) fail(TM_EINVAL, "key_off[0] != 0");
+        for (uint64_t i = 0; i < N; ++i)
+            if (key_off[i + 1] < key_off[i]) fail(TM_EINVAL, "key_off not non-decreasing");
+    }
+    const uint64_t K = key_off[N];
+    if (K > 0xFFFFFFFFull) fail(TM_ERANGE, "more than 2^32-1 keys");
+    if (K > 0 && !keys) fail(TM_EINVAL, "keys is NULL");
+    db->n_sets = N;
+    db->n_entries = K;
+
+    // S0a: encode every set on the GPU
+    DevBuf d_bytes, d_voff, d_tidx, d_soff, d_vsig, d_planes, d_sorted, d_idx, d_idx2, d_key, d_key2;
+    struct Releaser {
+        std::vector<DevBuf *> v;
+        ~Releaser() {
+            for (auto *b : v) b->release();
+        }
+    } rel{{&d_bytes, &d_voff, &d_tidx, &d_soff, &d_vsig, &d_planes, &d_sorted, &d_idx, &d_idx2, &d_key, &d_key2}};
+    std::vector<Sig> usig;            // distinct signatures, lexicographic
+    std::vector<uint64_t> ustart;     // group starts into the sorted entry order
+    std::vector<uint32_t> h_idx(N);   // sorted order of sets
+    if (N > 0) {
+        d_bytes.ensure(std::max<uint64_t>(sets->n_bytes, 1));
+        d_voff.ensure((sets->n_vocab + 1) * 8);
+        d_soff.ensure((N + 1) * 8);
+        if (sets->n_bytes) TMCK(cudaMemcpyAsync(d_bytes.p, sets->vocab_bytes, sets->n_bytes, cudaMemcpyHostToDevice, s));
+        if (sets->n_vocab) TMCK(cudaMemcpyAsync(d_voff.p, sets->vocab_off, (sets->n_vocab + 1) * 8, cudaMemcpyHostToDevice, s));
+        TMCK(cudaMemcpyAsync(d_soff.p, sets->set_off, (N + 1) * 8, cudaMemcpyHostToDevice, s));
+        if (sets->tag_idx && sets->n_tags) {
+            d_tidx.ensure(sets->n_tags * 4);
+            TMCK(cudaMemcpyAsync(d_tidx.p, sets->tag_idx, sets->n_tags * 4, cudaMemcpyHostToDevice, s));
+        }
+        d_vsig.ensure(std::max<uint64_t>(sets->n_vocab, 1) * 24);
+        d_planes.ensure(N * 24);
+        uint64_t *w0 = d_planes.as<uint64_t>(), *w1 = w0 + N, *w2 = w1 + N;
+        TMCK(launch_hash_vocab(d_bytes.as<uint8_t>(), d_voff.as<uint64_t>(), sets->n_vocab, d_vsig.as<uint64_t>(), s));
+        TMCK(launch_encode_sets(d_vsig.as<uint64_t>(), (sets->tag_idx && sets->n_tags) ? d_tidx.as<uint32_t>() : nullptr,
+                                d_soff.as<uint64_t>(), N, w0, w1, w2, s));
+        // S0b: lexicographic sort of the signatures (LSD: word 2, then 1, then 0; stable)
+        d_idx.ensure(N * 4);
+        d_idx2.ensure(N * 4);
+        d_key.ensure(N * 8);
+        d_key2.ensure(N * 8);
+        TMCK(launch_iota(d_idx.as<uint32_t>(), N, s));
+        const uint64_t *planes[3] = {w0, w1, w2};
+        for (int w = 2; w >= 0; --w) {
+            TMCK(launch_gather_u64(planes[w], d_idx.as<uint32_t>(), N, d_key.as<uint64_t>(), s));
+            size_t tb = 0;
+            TMCK(cub_sort_pairs_u64_u32(d_key.as<uint64_t>(), d_key2.as<uint64_t>(), d_idx.as<uint32_t>(),
+                                        d_idx2.as<uint32_t>(), N, nullptr, &tb, s));
+            TMCK(cub_sort_pairs_u64_u32(d_key.as<uint64_t>(), d_key2.as<uint64_t>(), d_idx.as<uint32_t>(),
+                                        d_idx2.as<uint32_t>(), N, cub_tmp(db, tb), &tb, s));
+            std::swap(d_idx, d_idx2);
+        }
+        d_sorted.ensure(N * 24);
+        uint64_t *s0 = d_sorted.as<uint64_t>(), *s1 = s0 + N, *s2 = s1 + N;
+        TMCK(launch_gather_planes(w0, w1, w2, d_idx.as<uint32_t>(), N, s0, s1, s2, s));
+        std::vector<uint64_t> hs(3 * N);
+        TMCK(cudaMemcpyAsync(hs.data(), d_sorted.p, N * 24, cudaMemcpyDeviceToHost, s));
+        TMCK(cudaMemcpyAsync(h_idx.data(), d_idx.p, N * 4, cudaMemcpyDeviceToHost, s));
+        TMCK(cudaStreamSynchronize(s));
+        // distinct signatures (reading R10: identical signatures share a row)
+        usig.reserve(N);
+        ustart.reserve(N + 1);
+        for (uint64_t i = 0; i < N; ++i) {
+            Sig g{{hs[i], hs[N + i], hs[2 * N + i]}};
+            if (i == 0 || g.w[0] != usig.back().w[0] || g.w[1] != usig.back().w[1] || g.w[2] != usig.back().w[2]) {
+                usig.push_back(g);
+                ustart.push_back(i);
+            }
+        }
+        ustart.push_back(N);
+    }
+    const uint64_t U = usig.size();
+    db->n_unique = U;
+
+    // S0c: Algorithm 1 over the distinct signatures
+    std::vector<uint32_t> order;
+    std::vector<Partition> parts;
+    alg1_partition(usig.data(), U, db->cfg.max_partition, order, parts);
+    db->n_parts_total = parts.size();
+    const std::vector<uint32_t> owner = assign_shards(parts, std::max(1u, db->cfg.n_shards));
+
+    // S0d: layout -- kept partitions in acceptance order, each padded to 32 rows
+    std::vector<uint32_t> keep;
+    for (uint32_t i = 0; i < parts.size(); ++i)
+        if (owner[i] == db->cfg.shard) keep.push_back(i);
+    const uint64_t P = keep.size();
+    uint64_t rows = 0;
+    for (uint32_t i : keep) rows += ((parts[i].end - parts[i].begin) + kTile - 1) / kTile * kTile;
+    if (rows > 0xFFFFFFF0ull) fail(TM_ERANGE, "more than 2^32 rows");
+    db->n_parts = P;
+    db->n_rows = rows;
+    std::vector<uint64_t> hp(3 * std::max<uint64_t>(rows, 1), ~0ULL);
+    std::vector<uint32_t> hko(rows + 1, 0), hkeys;
+    hkeys.reserve(K);
+    db->h_masks.assign(3 * P, 0);
+    db->h_sizes.assign(P, 0);
+    db->h_part_row.assign(P + 1, 0);
+    std::vector<uint32_t> hpn(std::max<uint64_t>(P, 1), 0);
+    uint64_t r = 0;
+    for (uint64_t pi = 0; pi < P; ++pi) {
+        const Partition &pt = parts[keep[pi]];
+        db->h_part_row[pi] = (uint32_t)r;
+        const uint64_t np = pt.end - pt.begin;
+        db->h_sizes[pi] = np;
+        hpn[pi] = (uint32_t)np;
+        for (int w = 0; w < 3; ++w) db->h_masks[3 * pi + w] = pt.mask.w[w];
+        for (uint64_t m = 0; m < np; ++m, ++r) {
+            const uint32_t u = order[pt.begin + m];
+            hp[r] = usig[u].w[0];
+            hp[rows + r] = usig[u].w[1];
+            hp[2 * rows + r] = usig[u].w[2];
+            for (uint64_t e = ustart[u]; e < ustart[u + 1]; ++e) {  // entries with this signature, set order
+                const uint32_t set = h_idx[e];
+                for (uint64_t k = key_off[set]; k < key_off[set + 1]; ++k) hkeys.push_back(keys[k]);
+            }
+            hko[r + 1] = (uint32_t)hkeys.size();
+        }
+        const uint64_t padded = (np + kTile - 1) / kTile * kTile;
+        for (uint64_t m = np; m < padded; ++m, ++r) hko[r + 1] = (uint32_t)hkeys.size();  // padding rows: no keys
+    }
+    db->h_part_row[P] = (uint32_t)r;
+    db->n_entries = hkeys.size();
+
+    db->planes.ensure(std::max<uint64_t>(rows, 1) * 24);
+    db->key_off.ensure((rows + 1) * 4);
+    db->keys.ensure(std::max<uint64_t>(hkeys.size(), 1) * 4);
+    db->masks.ensure(std::max<uint64_t>(P, 1) * 24);
+    db->part_row.ensure((P + 1) * 4);
+    db->part_n.ensure(std::max<uint64_t>(P, 1) * 4);
+    if (rows) TMCK(cudaMemcpyAsync(db->planes.p, hp.data(), rows * 24, cudaMemcpyHostToDevice, s));
+    TMCK(cudaMemcpyAsync(db->key_off.p, hko.data(), (rows + 1) * 4, cudaMemcpyHostToDevice, s));
+    if (!hkeys.empty()) TMCK(cudaMemcpyAsync(db->keys.p, hkeys.data(), hkeys.size() * 4, cudaMemcpyHostToDevice, s));
+    if (P) {
+        TMCK(cudaMemcpyAsync(db->masks.p, db->h_masks.data(), P * 24, cudaMemcpyHostToDevice, s));
+        TMCK(cudaMemcpyAsync(db->part_n.p, hpn.data(), P * 4, cudaMemcpyHostToDevice, s));
+    }
+    TMCK(cudaMemcpyAsync(db->part_row.p, db->h_part_row.data(), (P + 1) * 4, cudaMemcpyHostToDevice, s));
+    TMCK(cudaStreamSynchronize(s));
+    db->build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+tm_db *new_db(const tm_config *cfg) {
+    tm_db *db = new tm_db();
+    if (cfg) db->cfg = *cfg;
+    if (db->cfg.max_partition == 0) db->cfg.max_partition = TM_DEFAULT_MAX_PARTITION;
+    if (db->cfg.n_shards == 0) db->cfg.n_shards = 1;
+    return db;
+}
+
+void destroy_db(tm_db *db) {
+    if (!db) return;
+    int prev = -1;
+    cudaGetDevice(&prev);
+    cudaSetDevice(db->device);
+    if (db->stream) cudaStreamSynchronize(db->stream);
+    for (DevBuf *b : {&db->planes, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
+                      &db->in_voff, &db->in_tidx, &db->in_soff, &db->vsig, &db->qplanes, &db->bm, &db->word_off,
+                      &db->qidx, &db->qoff, &db->item_cnt, &db->item_off, &db->out, &db->out_alt, &db->res_q,
+                      &db->res_k, &db->tmp, &db->ctr})
+        b->release();
+    for (auto &e : db->ev)
+        if (e) cudaEventDestroy(e);
+    if (db->h_ctr) cudaFreeHost(db->h_ctr);
+    if (db->h_nuniq) cudaFreeHost(db->h_nuniq);
+    if (db->stream) cudaStreamDestroy(db->stream);
+    if (prev >= 0) cudaSetDevice(prev);
+    delete db;
+}
+
+int check_device(int dev) {
+    int n = 0;
+    cudaError_t e = cudaGetDeviceCount(&n);
+    if (e != cudaSuccess || n == 0) {
+        cudaGetLastError();
+        fail(TM_ECUDA, "no CUDA device available (the library has no CPU fallback)");
+    }
+    if (dev < 0) TMCK(cudaGetDevice(&dev));
+    if (dev >= n) fail(TM_EINVAL, "device ordinal out of range");
+    cudaDeviceProp prop;
+    TMCK(cudaGetDeviceProperties(&prop, dev));
+    if (prop.major != 10) fail(TM_ECUDA, std::string("device is not sm_100 (Blackwell B200): ") + prop.name);
+    return dev;
+}
+
+}  // namespace
+}  // namespace tmb
+
+// ==================================================================== ABI ==
+#define TM_API_BEGIN \
+    try {            \
+        tmb::set_error("");
+#define TM_API_END                                                   \
+    }                                                                \
+    catch (const tmb::StatusFail &f) {                                \
+        tmb::set_error(f.msg);                                        \
+        return f.s;                                                  \
+    }                                                                \
+    catch (const tmb::CudaFail &f) {                                  \
+        return tmb::translate(f);                                     \
+    }                                                                \
+    catch (const std::bad_alloc &) {                                 \
+        tmb::set_error("host allocation failed");                    \
+        return TM_ENOMEM;                                            \
+    }                                                                \
+    catch (...) {                                                    \
+        tmb::set_error("unexpected exception");                      \
+        return TM_ESTATE;                                            \
+    }
+
+extern "C" {
+
+uint32_t tm_abi_version(void) { return TM_ABI_VERSION; }
+
+const char *tm_strerror(tm_status s) {
+    switch (s) {
+        case TM_OK: return "ok";
+        case TM_EINVAL: return "invalid argument";
+        case TM_ENOMEM: return "out of memory";
+        case TM_ECUDA: return "CUDA error";
+        case TM_ENCCL: return "NCCL error";
+        case TM_ERANGE: return "size out of range";
+        case TM_ESTATE: return "invalid state";
+    }
+    return "unknown status";
+}
+
+const char *tm_last_error(void) { return tmb::g_err.c_str(); }
+
+tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys, const tm_config *cfg,
+                   tm_db **out) {
+    tm_db *db = nullptr;
+    TM_API_BEGIN
+    if (!out) fail(TM_EINVAL, "out is NULL");
+    check_tagsets_host(sets, "sets");
+    if (cfg) {
+        if (cfg->n_shards > 1 && cfg->shard >= cfg->n_shards) fail(TM_EINVAL, "shard >= n_shards");
+        if (cfg->tile_filter > 2) fail(TM_EINVAL, "tile_filter must be 0, 1 or 2");
+        if (cfg->reserved[0] | cfg->reserved[1] | cfg->reserved[2]) fail(TM_EINVAL, "reserved fields must be 0");
+    }
+    const int dev = check_device(cfg ? cfg->device : -1);
+    DeviceGuard g(dev);
+    db = new_db(cfg);
+    db->device = dev;
+    TMCK(cudaStreamCreateWithFlags(&db->stream, cudaStreamNonBlocking));
+    for (auto &e : db->ev) TMCK(cudaEventCreate(&e));
+    TMCK(cudaMallocHost((void **)&db->h_ctr, sizeof(DevCounters)));
+    TMCK(cudaMallocHost((void **)&db->h_nuniq, 8));
+    db->scan_grid = scan_grid(dev);
+    build_impl(db, sets, key_off, keys);
+    db->st.n_sets = db->n_sets;
+    *out = db;
+    db = nullptr;
+    return TM_OK;
+    }
+    catch (const tmb::StatusFail &f) {
+        tmb::set_error(f.msg);
+        tmb::destroy_db(db);
+        return f.s;
+    }
+    catch (const tmb::CudaFail &f) {
+        tm_status s = tmb::translate(f);
+        tmb::destroy_db(db);
+        return s;
+    }
+    catch (const std::bad_alloc &) {
+        tmb::set_error("host allocation failed");
+        tmb::destroy_db(db);
+        return TM_ENOMEM;
+    }
+    catch (...) {
+        tmb::set_error("unexpected exception");
+        tmb::destroy_db(db);
+        return TM_ESTATE;
+    }
+}
+
+tm_status tm_match_batch(tm_db *db, const tm_tagsets *q, int unique, tm_pairs *out) {
+    TM_API_BEGIN
+    if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
+    if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
+    check_tagsets_host(q, "queries");
+    DeviceGuard g(db->device);
+    cudaStream_t s = db->stream;
+    // one H2D copy of the query batch
+    tm_tagsets dq = *q;
+    dq.vocab_bytes = nullptr;
+    dq.vocab_off = nullptr;
+    db->in_soff.ensure((q->n_sets + 1) * 8);
+    TMCK(cudaMemcpyAsync(db->in_soff.p, q->set_off, (q->n_sets + 1) * 8, cudaMemcpyHostToDevice, s));
+    dq.set_off = db->in_soff.as<uint64_t>();
+    if (q->n_bytes) {
+        db->in_bytes.ensure(q->n_bytes);
+        TMCK(cudaMemcpyAsync(db->in_bytes.p, q->vocab_bytes, q->n_bytes, cudaMemcpyHostToDevice, s));
+        dq.vocab_bytes = db->in_bytes.as<uint8_t>();
+    }
+    if (q->n_vocab) {
+        db->in_voff.ensure((q->n_vocab + 1) * 8);
+        TMCK(cudaMemcpyAsync(db->in_voff.p, q->vocab_off, (q->n_vocab + 1) * 8, cudaMemcpyHostToDevice, s));
+        dq.vocab_off = db->in_voff.as<uint64_t>();
+    }
+    if (q->tag_idx && q->n_tags) {
+        db->in_tidx.ensure(q->n_tags * 4);
+        TMCK(cudaMemcpyAsync(db->in_tidx.p, q->tag_idx, q->n_tags * 4, cudaMemcpyHostToDevice, s));
+        dq.tag_idx = db->in_tidx.as<uint32_t>();
+    } else {
+        dq.tag_idx = nullptr;
+    }
+    const uint64_t n = match_core(db, &dq, unique, s);
+    PinnedBlock *blk = pinned_get(std::max<uint64_t>(n, 1) * 8);
+    uint32_t *hq = static_cast<uint32_t *>(blk->p), *hk = hq + n;
+    if (n) {
+        cudaError_t e1 = cudaMemcpyAsync(hq, db->res_q.p, n * 4, cudaMemcpyDeviceToHost, s);
+        cudaError_t e2 = cudaMemcpyAsync(hk, db->res_k.p, n * 4, cudaMemcpyDeviceToHost, s);
+        if (e1 != cudaSuccess || e2 != cudaSuccess) {
+            pinned_put(blk);
+            throw CudaFail{e1 != cudaSuccess ? e1 : e2, "cudaMemcpyAsync(D2H results)", __LINE__};
+        }
+    }
+    try {
+        finish_timing(db, s);
+    } catch (...) {
+        pinned_put(blk);
+        throw;
+    }
+    out->n = n;
+    out->query = hq;
+    out->key = hk;
+    out->priv_ = blk;
+    return TM_OK;
+    TM_API_END
+}
+
+tm_status tm_match_batch_device(tm_db *db, const tm_tagsets *q, int unique, tm_dev_pairs *out, void *stream) {
+    TM_API_BEGIN
+    if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
+    if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
+    check_tagsets_device(q);
+    DeviceGuard g(db->device);
+    cudaStream_t s = stream ? static_cast<cudaStream_t>(stream) : db->stream;
+    tm_tagsets dq = *q;
+    if (!dq.n_tags) dq.tag_idx = nullptr;
+    const uint64_t n = match_core(db, &dq, unique, s);
+    finish_timing(db, s);
+    out->n = n;
+    out->query = db->res_q.as<uint32_t>();
+    out->key = db->res_k.as<uint32_t>();
+    return TM_OK;
+    TM_API_END
+}
+
+void tm_pairs_free(tm_pairs *p) {
+    if (!p) return;
+    if (p->priv_) tmb::pinned_put(static_cast<tmb::PinnedBlock *>(p->priv_));
+    p->n = 0;
+    p->query = nullptr;
+    p->key = nullptr;
+    p->priv_ = nullptr;
+}
+
+void tm_free(tm_db *db) { tmb::destroy_db(db); }
+
+tm_status tm_encode(const tm_tagsets *sets, uint64_t *sig_out, int device) {
+    TM_API_BEGIN
+    check_tagsets_host(sets, "sets");
+    if (sets->n_sets && !sig_out) fail(TM_EINVAL, "sig_out is NULL");
+    const int dev = check_device(device);
+    DeviceGuard g(dev);
+    const uint64_t N = sets->n_sets;
+    if (!N) return TM_OK;
+    cudaStream_t s;
+    TMCK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    DevBuf b, vo, ti, so, vs, pl;
+    struct Rel {
+        std::vector<DevBuf *> v;
+        cudaStream_t s;
+        ~Rel() {
+            cudaStreamSynchronize(s);
+            for (auto *x : v) x->release();
+            cudaStreamDestroy(s);
+        }
+    } rel{{&b, &vo, &ti, &so, &vs, &pl}, s};
+    b.ensure(std::max<uint64_t>(sets->n_bytes, 1));
+    vo.ensure((sets->n_vocab + 1) * 8);
+    so.ensure((N + 1) * 8);
+    vs.ensure(std::max<uint64_t>(sets->n_vocab, 1) * 24);
+    pl.ensure(N * 24);
+    if (sets->n_bytes) TMCK(cudaMemcpyAsync(b.p, sets->vocab_bytes, sets->n_bytes, cudaMemcpyHostToDevice, s));
+    if (sets->n_vocab) TMCK(cudaMemcpyAsync(vo.p, sets->vocab_off, (sets->n_vocab + 1) * 8, cudaMemcpyHostToDevice, s));
+    TMCK(cudaMemcpyAsync(so.p, sets->set_off, (N + 1) * 8, cudaMemcpyHostToDevice, s));
+    const uint32_t *dti = nullptr;
+    if (sets->tag_idx && sets->n_tags) {
+        ti.ensure(sets->n_tags * 4);
+        TMCK(cudaMemcpyAsync(ti.p, sets->tag_idx, sets->n_tags * 4, cudaMemcpyHostToDevice, s));
+        dti = ti.as<uint32_t>();
+    }
+    uint64_t *w0 = pl.as<uint64_t>(), *w1 = w0 + N, *w2 = w1 + N;
+    TMCK(launch_hash_vocab(b.as<uint8_t>(), vo.as<uint64_t>(), sets->n_vocab, vs.as<uint64_t>(), s));
+    TMCK(launch_encode_sets(vs.as<uint64_t>(), dti, so.as<uint64_t>(), N, w0, w1, w2, s));
+    std::vector<uint64_t> h(3 * N);
+    TMCK(cudaMemcpyAsync(h.data(), pl.p, N * 24, cudaMemcpyDeviceToHost, s));
+    TMCK(cudaStreamSynchronize(s));
+    for (uint64_t i = 0; i < N; ++i) {
+        sig_out[3 * i] = h[i];
+        sig_out[3 * i + 1] = h[N + i];
+        sig_out[3 * i + 2] = h[2 * N + i];
+    }
+    return TM_OK;
+    TM_API_END
+}
+
+tm_status tm_stats(const tm_db *db, tm_stats_t *out) {
+    TM_API_BEGIN
+    if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
+    *out = db->st;
+    out->n_sets = db->n_sets;
+    out->n_entries = db->n_entries;
+    out->n_unique = db->n_unique;
+    out->n_rows = db->n_rows;
+    out->n_partitions = db->n_parts;
+    out->n_partitions_total = db->n_parts_total;
+    out->build_ms = db->build_ms;
+    return TM_OK;
+    TM_API_END
+}
+
+tm_status tm_partitions(const tm_db *db, uint64_t *masks, uint64_t *sizes) {
+    TM_API_BEGIN
+    if (!db) fail(TM_EINVAL, "db is NULL");
+    if (masks && !db->h_masks.empty()) std::memcpy(masks, db->h_masks.data(), db->h_masks.size() * 8);
+    if (sizes && !db->h_sizes.empty()) std::memcpy(sizes, db->h_sizes.data(), db->h_sizes.size() * 8);
+    return TM_OK;
+    TM_API_END
+}
+
+tm_status tm_partition_sigs(const tm_db *db, uint64_t p, uint64_t *sig_out) {
+    TM_API_BEGIN
+    if (!db || !sig_out) fail(TM_EINVAL, "db or sig_out is NULL");
+    if (p >= db->n_parts) fail(TM_EINVAL, "partition index out of range");
+    DeviceGuard g(db->device);
+    const uint64_t r0 = db->h_part_row[p], n = db->h_sizes[p];
+    std::vector<uint64_t> h(3 * n);
+    const uint64_t *d = db->planes.as<uint64_t>();
+    for (int w = 0; w < 3; ++w)
+        if (n) TMCK(cudaMemcpy(h.data() + w * n, d + w * db->n_rows + r0, n * 8, cudaMemcpyDeviceToHost));
+    for (uint64_t i = 0; i < n; ++i)
+        for (int w = 0; w < 3; ++w) sig_out[3 * i + w] = h[w * n + i];
+    return TM_OK;
+    TM_API_END
+}
+
+}  // extern "C"

@@ -1,0 +1,110 @@
+// tm_internal.h -- internal declarations of the TagMatch B200 library (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "tagmatch.h"
+
+namespace tmb {
+
+// ---------------------------------------------------------------- layout --
+// Signatures are 3 x 64-bit words; position p is word p>>6, bit 63-(p&63)
+// (reading R3).  In HBM they live as three SoA planes so that a warp
+// reading 32 consecutive rows issues fully coalesced 256-B loads per plane.
+constexpr int kWords = 3;
+constexpr int kBits = 192;
+constexpr int kHashes = 7;
+constexpr int kTile = 32;  // rows per warp tile (= one warp, Alg. 4 "thread block")
+
+// Scan-kernel geometry.
+constexpr int kScanWarps = 8;      // warps per CTA
+constexpr int kChunk = 1024;       // queries per work item (per-partition batch)
+constexpr int kRangeRows = 2048;   // rows per work item
+
+struct DevCounters {            // zeroed at the start of every match call
+    unsigned long long n_out;   // (q,key) pairs emitted (may exceed capacity)
+    unsigned long long n_items; // work items (written by the work-list kernel)
+    unsigned long long item_ctr;// persistent-kernel work counter
+    unsigned long long tile_tests;
+    unsigned long long pair_checks;
+    unsigned long long matched_sets;
+    unsigned long long routed;      // R = routed (q, p) pairs
+    unsigned long long candidates;  // sum |P| over routed pairs
+};
+
+struct ScanParams {
+    const uint64_t *w0, *w1, *w2;     // db planes [rows]
+    const uint32_t *key_off;          // [rows+1]
+    const uint32_t *keys;             // [K]
+    const uint32_t *part_row;         // [P+1] padded row offsets
+    const uint32_t *part_n;           // [P] real rows
+    const uint64_t *q0, *q1, *q2;     // query planes [Q]
+    const uint32_t *qidx;             // routed query ids, partition-major [R]
+    unsigned long long qcap;          // capacity of qidx (scan is skipped if R > qcap)
+    const unsigned long long *qoff;   // [P+1] offsets into qidx
+    const unsigned long long *item_off; // [P+1]
+    uint32_t n_parts;
+    uint64_t *out;                    // (q<<32 | key) [cap]
+    unsigned long long cap;
+    DevCounters *ctr;
+    uint32_t filter;                  // 0 prefix, 1 AND, 2 none
+};
+
+// ------------------------------------------------------------ launchers --
+// All launchers are asynchronous on `s` and return the launch error.
+cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_t n_vocab, uint64_t *vsig,
+                              cudaStream_t s);
+cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, const uint64_t *set_off,
+                               uint64_t n_sets, uint64_t *w0, uint64_t *w1, uint64_t *w2, cudaStream_t s);
+cudaError_t launch_route_bitmap(const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
+                                const uint64_t *q2, uint64_t n_q, uint32_t *bm, cudaStream_t s);
+cudaError_t launch_route_scatter(const uint32_t *bm, const unsigned long long *word_off, uint64_t n_words,
+                                 uint32_t qw, uint32_t *qidx, unsigned long long cap, cudaStream_t s);
+cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const uint32_t *part_row,
+                         const uint32_t *part_n, uint32_t n_parts, unsigned long long *qoff,
+                         unsigned long long *item_cnt, DevCounters *ctr, cudaStream_t s);
+cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s);
+int scan_grid(int device);
+cudaError_t launch_split(const uint64_t *pairs, uint64_t n, uint32_t *q, uint32_t *k, cudaStream_t s);
+cudaError_t launch_gather_planes(const uint64_t *src0, const uint64_t *src1, const uint64_t *src2,
+                                 const uint32_t *idx, uint64_t n, uint64_t *d0, uint64_t *d1, uint64_t *d2,
+                                 cudaStream_t s);
+cudaError_t launch_gather_u64(const uint64_t *src, const uint32_t *idx, uint64_t n, uint64_t *dst,
+                              cudaStream_t s);
+cudaError_t launch_iota(uint32_t *v, uint64_t n, cudaStream_t s);
+
+// CUB wrappers (temp storage managed by the caller through `tmp`/`tmp_bytes`).
+cudaError_t cub_exclusive_popc_scan(const uint32_t *bm, unsigned long long *out, uint64_t n, void *tmp,
+                                    size_t *tmp_bytes, cudaStream_t s);
+cudaError_t cub_exclusive_scan_u64(const unsigned long long *in, unsigned long long *out, uint64_t n, void *tmp,
+                                   size_t *tmp_bytes, cudaStream_t s);
+cudaError_t cub_sort_pairs_u64_u32(const uint64_t *kin, uint64_t *kout, const uint32_t *vin, uint32_t *vout,
+                                   uint64_t n, void *tmp, size_t *tmp_bytes, cudaStream_t s);
+cudaError_t cub_sort_keys_u64(uint64_t *k, uint64_t *kalt, uint64_t n, int end_bit, int *sel, void *tmp,
+                              size_t *tmp_bytes, cudaStream_t s);
+cudaError_t cub_unique_u64(const uint64_t *in, uint64_t *out, unsigned long long *n_out, uint64_t n, void *tmp,
+                           size_t *tmp_bytes, cudaStream_t s);
+
+// ---------------------------------------------------------- host build --
+struct Sig {
+    uint64_t w[3];
+};
+
+struct Partition {
+    Sig mask;
+    uint64_t begin, end;  // range in the unique-signature order produced by alg1
+};
+
+// Algorithm 1 over `n` distinct signatures given in lexicographic order.
+// Writes `order` (a stable permutation: members of each partition contiguous,
+// lexicographic inside) and the partitions in FIFO acceptance order.
+void alg1_partition(const Sig *sigs, uint64_t n, uint32_t max_p, std::vector<uint32_t> &order,
+                    std::vector<Partition> &parts);
+
+void set_error(const std::string &msg);
+
+}  // namespace tmb

@@ -1,0 +1,525 @@
+// tm_kernels.cu -- sm_100a kernels of the TagMatch hot path.
+//
+// Stage map (sec. 3):
+//   k_hash_vocab     S1  tag string -> 7 Bloom positions (reading R1)
+//   k_encode_sets    S1  OR of a set's tag signatures
+//   k_route_bitmap   S2  mask_p subset-of q for every (q, p) (Alg. 2)
+//   k_route_scatter  S2  per-partition query lists (partition-major CSR)
+//   k_items          S3  per-partition batches cut into work items
+//   k_scan           S4-S7 persistent subset-scan: tile pre-filter (Alg. 4,
+//                        PAPER.md:164-198), subset check (Alg. 3),
+//                        warp-aggregated compaction fused with the
+//                        set-id -> key lookup
+//   k_split          S8  sorted (q<<32|key) -> query[], key[]
+// plus CUB scans / radix sorts / unique (S2, S8) and small gather kernels used
+// by tm_build.
+#include <cub/cub.cuh>
+
+#include "tm_internal.h"
+
+namespace tmb {
+
+namespace {
+
+constexpr uint64_t kFnvOffset = 0xcbf29ce484222325ULL;
+constexpr uint64_t kFnvPrime = 0x100000001b3ULL;
+constexpr uint64_t kGolden = 0x9e3779b97f4a7c15ULL;
+
+__device__ __forceinline__ uint64_t splitmix_out(uint64_t z) {
+    z = (z ^ (z >> 30)) * 0xbf58476d1ce4e5b9ULL;
+    z = (z ^ (z >> 27)) * 0x94d049bb133111ebULL;
+    return z ^ (z >> 31);
+}
+
+inline unsigned grid_for(uint64_t n, unsigned bs) {
+    uint64_t g = (n + bs - 1) / bs;
+    return (unsigned)(g ? g : 1);
+}
+
+// ------------------------------------------------------------------ S1 ---
+// One thread per vocabulary string: FNV-1a-64 of the bytes, then positions
+// floor(z*192/2^64) of the first 7 SplitMix64 outputs seeded with it.
+__global__ void k_hash_vocab(const uint8_t *__restrict__ bytes, const uint64_t *__restrict__ off, uint64_t n,
+                             uint64_t *__restrict__ vsig) {
+    uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (v >= n) return;
+    uint64_t b = off[v], e = off[v + 1];
+    uint64_t h = kFnvOffset;
+    for (uint64_t i = b; i < e; ++i) {
+        h ^= (uint64_t)__ldg(bytes + i);
+        h *= kFnvPrime;
+    }
+    uint64_t s[3] = {0, 0, 0};
+    uint64_t state = h;
+#pragma unroll
+    for (int r = 0; r < kHashes; ++r) {
+        state += kGolden;
+        const uint64_t z = splitmix_out(state);
+        const uint32_t p = (uint32_t)__umul64hi(z, (uint64_t)kBits);
+        const uint64_t bit = 1ULL << (63 - (p & 63));
+        s[0] |= (p < 64) ? bit : 0ULL;
+        s[1] |= (p >= 64 && p < 128) ? bit : 0ULL;
+        s[2] |= (p >= 128) ? bit : 0ULL;
+    }
+    vsig[3 * v + 0] = s[0];
+    vsig[3 * v + 1] = s[1];
+    vsig[3 * v + 2] = s[2];
+}
+
+// One thread per set; writes the three signature planes.
+__global__ void k_encode_sets(const uint64_t *__restrict__ vsig, const uint32_t *__restrict__ tag_idx,
+                              const uint64_t *__restrict__ set_off, uint64_t n, uint64_t *__restrict__ w0,
+                              uint64_t *__restrict__ w1, uint64_t *__restrict__ w2) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    uint64_t b = set_off[i], e = set_off[i + 1];
+    uint64_t a0 = 0, a1 = 0, a2 = 0;
+    for (uint64_t t = b; t < e; ++t) {
+        const uint64_t v = tag_idx ? (uint64_t)__ldg(tag_idx + t) : t;
+        a0 |= __ldg(vsig + 3 * v + 0);
+        a1 |= __ldg(vsig + 3 * v + 1);
+        a2 |= __ldg(vsig + 3 * v + 2);
+    }
+    w0[i] = a0;
+    w1[i] = a1;
+    w2[i] = a2;
+}
+
+// ------------------------------------------------------------------ S2 ---
+// Warp w of the grid owns 32 consecutive queries (one per lane) and tests them
+// against every partition mask staged in shared memory; bitmap word
+// bm[p * QW + qw] = ballot(mask_p subset-of q) for query word qw.
+constexpr int kRouteWarps = 8;
+constexpr int kRouteMaskTile = 512;
+
+__global__ void __launch_bounds__(kRouteWarps * 32) k_route_bitmap(const uint64_t *__restrict__ masks,
+                                                                   uint32_t n_parts, const uint64_t *__restrict__ q0,
+                                                                   const uint64_t *__restrict__ q1,
+                                                                   const uint64_t *__restrict__ q2, uint64_t n_q,
+                                                                   uint32_t *__restrict__ bm, uint64_t qw_total) {
+    __shared__ uint64_t sm[3 * kRouteMaskTile];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint64_t qw = (uint64_t)blockIdx.x * kRouteWarps + warp;
+    const uint64_t q = qw * 32 + lane;
+    const bool valid = q < n_q;
+    uint64_t a0 = 0, a1 = 0, a2 = 0;
+    if (valid) {
+        a0 = q0[q];
+        a1 = q1[q];
+        a2 = q2[q];
+    }
+    for (uint32_t base = 0; base < n_parts; base += kRouteMaskTile) {
+        const uint32_t nm = min((uint32_t)kRouteMaskTile, n_parts - base);
+        __syncthreads();
+        for (uint32_t i = threadIdx.x; i < 3 * nm; i += blockDim.x) sm[i] = masks[3 * (uint64_t)base + i];
+        __syncthreads();
+        if (qw >= qw_total) continue;
+        for (uint32_t g = 0; g < nm; g += 32) {
+            uint32_t mine = 0;
+            const uint32_t ng = min(32u, nm - g);
+            for (uint32_t j = 0; j < ng; ++j) {
+                const uint64_t *m = sm + 3 * (g + j);
+                const bool ok = valid && (((m[0] & ~a0) | (m[1] & ~a1) | (m[2] & ~a2)) == 0);
+                const uint32_t b = __ballot_sync(0xffffffffu, ok);
+                if ((uint32_t)lane == j) mine = b;
+            }
+            if ((uint32_t)lane < ng) bm[(uint64_t)(base + g + lane) * qw_total + qw] = mine;
+        }
+    }
+}
+
+// One thread per bitmap word: write the word's query ids at its scanned offset.
+__global__ void k_route_scatter(const uint32_t *__restrict__ bm, const unsigned long long *__restrict__ word_off,
+                                uint64_t n_words, uint32_t qw_total, uint32_t *__restrict__ qidx,
+                                unsigned long long cap) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n_words) return;
+    uint32_t b = bm[i];
+    if (!b) return;
+    unsigned long long o = word_off[i];
+    const uint32_t qbase = (uint32_t)(i % qw_total) * 32u;
+    while (b) {
+        const int l = __ffs(b) - 1;
+        b &= b - 1;
+        if (o < cap) qidx[o] = qbase + (uint32_t)l;
+        ++o;
+    }
+}
+
+// ------------------------------------------------------------------ S3 ---
+// Per partition: routed query count -> (chunks of kChunk queries) x (ranges of
+// kRangeRows rows) work items.
+__global__ void k_items(const unsigned long long *__restrict__ word_off, uint32_t qw_total,
+                        const uint32_t *__restrict__ part_row, const uint32_t *__restrict__ part_n, uint32_t n_parts,
+                        unsigned long long *__restrict__ qoff, unsigned long long *__restrict__ item_cnt,
+                        DevCounters *ctr) {
+    uint32_t p = blockIdx.x * blockDim.x + threadIdx.x;
+    if (p > n_parts) return;
+    const unsigned long long o = word_off[(uint64_t)p * qw_total];
+    qoff[p] = o;
+    if (p == n_parts) {
+        item_cnt[p] = 0;
+        ctr->routed = o;
+        return;
+    }
+    const unsigned long long nq = word_off[(uint64_t)(p + 1) * qw_total] - o;
+    const uint32_t rows = part_row[p + 1] - part_row[p];
+    const unsigned long long nchunk = (nq + kChunk - 1) / kChunk;
+    const unsigned long long nrange = (rows + kRangeRows - 1) / kRangeRows;
+    item_cnt[p] = nchunk * nrange;
+    if (nq) atomicAdd(&ctr->candidates, nq * (unsigned long long)part_n[p]);
+}
+
+// ------------------------------------------------------------- S4..S7 ---
+struct ScanSmem {
+    uint64_t q0[kChunk], q1[kChunk], q2[kChunk];  // the item's query batch (SoA)
+    uint32_t qid[kChunk];                          // batch slot -> query index in the call
+    uint16_t surv[kScanWarps][kChunk];             // per-warp survivor lists (Alg. 4 "Q in shared memory")
+    unsigned long long item;
+};
+
+__device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
+    return __shfl_sync(0xffffffffu, v, src);
+}
+
+__device__ __forceinline__ uint64_t keep_mask_before(uint64_t x) {
+    // bits strictly before (more significant than) the leftmost one-bit of x; x != 0
+    const int c = __clzll((long long)x);
+    return c ? (~0ULL << (64 - c)) : 0ULL;
+}
+
+// Alg. 4 (reading R6): prefix = first with every position
+// >= leftmost_nonzero_bit(first XOR last) cleared; whole first if equal.
+__device__ __forceinline__ void tile_prefix(uint64_t f0, uint64_t f1, uint64_t f2, uint64_t l0, uint64_t l1,
+                                            uint64_t l2, uint64_t &p0, uint64_t &p1, uint64_t &p2) {
+    const uint64_t x0 = f0 ^ l0, x1 = f1 ^ l1, x2 = f2 ^ l2;
+    uint64_t k0 = ~0ULL, k1 = ~0ULL, k2 = ~0ULL;
+    if (x0) {
+        k0 = keep_mask_before(x0);
+        k1 = 0;
+        k2 = 0;
+    } else if (x1) {
+        k1 = keep_mask_before(x1);
+        k2 = 0;
+    } else if (x2) {
+        k2 = keep_mask_before(x2);
+    }
+    p0 = f0 & k0;
+    p1 = f1 & k1;
+    p2 = f2 & k2;
+}
+
+// Emit the (query, key) pairs of the lanes whose set matched query slot `slot`
+// (warp-uniform call: `hit` = ballot of matching lanes, non-zero).
+__device__ __forceinline__ void emit_keys(bool m, uint32_t row, uint32_t qg, const ScanParams &p, int lane) {
+    uint32_t kb = 0, nk = 0;
+    if (m) {
+        kb = __ldg(p.key_off + row);
+        nk = __ldg(p.key_off + row + 1) - kb;
+    }
+    uint32_t incl = nk;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    unsigned long long base = 0;
+    if (lane == 31 && total) base = atomicAdd(&p.ctr->n_out, (unsigned long long)total);
+    base = __shfl_sync(0xffffffffu, base, 31);
+    unsigned long long o = base + (incl - nk);
+    const uint64_t hi = (uint64_t)qg << 32;
+    for (uint32_t j = 0; j < nk; ++j, ++o)
+        if (o < p.cap) p.out[o] = hi | (uint64_t)__ldg(p.keys + kb + j);
+}
+
+// Persistent subset-scan kernel.  Work item = (partition p, query chunk c,
+// row range r); items are taken from a global counter.  The CTA stages the
+// chunk's query signatures in shared memory once; each warp then owns a
+// 32-row tile (one set per lane, held in registers), derives the tile's
+// common prefix (or AND), compacts the chunk's queries that contain it into a
+// shared-memory survivor list with ballot/popc, and checks every survivor
+// against its 32 sets: s & ~q == 0 in all three words.  Matches are appended
+// with one atomic per warp and expanded to keys in place.
+__global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
+    __shared__ ScanSmem sm;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t lt_mask = (1u << lane) - 1u;
+    unsigned long long st_tests = 0, st_checks = 0, st_matched = 0;
+    const unsigned long long n_items = p.item_off[p.n_parts];
+    if (blockIdx.x == 0 && threadIdx.x == 0) p.ctr->n_items = n_items;
+    if (p.ctr->routed > p.qcap) return;  // query lists truncated: the host grows qidx and re-runs
+
+    for (;;) {
+        if (threadIdx.x == 0) sm.item = atomicAdd(&p.ctr->item_ctr, 1ULL);
+        __syncthreads();
+        const unsigned long long item = sm.item;
+        if (item >= n_items) break;
+        // partition: last p with item_off[p] <= item
+        uint32_t lo = 0, hi = p.n_parts;  // invariant: item_off[lo] <= item < item_off[hi]
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (__ldg(p.item_off + mid) <= item) lo = mid; else hi = mid;
+        }
+        const uint32_t part = lo;
+        const uint32_t prow = __ldg(p.part_row + part);
+        const uint32_t rows = __ldg(p.part_row + part + 1) - prow;
+        const uint32_t real_end = prow + __ldg(p.part_n + part);
+        const uint32_t nrange = (rows + kRangeRows - 1) / kRangeRows;
+        const unsigned long long local = item - __ldg(p.item_off + part);
+        const uint32_t chunk = (uint32_t)(local / nrange), range = (uint32_t)(local % nrange);
+        const unsigned long long qbeg = __ldg(p.qoff + part) + (unsigned long long)chunk * kChunk;
+        const uint32_t nq = (uint32_t)min((unsigned long long)kChunk, __ldg(p.qoff + part + 1) - qbeg);
+        const uint32_t rlo = prow + range * kRangeRows;
+        const uint32_t rhi = min(rlo + (uint32_t)kRangeRows, prow + rows);
+
+        // stage the query batch (the batch of queries of partition p)
+        for (uint32_t i = threadIdx.x; i < nq; i += blockDim.x) {
+            const uint32_t q = __ldg(p.qidx + qbeg + i);
+            sm.qid[i] = q;
+            sm.q0[i] = __ldg(p.q0 + q);
+            sm.q1[i] = __ldg(p.q1 + q);
+            sm.q2[i] = __ldg(p.q2 + q);
+        }
+        __syncthreads();
+
+        const uint32_t ntile = (rhi - rlo) / kTile;
+        // small ranges: split the batch across warps so every warp has work
+        const uint32_t nsplit = ntile >= (uint32_t)kScanWarps ? 1u : (uint32_t)kScanWarps / max(ntile, 1u);
+        const uint32_t subsz = ((nq + nsplit - 1) / nsplit + 31) & ~31u;
+        const uint32_t units = ntile * nsplit;
+        for (uint32_t u = warp; u < units; u += kScanWarps) {
+            const uint32_t tile = u / nsplit, sub = u % nsplit;
+            const uint32_t row0 = rlo + tile * kTile;
+            const uint32_t row = row0 + lane;
+            const uint32_t nvalid = min(32u, real_end - row0);
+            const bool valid = (uint32_t)lane < nvalid;
+            const uint64_t s0 = __ldg(p.w0 + row), s1 = __ldg(p.w1 + row), s2 = __ldg(p.w2 + row);
+            const uint32_t qs = sub * subsz, qe = min(nq, qs + subsz);
+            if (qs >= qe) continue;
+            uint64_t f0, f1, f2;
+            if (p.filter == 0) {
+                tile_prefix(shfl64(s0, 0), shfl64(s1, 0), shfl64(s2, 0), shfl64(s0, nvalid - 1),
+                            shfl64(s1, nvalid - 1), shfl64(s2, nvalid - 1), f0, f1, f2);
+            } else if (p.filter == 1) {
+                f0 = valid ? s0 : ~0ULL;
+                f1 = valid ? s1 : ~0ULL;
+                f2 = valid ? s2 : ~0ULL;
+#pragma unroll
+                for (int o = 16; o; o >>= 1) {
+                    f0 &= __shfl_xor_sync(0xffffffffu, f0, o);
+                    f1 &= __shfl_xor_sync(0xffffffffu, f1, o);
+                    f2 &= __shfl_xor_sync(0xffffffffu, f2, o);
+                }
+            } else {
+                f0 = f1 = f2 = 0;
+            }
+            // Alg. 4: keep the batch's queries that contain the tile prefix
+            uint16_t *surv = sm.surv[warp];
+            uint32_t cnt = 0;
+            for (uint32_t qb = qs; qb < qe; qb += 32) {
+                const uint32_t i = qb + lane;
+                bool ok = false;
+                if (i < qe) ok = ((f0 & ~sm.q0[i]) | (f1 & ~sm.q1[i]) | (f2 & ~sm.q2[i])) == 0;
+                const uint32_t b = __ballot_sync(0xffffffffu, ok);
+                if (ok) surv[cnt + __popc(b & lt_mask)] = (uint16_t)i;
+                cnt += __popc(b);
+            }
+            __syncwarp();
+            st_tests += qe - qs;
+            st_checks += (unsigned long long)cnt * nvalid;
+            // Alg. 3: every surviving query against the warp's 32 sets
+            uint32_t k = 0;
+            for (; k + 1 < cnt; k += 2) {
+                const uint32_t ia = surv[k], ib = surv[k + 1];
+                const bool ma = valid && ((s0 & ~sm.q0[ia]) | (s1 & ~sm.q1[ia]) | (s2 & ~sm.q2[ia])) == 0;
+                const bool mb = valid && ((s0 & ~sm.q0[ib]) | (s1 & ~sm.q1[ib]) | (s2 & ~sm.q2[ib])) == 0;
+                const uint32_t ba = __ballot_sync(0xffffffffu, ma);
+                const uint32_t bb = __ballot_sync(0xffffffffu, mb);
+                if (ba | bb) {
+                    if (ba) {
+                        st_matched += __popc(ba);
+                        emit_keys(ma, row, sm.qid[ia], p, lane);
+                    }
+                    if (bb) {
+                        st_matched += __popc(bb);
+                        emit_keys(mb, row, sm.qid[ib], p, lane);
+                    }
+                }
+            }
+            if (k < cnt) {
+                const uint32_t ia = surv[k];
+                const bool ma = valid && ((s0 & ~sm.q0[ia]) | (s1 & ~sm.q1[ia]) | (s2 & ~sm.q2[ia])) == 0;
+                const uint32_t ba = __ballot_sync(0xffffffffu, ma);
+                if (ba) {
+                    st_matched += __popc(ba);
+                    emit_keys(ma, row, sm.qid[ia], p, lane);
+                }
+            }
+            __syncwarp();
+        }
+        __syncthreads();
+    }
+    if (lane == 0) {
+        atomicAdd(&p.ctr->tile_tests, st_tests);
+        atomicAdd(&p.ctr->pair_checks, st_checks);
+        atomicAdd(&p.ctr->matched_sets, st_matched);
+    }
+}
+
+// ------------------------------------------------------------------ S8 ---
+__global__ void k_split(const uint64_t *__restrict__ pairs, uint64_t n, uint32_t *__restrict__ q,
+                        uint32_t *__restrict__ k) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const uint64_t v = pairs[i];
+    q[i] = (uint32_t)(v >> 32);
+    k[i] = (uint32_t)v;
+}
+
+// ---------------------------------------------------------------- build ---
+__global__ void k_gather_planes(const uint64_t *__restrict__ s0, const uint64_t *__restrict__ s1,
+                                const uint64_t *__restrict__ s2, const uint32_t *__restrict__ idx, uint64_t n,
+                                uint64_t *__restrict__ d0, uint64_t *__restrict__ d1, uint64_t *__restrict__ d2) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const uint32_t j = idx[i];
+    d0[i] = s0[j];
+    d1[i] = s1[j];
+    d2[i] = s2[j];
+}
+
+__global__ void k_gather_u64(const uint64_t *__restrict__ s, const uint32_t *__restrict__ idx, uint64_t n,
+                             uint64_t *__restrict__ d) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i < n) d[i] = s[idx[i]];
+}
+
+__global__ void k_iota(uint32_t *v, uint64_t n) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i < n) v[i] = (uint32_t)i;
+}
+
+struct PopcAt {
+    const uint32_t *bm;
+    uint64_t n;
+    __device__ unsigned long long operator()(const uint64_t &i) const {
+        return i < n ? (unsigned long long)__popc(bm[i]) : 0ULL;
+    }
+};
+
+}  // namespace
+
+// ------------------------------------------------------------ launchers ---
+cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_t n_vocab, uint64_t *vsig,
+                              cudaStream_t s) {
+    if (!n_vocab) return cudaSuccess;
+    k_hash_vocab<<<grid_for(n_vocab, 256), 256, 0, s>>>(bytes, off, n_vocab, vsig);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, const uint64_t *set_off,
+                               uint64_t n_sets, uint64_t *w0, uint64_t *w1, uint64_t *w2, cudaStream_t s) {
+    if (!n_sets) return cudaSuccess;
+    k_encode_sets<<<grid_for(n_sets, 256), 256, 0, s>>>(vsig, tag_idx, set_off, n_sets, w0, w1, w2);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_route_bitmap(const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
+                                const uint64_t *q2, uint64_t n_q, uint32_t *bm, cudaStream_t s) {
+    const uint64_t qw = (n_q + 31) / 32;
+    if (!qw || !n_parts) return cudaSuccess;
+    k_route_bitmap<<<grid_for(qw, kRouteWarps), kRouteWarps * 32, 0, s>>>(masks, n_parts, q0, q1, q2, n_q, bm, qw);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_route_scatter(const uint32_t *bm, const unsigned long long *word_off, uint64_t n_words,
+                                 uint32_t qw, uint32_t *qidx, unsigned long long cap, cudaStream_t s) {
+    if (!n_words) return cudaSuccess;
+    k_route_scatter<<<grid_for(n_words, 256), 256, 0, s>>>(bm, word_off, n_words, qw, qidx, cap);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const uint32_t *part_row,
+                         const uint32_t *part_n, uint32_t n_parts, unsigned long long *qoff,
+                         unsigned long long *item_cnt, DevCounters *ctr, cudaStream_t s) {
+    k_items<<<grid_for((uint64_t)n_parts + 1, 256), 256, 0, s>>>(word_off, qw, part_row, part_n, n_parts, qoff,
+                                                                 item_cnt, ctr);
+    return cudaGetLastError();
+}
+
+int scan_grid(int device) {
+    int sms = 0, per = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_scan, kScanWarps * 32, 0);
+    if (per < 1) per = 1;
+    if (sms < 1) sms = 1;
+    return sms * per;
+}
+
+cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s) {
+    k_scan<<<grid, kScanWarps * 32, 0, s>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_split(const uint64_t *pairs, uint64_t n, uint32_t *q, uint32_t *k, cudaStream_t s) {
+    if (!n) return cudaSuccess;
+    k_split<<<grid_for(n, 256), 256, 0, s>>>(pairs, n, q, k);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_gather_planes(const uint64_t *src0, const uint64_t *src1, const uint64_t *src2,
+                                 const uint32_t *idx, uint64_t n, uint64_t *d0, uint64_t *d1, uint64_t *d2,
+                                 cudaStream_t s) {
+    if (!n) return cudaSuccess;
+    k_gather_planes<<<grid_for(n, 256), 256, 0, s>>>(src0, src1, src2, idx, n, d0, d1, d2);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_gather_u64(const uint64_t *src, const uint32_t *idx, uint64_t n, uint64_t *dst,
+                              cudaStream_t s) {
+    if (!n) return cudaSuccess;
+    k_gather_u64<<<grid_for(n, 256), 256, 0, s>>>(src, idx, n, dst);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_iota(uint32_t *v, uint64_t n, cudaStream_t s) {
+    if (!n) return cudaSuccess;
+    k_iota<<<grid_for(n, 256), 256, 0, s>>>(v, n);
+    return cudaGetLastError();
+}
+
+// ----------------------------------------------------------------- CUB ---
+cudaError_t cub_exclusive_popc_scan(const uint32_t *bm, unsigned long long *out, uint64_t n, void *tmp,
+                                    size_t *tmp_bytes, cudaStream_t s) {
+    // out[0..n] = exclusive prefix of popc(bm[i]); out[n] = total
+    cub::CountingInputIterator<uint64_t> cnt(0);
+    cub::TransformInputIterator<unsigned long long, PopcAt, cub::CountingInputIterator<uint64_t>> it(cnt,
+                                                                                                    PopcAt{bm, n});
+    return cub::DeviceScan::ExclusiveSum(tmp, *tmp_bytes, it, out, (int64_t)(n + 1), s);
+}
+
+cudaError_t cub_exclusive_scan_u64(const unsigned long long *in, unsigned long long *out, uint64_t n, void *tmp,
+                                   size_t *tmp_bytes, cudaStream_t s) {
+    return cub::DeviceScan::ExclusiveSum(tmp, *tmp_bytes, in, out, (int64_t)n, s);
+}
+
+cudaError_t cub_sort_pairs_u64_u32(const uint64_t *kin, uint64_t *kout, const uint32_t *vin, uint32_t *vout,
+                                   uint64_t n, void *tmp, size_t *tmp_bytes, cudaStream_t s) {
+    return cub::DeviceRadixSort::SortPairs(tmp, *tmp_bytes, kin, kout, vin, vout, (int64_t)n, 0, 64, s);
+}
+
+cudaError_t cub_sort_keys_u64(uint64_t *k, uint64_t *kalt, uint64_t n, int end_bit, int *sel, void *tmp,
+                              size_t *tmp_bytes, cudaStream_t s) {
+    cub::DoubleBuffer<uint64_t> db(k, kalt);
+    cudaError_t e = cub::DeviceRadixSort::SortKeys(tmp, *tmp_bytes, db, (int64_t)n, 0, end_bit, s);
+    if (sel) *sel = db.selector;
+    return e;
+}
+
+cudaError_t cub_unique_u64(const uint64_t *in, uint64_t *out, unsigned long long *n_out, uint64_t n, void *tmp,
+                           size_t *tmp_bytes, cudaStream_t s) {
+    return cub::DeviceSelect::Unique(tmp, *tmp_bytes, in, out, n_out, (int64_t)n, s);
+}
+
+}  // namespace tmb

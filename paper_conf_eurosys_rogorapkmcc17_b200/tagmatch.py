@@ -1,0 +1,250 @@
+"""Thin ctypes binding of libtagmatch.so (include/tagmatch.h).
+
+Argument marshalling only: every step of the matching path runs in the
+library's CUDA kernels.  There is no CPU fallback -- if the extension is
+missing or no B200 is visible, calls raise.
+
+Names follow the ABI: tm_build / tm_match_batch / tm_match_batch_device /
+tm_free / tm_encode / tm_stats / tm_partitions.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libtagmatch.so")
+
+TM_DEFAULT_MAX_PARTITION = 200_000
+TM_NO_PARTITIONING = 0xFFFFFFFF
+STATUS = {0: "TM_OK", -1: "TM_EINVAL", -2: "TM_ENOMEM", -3: "TM_ECUDA", -4: "TM_ENCCL", -5: "TM_ERANGE",
+          -6: "TM_ESTATE"}
+
+
+class TagMatchError(RuntimeError):
+    def __init__(self, status: int, detail: str):
+        super().__init__(f"{STATUS.get(status, status)}: {detail}")
+        self.status = status
+
+
+class tm_tagsets(ctypes.Structure):
+    _fields_ = [("vocab_bytes", ctypes.c_void_p), ("vocab_off", ctypes.c_void_p), ("tag_idx", ctypes.c_void_p),
+                ("set_off", ctypes.c_void_p), ("n_bytes", ctypes.c_uint64), ("n_vocab", ctypes.c_uint64),
+                ("n_tags", ctypes.c_uint64), ("n_sets", ctypes.c_uint64)]
+
+
+class tm_config(ctypes.Structure):
+    _fields_ = [("max_partition", ctypes.c_uint32), ("device", ctypes.c_int32), ("n_shards", ctypes.c_uint32),
+                ("shard", ctypes.c_uint32), ("tile_filter", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+
+
+class tm_pairs(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_uint64), ("query", ctypes.POINTER(ctypes.c_uint32)),
+                ("key", ctypes.POINTER(ctypes.c_uint32)), ("priv_", ctypes.c_void_p)]
+
+
+class tm_dev_pairs(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_uint64), ("query", ctypes.c_void_p), ("key", ctypes.c_void_p)]
+
+
+class tm_stats_t(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_uint64) for n in
+                ("n_sets", "n_entries", "n_unique", "n_rows", "n_partitions", "n_partitions_total")] + \
+               [("build_ms", ctypes.c_double)] + \
+               [(n, ctypes.c_uint64) for n in
+                ("n_queries", "routed", "candidate_pairs", "tile_tests", "pair_checks", "matched_sets",
+                 "emitted_pairs", "result_pairs", "work_items", "retries")] + \
+               [(n, ctypes.c_double) for n in ("encode_ms", "route_ms", "scan_ms", "merge_ms", "total_ms")] + \
+               [("scan_launches", ctypes.c_uint32), ("kernel_launches", ctypes.c_uint32)]
+
+    def as_dict(self):
+        return {n: getattr(self, n) for n, _ in self._fields_}
+
+
+EXPORTS = ["tm_build", "tm_match_batch", "tm_match_batch_device", "tm_pairs_free", "tm_free", "tm_strerror",
+           "tm_last_error", "tm_abi_version", "tm_encode", "tm_stats", "tm_partitions", "tm_partition_sigs"]
+
+_lib = None
+
+
+def load(path: str = LIB_PATH):
+    """Load the in-tree library.  Raises if it is missing: there is no fallback."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"{path} not built: run __graft_entry__.build() "
+                          "(python -m paper_conf_eurosys_rogorapkmcc17_b200._build)")
+    L = ctypes.CDLL(path)
+    vp, P = ctypes.c_void_p, ctypes.POINTER
+    L.tm_build.restype = ctypes.c_int
+    L.tm_build.argtypes = [P(tm_tagsets), vp, vp, P(tm_config), P(vp)]
+    L.tm_match_batch.restype = ctypes.c_int
+    L.tm_match_batch.argtypes = [vp, P(tm_tagsets), ctypes.c_int, P(tm_pairs)]
+    L.tm_match_batch_device.restype = ctypes.c_int
+    L.tm_match_batch_device.argtypes = [vp, P(tm_tagsets), ctypes.c_int, P(tm_dev_pairs), vp]
+    L.tm_pairs_free.argtypes = [P(tm_pairs)]
+    L.tm_free.argtypes = [vp]
+    L.tm_strerror.restype = ctypes.c_char_p
+    L.tm_strerror.argtypes = [ctypes.c_int]
+    L.tm_last_error.restype = ctypes.c_char_p
+    L.tm_abi_version.restype = ctypes.c_uint32
+    L.tm_encode.restype = ctypes.c_int
+    L.tm_encode.argtypes = [P(tm_tagsets), vp, ctypes.c_int]
+    L.tm_stats.restype = ctypes.c_int
+    L.tm_stats.argtypes = [vp, P(tm_stats_t)]
+    L.tm_partitions.restype = ctypes.c_int
+    L.tm_partitions.argtypes = [vp, vp, vp]
+    L.tm_partition_sigs.restype = ctypes.c_int
+    L.tm_partition_sigs.argtypes = [vp, ctypes.c_uint64, vp]
+    _lib = L
+    return L
+
+
+def _check(st: int):
+    if st != 0:
+        raise TagMatchError(st, load().tm_last_error().decode(errors="replace"))
+
+
+def _ptr(a):
+    if a is None:
+        return None
+    return ctypes.c_void_p(a.ctypes.data) if a.size else None
+
+
+class HostTagSets:
+    """Host-side tm_tagsets; keeps the numpy arrays alive while referenced."""
+
+    def __init__(self, vocab_bytes, vocab_off, tag_idx, set_off):
+        self.vb = np.ascontiguousarray(vocab_bytes, dtype=np.uint8)
+        self.vo = np.ascontiguousarray(vocab_off, dtype=np.uint64)
+        self.ti = None if tag_idx is None else np.ascontiguousarray(tag_idx, dtype=np.uint32)
+        self.so = np.ascontiguousarray(set_off, dtype=np.uint64)
+        n_tags = int(self.so[-1]) if self.so.size else 0
+        self.c = tm_tagsets(_ptr(self.vb), _ptr(self.vo), _ptr(self.ti) if self.ti is not None else None,
+                            _ptr(self.so), self.vb.size, max(self.vo.size - 1, 0), n_tags, max(self.so.size - 1, 0))
+
+    @classmethod
+    def of(cls, ts):
+        """From any object with vocab_bytes / vocab_off / tag_idx / set_off (e.g. tmgen.TagSets)."""
+        return cls(ts.vocab_bytes, ts.vocab_off, ts.tag_idx, ts.set_off)
+
+
+def device_tagsets(vocab_bytes_ptr, vocab_off_ptr, tag_idx_ptr, set_off_ptr, n_bytes, n_vocab, n_tags, n_sets):
+    """tm_tagsets of device pointers (ints, e.g. torch tensor data_ptr())."""
+    return tm_tagsets(vocab_bytes_ptr or None, vocab_off_ptr or None, tag_idx_ptr or None, set_off_ptr or None,
+                      n_bytes, n_vocab, n_tags, n_sets)
+
+
+def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0) -> tm_config:
+    c = tm_config()
+    c.max_partition = max_partition
+    c.device = device
+    c.n_shards = n_shards
+    c.shard = shard
+    c.tile_filter = tile_filter
+    return c
+
+
+class Database:
+    """A tm_db handle: tm_build on construction, tm_free on close()."""
+
+    def __init__(self, sets, key_off=None, keys=None, max_partition=0, device=-1, n_shards=1, shard=0,
+                 tile_filter=0):
+        L = load()
+        self._sets = sets if isinstance(sets, HostTagSets) else HostTagSets.of(sets)
+        self._ko = None if key_off is None else np.ascontiguousarray(key_off, dtype=np.uint64)
+        self._ks = np.ascontiguousarray(keys if keys is not None else np.zeros(0), dtype=np.uint32)
+        cfg = make_config(max_partition, device, n_shards, shard, tile_filter)
+        h = ctypes.c_void_p()
+        _check(L.tm_build(ctypes.byref(self._sets.c), _ptr(self._ko), _ptr(self._ks) if self._ks.size else None,
+                          ctypes.byref(cfg), ctypes.byref(h)))
+        self.h = h
+        del self._sets  # inputs are not retained by the library
+
+    def match_batch(self, queries, unique: bool) -> tuple[np.ndarray, np.ndarray]:
+        """tm_match_batch: host queries -> sorted (query, key) arrays (copies out of pinned memory)."""
+        L = load()
+        q = queries if isinstance(queries, HostTagSets) else HostTagSets.of(queries)
+        out = tm_pairs()
+        _check(L.tm_match_batch(self.h, ctypes.byref(q.c), int(bool(unique)), ctypes.byref(out)))
+        try:
+            n = out.n
+            if n:
+                qa = np.ctypeslib.as_array(out.query, shape=(n,)).copy()
+                ka = np.ctypeslib.as_array(out.key, shape=(n,)).copy()
+            else:
+                qa = np.zeros(0, np.uint32)
+                ka = np.zeros(0, np.uint32)
+        finally:
+            L.tm_pairs_free(ctypes.byref(out))
+        return qa, ka
+
+    def match_batch_raw(self, queries: HostTagSets, unique: bool) -> tm_pairs:
+        """tm_match_batch returning the library-owned pinned tm_pairs (caller must free_pairs)."""
+        out = tm_pairs()
+        _check(load().tm_match_batch(self.h, ctypes.byref(queries.c), int(bool(unique)), ctypes.byref(out)))
+        return out
+
+    @staticmethod
+    def free_pairs(p: tm_pairs):
+        load().tm_pairs_free(ctypes.byref(p))
+
+    def match_batch_device(self, dq: tm_tagsets, unique: bool, stream: int = 0) -> tm_dev_pairs:
+        """tm_match_batch_device: device-resident queries; result stays in device memory."""
+        out = tm_dev_pairs()
+        _check(load().tm_match_batch_device(self.h, ctypes.byref(dq), int(bool(unique)), ctypes.byref(out),
+                                            ctypes.c_void_p(stream) if stream else None))
+        return out
+
+    def stats(self) -> dict:
+        s = tm_stats_t()
+        _check(load().tm_stats(self.h, ctypes.byref(s)))
+        return s.as_dict()
+
+    def partitions(self) -> tuple[np.ndarray, np.ndarray]:
+        n = self.stats()["n_partitions"]
+        masks = np.zeros((n, 3), np.uint64)
+        sizes = np.zeros(n, np.uint64)
+        if n:
+            _check(load().tm_partitions(self.h, _ptr(masks), _ptr(sizes)))
+        return masks, sizes
+
+    def partition_sigs(self, p: int, size: int) -> np.ndarray:
+        out = np.zeros((size, 3), np.uint64)
+        if size:
+            _check(load().tm_partition_sigs(self.h, p, _ptr(out)))
+        return out
+
+    def close(self):
+        if getattr(self, "h", None):
+            load().tm_free(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def encode(sets, device: int = -1) -> np.ndarray:
+    """tm_encode: Bloom signatures [n_sets, 3] uint64 computed on the GPU."""
+    L = load()
+    s = sets if isinstance(sets, HostTagSets) else HostTagSets.of(sets)
+    n = s.c.n_sets
+    out = np.zeros((n, 3), np.uint64)
+    _check(L.tm_encode(ctypes.byref(s.c), _ptr(out), device))
+    return out
+
+
+def abi_version() -> int:
+    return int(load().tm_abi_version())

@@ -1,0 +1,233 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the oracle, element by
+element, on seeded inputs.  Bit-exact: this is integer / bitwise work, and the
+output is the canonically sorted (query, key) pair list.
+
+Run with `pytest -m gpu` on a B200.
+"""
+import random
+
+import numpy as np
+import pytest
+
+import tmgen
+from oracle import o1, o2
+
+pytestmark = pytest.mark.gpu
+
+tmb = pytest.importorskip("paper_conf_eurosys_rogorapkmcc17_b200")
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    from paper_conf_eurosys_rogorapkmcc17_b200 import _build
+    _build.build()
+    tmb.load()
+
+
+def assert_pairs_equal(got, want, what=""):
+    gq, gk = got
+    wq, wk = want
+    assert gq.size == wq.size, f"{what}: {gq.size} pairs vs oracle {wq.size}"
+    bad = np.nonzero((gq != wq) | (gk != wk))[0]
+    assert bad.size == 0, f"{what}: first mismatch at {bad[:5]}: got {gq[bad[0]], gk[bad[0]]} want {wq[bad[0]], wk[bad[0]]}"
+
+
+def oracle_pairs(wl, unique, qsel=None, brute=True, max_p=50_000):
+    db = o2.encode(wl.db)
+    qs = o2.encode(wl.queries)
+    qid = None
+    if qsel is not None:
+        qs = qs[qsel]
+        qid = np.asarray(qsel, np.uint32)
+    if brute:
+        return o2.match_brute(db, wl.key_off, wl.keys, qs, unique, qid=qid)
+    q, k, _ = o2.Index(db, max_p).match(wl.key_off, wl.keys, qs, unique, qid=qid)
+    return q, k
+
+
+def tagsets(strings_per_set, vocab=None):
+    """Build a tmgen.TagSets from python lists of byte strings (direct form)."""
+    flat = [t for s in strings_per_set for t in s]
+    vb = np.frombuffer(b"".join(flat), np.uint8) if flat and any(flat) else np.zeros(0, np.uint8)
+    vo = np.zeros(len(flat) + 1, np.uint64)
+    vo[1:] = np.cumsum([len(t) for t in flat]) if flat else []
+    so = np.zeros(len(strings_per_set) + 1, np.uint64)
+    so[1:] = np.cumsum([len(s) for s in strings_per_set]) if strings_per_set else []
+    return tmgen.TagSets(vb, vo, np.arange(len(flat), dtype=np.uint32), so)
+
+
+# ------------------------------------------------------------------ encoder --
+def test_encode_bit_exact_c1(c1):
+    got = tmb.encode(c1.db)
+    want = o2.encode(c1.db)
+    assert np.array_equal(got, want)
+    gq = tmb.encode(c1.queries)
+    assert np.array_equal(gq, o2.encode(c1.queries))
+
+
+def test_encode_special_strings():
+    rnd = random.Random(5)
+    sets = [[b""], [b"cat"], [b"fr_cat", b"cat"], [b"u123", b"u123"], [bytes(range(256))],
+            [bytes(rnd.getrandbits(8) for _ in range(rnd.randrange(0, 70))) for _ in range(rnd.randrange(0, 9))]]
+    sets += [[bytes(rnd.getrandbits(8) for _ in range(rnd.randrange(0, 30))) for _ in range(rnd.randrange(0, 6))]
+             for _ in range(300)]
+    ts = tagsets(sets)
+    got = tmb.encode(ts)
+    for i, s in enumerate(sets):
+        assert tuple(int(x) for x in got[i]) == o1.words(o1.encode(s)), i
+
+
+# ----------------------------------------------------------------- matching --
+@pytest.mark.parametrize("unique", [False, True])
+@pytest.mark.parametrize("tile_filter", [0, 1, 2])
+def test_c1_single_partition(c1, unique, tile_filter):
+    """BASELINE config 0: 10k sets, 1k queries, one mask-empty partition."""
+    want = oracle_pairs(c1, unique)
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=c1.max_partition, tile_filter=tile_filter) as db:
+        got = db.match_batch(c1.queries, unique)
+        st = db.stats()
+    assert_pairs_equal(got, want, "C1")
+    assert st["n_partitions"] == 1 and st["routed"] == c1.queries.n_sets
+    assert st["candidate_pairs"] == c1.queries.n_sets * c1.db.n_sets
+    if tile_filter == 2:
+        assert st["pair_checks"] == st["candidate_pairs"]
+
+
+@pytest.mark.parametrize("max_p", [200_000, 1000, 64, 1])
+def test_c1_metamorphic_max_partition(c1, max_p):
+    """The result is invariant under MAX_P (partitioning is lossless)."""
+    want = oracle_pairs(c1, False)
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=max_p) as db:
+        got = db.match_batch(c1.queries, False)
+    assert_pairs_equal(got, want, f"C1 MAX_P={max_p}")
+
+
+@pytest.mark.parametrize("max_p", [500, 2000])
+def test_partition_table_matches_oracle_alg1(c1, max_p):
+    """Library Alg. 1 == O2 Alg. 1 (same FIFO acceptance order, masks, members)."""
+    db_sig = o2.encode(c1.db)
+    ix = o2.Index(db_sig, max_p)
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=max_p) as db:
+        st = db.stats()
+        assert st["n_unique"] == c1.db.n_sets  # no signature collisions in C1
+        masks, sizes = db.partitions()
+        assert masks.shape[0] == ix.n_parts
+        assert np.array_equal(masks, ix.masks)
+        for p in range(ix.n_parts):
+            mem = ix.members[ix.part_off[p]:ix.part_off[p + 1]].astype(np.int64)
+            want = db_sig[mem]
+            want = want[np.lexsort((want[:, 2], want[:, 1], want[:, 0]))]
+            got = db.partition_sigs(p, int(sizes[p]))
+            assert np.array_equal(got, want), p  # members, lexicographically sorted
+
+
+def test_c2_full_parity():
+    """BASELINE config 1: 1M sets, 100k queries, MAX_P = 200K; the oracle
+    uses MAX_P = 50K so no partitioning misreading can hide."""
+    wl = tmgen.config("C2")
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition) as db:
+        for unique in (False, True):
+            got = db.match_batch(wl.queries, unique)
+            want = oracle_pairs(wl, unique, brute=False, max_p=50_000)
+            assert_pairs_equal(got, want, f"C2 unique={unique}")
+        st = db.stats()
+    # every query matches at least its base set
+    assert np.unique(got[0]).size == wl.queries.n_sets
+
+
+def test_c2_sampled_against_brute_force():
+    """The partitioned oracle is itself pinned to brute force on a query sample."""
+    wl = tmgen.config("C2")
+    rnd = np.random.default_rng(12)
+    qsel = np.sort(rnd.choice(wl.queries.n_sets, 512, replace=False))
+    want = oracle_pairs(wl, False, qsel=qsel, brute=True)
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition) as db:
+        gq, gk = db.match_batch(wl.queries, False)
+    keep = np.isin(gq, qsel)
+    assert_pairs_equal((gq[keep], gk[keep]), want, "C2 sample")
+
+
+# ------------------------------------------------------------- edge cases --
+def _edge_db():
+    """Empty sets, duplicates with different keys, repeated tags, ragged sizes."""
+    rnd = random.Random(17)
+    vocab = [f"t{i}".encode() for i in range(60)] + [b"", b"\xff\x00z"]
+    sets, keys = [], []
+    for i in range(1000):
+        s = [rnd.choice(vocab) for _ in range(rnd.randint(0, 6))]
+        sets.append(s)
+        keys.append([rnd.randrange(50) for _ in range(rnd.randint(0, 3))])
+    sets += [[], [], [b"t1", b"t1", b"t2"], [b"t2", b"t1"]]   # duplicates -> merged signatures
+    keys += [[7, 7], [8], [9], [9]]
+    queries = [[rnd.choice(vocab) for _ in range(rnd.randint(0, 14))] for _ in range(333)]
+    queries += [[], vocab, [b"zzz"]]
+    return sets, keys, queries
+
+
+@pytest.mark.parametrize("max_p", [0xFFFFFFFF, 50, 1])
+@pytest.mark.parametrize("unique", [False, True])
+def test_edge_cases(max_p, unique):
+    sets, keys, queries = _edge_db()
+    db_ts, q_ts = tagsets(sets), tagsets(queries)
+    key_off = np.zeros(len(keys) + 1, np.uint64)
+    key_off[1:] = np.cumsum([len(k) for k in keys])
+    flat = np.array([k for kl in keys for k in kl], np.uint32)
+    want = o1.match([o1.encode(s) for s in sets], keys, [o1.encode(q) for q in queries], unique)
+    with tmb.Database(db_ts, key_off, flat, max_partition=max_p) as db:
+        gq, gk = db.match_batch(q_ts, unique)
+        st = db.stats()
+    assert list(zip(gq.tolist(), gk.tolist())) == want
+    assert st["n_unique"] < len(sets)   # identical signatures merged (reading R10)
+
+
+def test_empty_inputs():
+    one = tagsets([[b"a"]])
+    empty_q = tagsets([])
+    with tmb.Database(one, keys=np.array([3], np.uint32)) as db:
+        q, k = db.match_batch(empty_q, False)
+        assert q.size == 0
+        q, k = db.match_batch(tagsets([[b"a", b"b"], [b"b"]]), False)
+        assert q.tolist() == [0] and k.tolist() == [3]
+    with tmb.Database(tagsets([]), key_off=np.zeros(1, np.uint64), keys=np.zeros(0, np.uint32)) as db:
+        q, k = db.match_batch(tagsets([[b"a"]]), True)
+        assert q.size == 0
+
+
+def test_output_overflow_retry():
+    """More pairs than the initial capacity: the library re-runs the scan."""
+    sets = [[]] * 3 + [[f"t{i}".encode()] for i in range(100)]
+    keys = [list(range(1500))] * 3 + [[i] for i in range(100)]   # > 64 * 4500 pairs > initial capacity
+    key_off = np.zeros(len(keys) + 1, np.uint64)
+    key_off[1:] = np.cumsum([len(k) for k in keys])
+    flat = np.array([k for kl in keys for k in kl], np.uint32)
+    queries = [[f"t{i}".encode() for i in range(j, j + 40)] for j in range(64)]
+    want = o1.match([o1.encode(s) for s in sets], keys, [o1.encode(q) for q in queries], False)
+    with tmb.Database(tagsets(sets), key_off, flat, max_partition=20) as db:
+        gq, gk = db.match_batch(tagsets(queries), False)
+        assert db.stats()["retries"] >= 1
+    assert list(zip(gq.tolist(), gk.tolist())) == want
+
+
+class _CAI:
+    """Expose a device pointer through __cuda_array_interface__ (torch.as_tensor reads it)."""
+
+    def __init__(self, ptr, n, typestr="<u4"):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3}
+
+
+def test_device_entry_point_matches_host(c1):
+    torch = pytest.importorskip("torch")
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=200_000) as db:
+        for unique in (False, True):
+            hq, hk = db.match_batch(c1.queries, unique)
+            t = [torch.from_numpy(np.ascontiguousarray(a)).cuda() for a in
+                 (c1.queries.vocab_bytes, c1.queries.vocab_off.view(np.int64), c1.queries.tag_idx.view(np.int32),
+                  c1.queries.set_off.view(np.int64))]
+            dq = tmb.device_tagsets(t[0].data_ptr(), t[1].data_ptr(), t[2].data_ptr(), t[3].data_ptr(),
+                                    c1.queries.vocab_bytes.size, c1.queries.vocab_off.size - 1,
+                                    c1.queries.tag_idx.size, c1.queries.n_sets)
+            stream = torch.cuda.current_stream().cuda_stream
+            out = db.match_batch_device(dq, unique, stream)
+            gq = torch.as_tensor(_CAI(out.query, out.n), device="cuda").cpu().numpy().view(np.uint32)
+            gk = torch.as_tensor(_CAI(out.key, out.n), device="cuda").cpu().numpy().view(np.uint32)
+            assert_pairs_equal((gq, gk), (hq, hk), f"device API unique={unique}")

@@ -146,7 +146,7 @@ class Workload:
 
 def generate(n_sets: int, n_queries: int, seed: int, extra: tuple[int, int] = (2, 4),
              total_tags: int = 0, max_partition: int = 200_000, nthreads: int = 0,
-             name: str = "custom", keep_ids: bool = False) -> Workload:
+             name: str = "custom", keep_ids: bool = False, query_seed: int | None = None) -> Workload:
     L = lib()
     h = L.tg_db_generate(seed, n_sets, nthreads)
     try:
@@ -158,7 +158,8 @@ def generate(n_sets: int, n_queries: int, seed: int, extra: tuple[int, int] = (2
         key_off = np.zeros(n + 1, np.uint64)
         keys = np.zeros(nk, np.uint32)
         L.tg_db_copy(h, _p(set_off), _p(tags), _p(key_off), _p(keys), None)
-        qh = L.tg_queries_generate(h, seed + (1 << 32), n_queries, extra[0], extra[1], total_tags, nthreads)
+        qs = seed + (1 << 32) if query_seed is None else query_seed
+        qh = L.tg_queries_generate(h, qs, n_queries, extra[0], extra[1], total_tags, nthreads)
         try:
             nq = L.tg_q_n(qh)
             nqt = L.tg_q_n_tags(qh)
