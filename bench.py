@@ -36,9 +36,11 @@ sys.path.insert(0, ROOT)
 METRIC = "queries/sec vs DB size at 1/2/4/8 B200; subset-scan HBM GB/s vs roofline"
 ALU_LANES_PER_SM_CLK = 64     # LOP3/IADD3 ALU pipe: 16 lanes/clk/SMSP x 4 SMSP (B300_MICROARCH.md)
 SM_COUNT = 148
-# algorithmic INT ops: ~4 per (tile, query) prefix test, 7 per (set, query) check
-OPS_PER_TILE_TEST = 4
-OPS_PER_PAIR_CHECK = 7
+# algorithmic INT ops per decision: every pre-filter test
+# (mask vs query) and every pair check (set vs query) needs at least one 64-bit
+# block test = and-not of both 32-bit halves + zero test = 3 ALU ops.
+OPS_PER_TILE_TEST = 3
+OPS_PER_PAIR_CHECK = 3
 
 
 def measured_peaks():

@@ -189,6 +189,7 @@ struct tm_db {
     // database (device)
     uint64_t n_sets = 0, n_entries = 0, n_unique = 0, n_rows = 0, n_parts = 0, n_parts_total = 0;
     DevBuf planes;   // 3 x rows u64
+    DevBuf tand;     // 3 x (rows / 32) u64: AND of each tile's real rows
     DevBuf key_off;  // rows + 1 u32
     DevBuf keys;     // K u32
     DevBuf masks;    // P x 3 u64
@@ -278,6 +279,9 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         sp.w0 = db->planes.as<uint64_t>();
         sp.w1 = sp.w0 + db->n_rows;
         sp.w2 = sp.w1 + db->n_rows;
+        sp.t0 = db->tand.as<uint64_t>();
+        sp.t1 = sp.t0 + db->n_rows / kTile;
+        sp.t2 = sp.t1 + db->n_rows / kTile;
         sp.key_off = db->key_off.as<uint32_t>();
         sp.keys = db->keys.as<uint32_t>();
         sp.part_row = db->part_row.as<uint32_t>();
@@ -549,8 +553,18 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
     }
     db->h_part_row[P] = (uint32_t)r;
     db->n_entries = hkeys.size();
+    // per-tile AND of the real rows (the lossless strengthening of Alg. 4's prefix)
+    const uint64_t ntiles = rows / kTile;
+    std::vector<uint64_t> ht(3 * std::max<uint64_t>(ntiles, 1), ~0ULL);
+    for (uint64_t pi = 0; pi < P; ++pi) {
+        const uint64_t r0 = db->h_part_row[pi], r1 = r0 + db->h_sizes[pi];
+        for (uint64_t rr = r0; rr < r1; ++rr)
+            for (int w = 0; w < 3; ++w) ht[w * ntiles + rr / kTile] &= hp[w * rows + rr];
+    }
 
     db->planes.ensure(std::max<uint64_t>(rows, 1) * 24);
+    db->tand.ensure(std::max<uint64_t>(ntiles, 1) * 24);
+    if (ntiles) TMCK(cudaMemcpyAsync(db->tand.p, ht.data(), ntiles * 24, cudaMemcpyHostToDevice, s));
     db->key_off.ensure((rows + 1) * 4);
     db->keys.ensure(std::max<uint64_t>(hkeys.size(), 1) * 4);
     db->masks.ensure(std::max<uint64_t>(P, 1) * 24);
@@ -582,7 +596,7 @@ void destroy_db(tm_db *db) {
     cudaGetDevice(&prev);
     cudaSetDevice(db->device);
     if (db->stream) cudaStreamSynchronize(db->stream);
-    for (DevBuf *b : {&db->planes, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
+    for (DevBuf *b : {&db->planes, &db->tand, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
                       &db->in_voff, &db->in_tidx, &db->in_soff, &db->vsig, &db->qplanes, &db->bm, &db->word_off,
                       &db->qidx, &db->qoff, &db->item_cnt, &db->item_off, &db->out, &db->out_alt, &db->res_q,
                       &db->res_k, &db->tmp, &db->ctr})

@@ -22,8 +22,8 @@ constexpr int kTile = 32;  // rows per warp tile (= one warp, Alg. 4 "thread blo
 
 // Scan-kernel geometry.
 constexpr int kScanWarps = 8;      // warps per CTA
-constexpr int kChunk = 1024;       // queries per work item (per-partition batch)
-constexpr int kRangeRows = 2048;   // rows per work item
+constexpr int kChunk = 512;        // queries per work item (per-partition batch)
+constexpr int kRangeRows = 8192;    // rows per work item (multiple of 256)
 
 struct DevCounters {            // zeroed at the start of every match call
     unsigned long long n_out;   // (q,key) pairs emitted (may exceed capacity)
@@ -38,6 +38,7 @@ struct DevCounters {            // zeroed at the start of every match call
 
 struct ScanParams {
     const uint64_t *w0, *w1, *w2;     // db planes [rows]
+    const uint64_t *t0, *t1, *t2;     // AND of each 32-row tile's real rows [rows / 32]
     const uint32_t *key_off;          // [rows+1]
     const uint32_t *keys;             // [K]
     const uint32_t *part_row;         // [P+1] padded row offsets

@@ -171,11 +171,22 @@ __global__ void k_items(const unsigned long long *__restrict__ word_off, uint32_
 }
 
 // ------------------------------------------------------------- S4..S7 ---
+// Two-level pre-filter (Alg. 4 generalised): level A tests the batch against
+// the common mask of a 256-row block (8 tiles), level B tests the level-A
+// survivors against the mask of each 32-row tile; only level-B survivors are
+// checked against the tile's 32 sets (Alg. 3).
+constexpr int kBlockTiles = 8;   // tiles per level-A block (256 rows)
+constexpr int kSubB = 128;       // level-B survivors buffered per pass
+constexpr int kQSub = 128;       // queries per unit
+
 struct ScanSmem {
     uint64_t q0[kChunk], q1[kChunk], q2[kChunk];  // the item's query batch (SoA)
     uint32_t qid[kChunk];                          // batch slot -> query index in the call
-    uint16_t surv[kScanWarps][kChunk];             // per-warp survivor lists (Alg. 4 "Q in shared memory")
+    uint16_t sa[kScanWarps][kChunk];               // per-warp level-A survivors (slots)
+    ulonglong2 sb01[kScanWarps][kSubB];            // per-warp level-B survivors: blocks 0 and 1
+    uint16_t sbi[kScanWarps][kSubB];               // per-warp level-B survivors: slots
     unsigned long long item;
+    unsigned int unit_ctr;
 };
 
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
@@ -209,8 +220,10 @@ __device__ __forceinline__ void tile_prefix(uint64_t f0, uint64_t f1, uint64_t f
     p2 = f2 & k2;
 }
 
-// Emit the (query, key) pairs of the lanes whose set matched query slot `slot`
-// (warp-uniform call: `hit` = ballot of matching lanes, non-zero).
+// Emit the (query, key) pairs of the lanes whose set matched (warp-uniform
+// call).  One atomic per warp reserves the output range (warp-aggregated
+// compaction replacing the per-pair atomic of PAPER.md:158); each matching
+// lane then writes its set's keys (key lookup).
 __device__ __forceinline__ void emit_keys(bool m, uint32_t row, uint32_t qg, const ScanParams &p, int lane) {
     uint32_t kb = 0, nk = 0;
     if (m) {
@@ -233,25 +246,54 @@ __device__ __forceinline__ void emit_keys(bool m, uint32_t row, uint32_t qg, con
         if (o < p.cap) p.out[o] = hi | (uint64_t)__ldg(p.keys + kb + j);
 }
 
+// Block 2 of one survivor whose blocks 0-1 passed in some lane, then emit.
+__device__ __forceinline__ void check_block2(bool hit01, uint32_t slot, uint64_t s2, uint32_t row,
+                                             const ScanSmem &sm, const ScanParams &p, int lane,
+                                             unsigned long long &matched) {
+    const bool m = hit01 && (s2 & ~sm.q2[slot]) == 0;
+    const uint32_t b = __ballot_sync(0xffffffffu, m);
+    if (b) {
+        matched += __popc(b);
+        emit_keys(m, row, sm.qid[slot], p, lane);
+    }
+}
+
+// Warp AND over the first n lanes (others contribute all-ones).
+__device__ __forceinline__ uint64_t warp_and(uint64_t v) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) v &= __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
 // Persistent subset-scan kernel.  Work item = (partition p, query chunk c,
-// row range r); items are taken from a global counter.  The CTA stages the
-// chunk's query signatures in shared memory once; each warp then owns a
-// 32-row tile (one set per lane, held in registers), derives the tile's
-// common prefix (or AND), compacts the chunk's queries that contain it into a
-// shared-memory survivor list with ballot/popc, and checks every survivor
-// against its 32 sets: s & ~q == 0 in all three words.  Matches are appended
-// with one atomic per warp and expanded to keys in place.
+// row range r) from a global counter; the CTA stages the chunk's query
+// signatures in shared memory, then its warps take units = (256-row block,
+// query sub-range) from a shared counter.  Per unit: level A compacts the
+// queries containing the block's common mask; per 32-row tile (one set per
+// lane, in registers) level B compacts the level-A survivors containing the
+// tile's mask, and each level-B survivor is checked block by block against
+// the 32 sets: blocks 0-1 for all, block 2 when some lane passed (the subset
+// check "amounts to a simple operation on each Bloom-filter block").
+// Filters: 0 = Alg. 4 common prefix of first/last row; 1 = AND of the rows
+// (precomputed per tile at build); 2 = none.
 __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
-    __shared__ ScanSmem sm;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    ScanSmem &sm = *reinterpret_cast<ScanSmem *>(smem_raw);
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
     unsigned long long st_tests = 0, st_checks = 0, st_matched = 0;
     const unsigned long long n_items = p.item_off[p.n_parts];
     if (blockIdx.x == 0 && threadIdx.x == 0) p.ctr->n_items = n_items;
     if (p.ctr->routed > p.qcap) return;  // query lists truncated: the host grows qidx and re-runs
+    uint16_t *sa = sm.sa[warp];
+    ulonglong2 *sb01 = sm.sb01[warp];
+    uint16_t *sbi = sm.sbi[warp];
 
     for (;;) {
-        if (threadIdx.x == 0) sm.item = atomicAdd(&p.ctr->item_ctr, 1ULL);
+        if (threadIdx.x == 0) {
+            sm.item = atomicAdd(&p.ctr->item_ctr, 1ULL);
+            sm.unit_ctr = 0;
+        }
         __syncthreads();
         const unsigned long long item = sm.item;
         if (item >= n_items) break;
@@ -284,79 +326,130 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
         __syncthreads();
 
         const uint32_t ntile = (rhi - rlo) / kTile;
-        // small ranges: split the batch across warps so every warp has work
-        const uint32_t nsplit = ntile >= (uint32_t)kScanWarps ? 1u : (uint32_t)kScanWarps / max(ntile, 1u);
+        const uint32_t nblock = (ntile + kBlockTiles - 1) / kBlockTiles;
+        // unit = (256-row block, query sub-range), taken dynamically through unit_ctr;
+        // few blocks: split the batch so every warp has work
+        const uint32_t nsplit = nblock >= (uint32_t)kScanWarps ? 1u : (uint32_t)kScanWarps / max(nblock, 1u);
         const uint32_t subsz = ((nq + nsplit - 1) / nsplit + 31) & ~31u;
-        const uint32_t units = ntile * nsplit;
-        for (uint32_t u = warp; u < units; u += kScanWarps) {
-            const uint32_t tile = u / nsplit, sub = u % nsplit;
-            const uint32_t row0 = rlo + tile * kTile;
-            const uint32_t row = row0 + lane;
-            const uint32_t nvalid = min(32u, real_end - row0);
-            const bool valid = (uint32_t)lane < nvalid;
-            const uint64_t s0 = __ldg(p.w0 + row), s1 = __ldg(p.w1 + row), s2 = __ldg(p.w2 + row);
+        const uint32_t units = nblock * nsplit;
+        for (;;) {
+            uint32_t u = 0;
+            if (lane == 0) u = atomicAdd(&sm.unit_ctr, 1u);
+            u = __shfl_sync(0xffffffffu, u, 0);
+            if (u >= units) break;
+            const uint32_t blk = u / nsplit, sub = u % nsplit;
             const uint32_t qs = sub * subsz, qe = min(nq, qs + subsz);
             if (qs >= qe) continue;
-            uint64_t f0, f1, f2;
+            const uint32_t t_first = blk * kBlockTiles, t_end = min(ntile, t_first + kBlockTiles);
+            const uint32_t brow0 = rlo + t_first * kTile;
+            const uint32_t bend = min(rlo + t_end * kTile, real_end);  // real rows of the block
+            // ---- level A: the block's common mask
+            uint64_t f0 = 0, f1 = 0, f2 = 0;
             if (p.filter == 0) {
-                tile_prefix(shfl64(s0, 0), shfl64(s1, 0), shfl64(s2, 0), shfl64(s0, nvalid - 1),
-                            shfl64(s1, nvalid - 1), shfl64(s2, nvalid - 1), f0, f1, f2);
+                tile_prefix(__ldg(p.w0 + brow0), __ldg(p.w1 + brow0), __ldg(p.w2 + brow0), __ldg(p.w0 + bend - 1),
+                            __ldg(p.w1 + bend - 1), __ldg(p.w2 + bend - 1), f0, f1, f2);
             } else if (p.filter == 1) {
-                f0 = valid ? s0 : ~0ULL;
-                f1 = valid ? s1 : ~0ULL;
-                f2 = valid ? s2 : ~0ULL;
-#pragma unroll
-                for (int o = 16; o; o >>= 1) {
-                    f0 &= __shfl_xor_sync(0xffffffffu, f0, o);
-                    f1 &= __shfl_xor_sync(0xffffffffu, f1, o);
-                    f2 &= __shfl_xor_sync(0xffffffffu, f2, o);
+                const uint32_t t = brow0 / kTile + lane;
+                const bool in = (uint32_t)lane < t_end - t_first;
+                f0 = warp_and(in ? __ldg(p.t0 + t) : ~0ULL);
+                f1 = warp_and(in ? __ldg(p.t1 + t) : ~0ULL);
+                f2 = warp_and(in ? __ldg(p.t2 + t) : ~0ULL);
+            }
+            uint32_t na = 0;
+            if ((f1 | f2) == 0) {
+                for (uint32_t qb = qs; qb < qe; qb += 32) {
+                    const uint32_t i = qb + lane;
+                    const bool ok = i < qe && (f0 & ~sm.q0[i]) == 0;
+                    const uint32_t b = __ballot_sync(0xffffffffu, ok);
+                    if (ok) sa[na + __popc(b & lt_mask)] = (uint16_t)i;
+                    na += __popc(b);
                 }
             } else {
-                f0 = f1 = f2 = 0;
+                for (uint32_t qb = qs; qb < qe; qb += 32) {
+                    const uint32_t i = qb + lane;
+                    const bool ok = i < qe && ((f0 & ~sm.q0[i]) | (f1 & ~sm.q1[i]) | (f2 & ~sm.q2[i])) == 0;
+                    const uint32_t b = __ballot_sync(0xffffffffu, ok);
+                    if (ok) sa[na + __popc(b & lt_mask)] = (uint16_t)i;
+                    na += __popc(b);
+                }
             }
-            // Alg. 4: keep the batch's queries that contain the tile prefix
-            uint16_t *surv = sm.surv[warp];
-            uint32_t cnt = 0;
-            for (uint32_t qb = qs; qb < qe; qb += 32) {
-                const uint32_t i = qb + lane;
-                bool ok = false;
-                if (i < qe) ok = ((f0 & ~sm.q0[i]) | (f1 & ~sm.q1[i]) | (f2 & ~sm.q2[i])) == 0;
-                const uint32_t b = __ballot_sync(0xffffffffu, ok);
-                if (ok) surv[cnt + __popc(b & lt_mask)] = (uint16_t)i;
-                cnt += __popc(b);
-            }
-            __syncwarp();
             st_tests += qe - qs;
-            st_checks += (unsigned long long)cnt * nvalid;
-            // Alg. 3: every surviving query against the warp's 32 sets
-            uint32_t k = 0;
-            for (; k + 1 < cnt; k += 2) {
-                const uint32_t ia = surv[k], ib = surv[k + 1];
-                const bool ma = valid && ((s0 & ~sm.q0[ia]) | (s1 & ~sm.q1[ia]) | (s2 & ~sm.q2[ia])) == 0;
-                const bool mb = valid && ((s0 & ~sm.q0[ib]) | (s1 & ~sm.q1[ib]) | (s2 & ~sm.q2[ib])) == 0;
-                const uint32_t ba = __ballot_sync(0xffffffffu, ma);
-                const uint32_t bb = __ballot_sync(0xffffffffu, mb);
-                if (ba | bb) {
-                    if (ba) {
-                        st_matched += __popc(ba);
-                        emit_keys(ma, row, sm.qid[ia], p, lane);
-                    }
-                    if (bb) {
-                        st_matched += __popc(bb);
-                        emit_keys(mb, row, sm.qid[ib], p, lane);
-                    }
-                }
-            }
-            if (k < cnt) {
-                const uint32_t ia = surv[k];
-                const bool ma = valid && ((s0 & ~sm.q0[ia]) | (s1 & ~sm.q1[ia]) | (s2 & ~sm.q2[ia])) == 0;
-                const uint32_t ba = __ballot_sync(0xffffffffu, ma);
-                if (ba) {
-                    st_matched += __popc(ba);
-                    emit_keys(ma, row, sm.qid[ia], p, lane);
-                }
-            }
             __syncwarp();
+            if (na == 0) continue;
+            // ---- per tile of the block
+            for (uint32_t t = t_first; t < t_end; ++t) {
+                const uint32_t row0 = rlo + t * kTile;
+                const uint32_t row = row0 + lane;
+                const uint32_t nvalid = min(32u, real_end - row0);
+                const bool valid = (uint32_t)lane < nvalid;
+                // rows are padded to whole tiles: every lane may load
+                const uint64_t s0 = __ldg(p.w0 + row), s1 = __ldg(p.w1 + row), s2 = __ldg(p.w2 + row);
+                uint64_t g0 = 0, g1 = 0, g2 = 0;
+                if (p.filter == 0) {
+                    tile_prefix(shfl64(s0, 0), shfl64(s1, 0), shfl64(s2, 0), shfl64(s0, nvalid - 1),
+                                shfl64(s1, nvalid - 1), shfl64(s2, nvalid - 1), g0, g1, g2);
+                } else if (p.filter == 1) {
+                    g0 = __ldg(p.t0 + row0 / kTile);
+                    g1 = __ldg(p.t1 + row0 / kTile);
+                    g2 = __ldg(p.t2 + row0 / kTile);
+                }
+                // 32-bit halves of blocks 0-1 (invalid lanes: all ones, never pass)
+                const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
+                const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
+                for (uint32_t pb = 0; pb < na; pb += kSubB) {
+                    const uint32_t pe = min(na, pb + (uint32_t)kSubB);
+                    // ---- level B: level-A survivors that contain the tile's mask
+                    uint32_t nb = 0;
+                    for (uint32_t j = pb; j < pe; j += 32) {
+                        const uint32_t jj = j + lane;
+                        bool ok = false;
+                        uint64_t a0 = 0, a1 = 0;
+                        uint32_t i = 0;
+                        if (jj < pe) {
+                            i = sa[jj];
+                            a0 = sm.q0[i];
+                            a1 = sm.q1[i];
+                            ok = ((g0 & ~a0) | (g1 & ~a1)) == 0 && (g2 == 0 || (g2 & ~sm.q2[i]) == 0);
+                        }
+                        const uint32_t b = __ballot_sync(0xffffffffu, ok);
+                        if (ok) {
+                            const uint32_t k = nb + __popc(b & lt_mask);
+                            sb01[k] = make_ulonglong2(a0, a1);
+                            sbi[k] = (uint16_t)i;
+                        }
+                        nb += __popc(b);
+                    }
+                    st_tests += pe - pb;
+                    st_checks += (unsigned long long)nb * nvalid;
+                    // pad to a multiple of 4 with zeros (masked by k < nb below)
+                    if ((uint32_t)lane < ((4 - (nb & 3)) & 3)) {
+                        sb01[nb + lane] = make_ulonglong2(0, 0);
+                        sbi[nb + lane] = 0;
+                    }
+                    __syncwarp();
+                    // ---- Alg. 3: blocks 0-1 of every survivor, 4 at a time; block 2 on a hit
+                    for (uint32_t k = 0; k < nb; k += 4) {
+                        const uint4 v0 = reinterpret_cast<const uint4 *>(sb01)[k];
+                        const uint4 v1 = reinterpret_cast<const uint4 *>(sb01)[k + 1];
+                        const uint4 v2 = reinterpret_cast<const uint4 *>(sb01)[k + 2];
+                        const uint4 v3 = reinterpret_cast<const uint4 *>(sb01)[k + 3];
+                        const bool h0 = ((a0l & ~v0.x) | (a0h & ~v0.y) | (a1l & ~v0.z) | (a1h & ~v0.w)) == 0;
+                        const bool h1 = ((a0l & ~v1.x) | (a0h & ~v1.y) | (a1l & ~v1.z) | (a1h & ~v1.w)) == 0;
+                        const bool h2 = ((a0l & ~v2.x) | (a0h & ~v2.y) | (a1l & ~v2.z) | (a1h & ~v2.w)) == 0;
+                        const bool h3 = ((a0l & ~v3.x) | (a0h & ~v3.y) | (a1l & ~v3.z) | (a1h & ~v3.w)) == 0;
+                        if (__any_sync(0xffffffffu, h0 | h1 | h2 | h3)) {
+                            if (__any_sync(0xffffffffu, h0)) check_block2(h0, sbi[k], s2, row, sm, p, lane, st_matched);
+                            if (k + 1 < nb && __any_sync(0xffffffffu, h1))
+                                check_block2(h1, sbi[k + 1], s2, row, sm, p, lane, st_matched);
+                            if (k + 2 < nb && __any_sync(0xffffffffu, h2))
+                                check_block2(h2, sbi[k + 2], s2, row, sm, p, lane, st_matched);
+                            if (k + 3 < nb && __any_sync(0xffffffffu, h3))
+                                check_block2(h3, sbi[k + 3], s2, row, sm, p, lane, st_matched);
+                        }
+                    }
+                    __syncwarp();
+                }
+            }
         }
         __syncthreads();
     }
@@ -451,14 +544,15 @@ cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const 
 int scan_grid(int device) {
     int sms = 0, per = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_scan, kScanWarps * 32, 0);
+    cudaFuncSetAttribute(k_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScanSmem));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_scan, kScanWarps * 32, sizeof(ScanSmem));
     if (per < 1) per = 1;
     if (sms < 1) sms = 1;
     return sms * per;
 }
 
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s) {
-    k_scan<<<grid, kScanWarps * 32, 0, s>>>(p);
+    k_scan<<<grid, kScanWarps * 32, sizeof(ScanSmem), s>>>(p);
     return cudaGetLastError();
 }
 
