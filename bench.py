@@ -15,6 +15,9 @@ e2e    : queries/s through tm_match_batch with pinned host queries (H2D inside
 N > 1  : one process per GPU (torchrun); every rank holds a replica of the
          database and matches its own query batch (replicated mode, PAPER.md:110,
          228: no data-path collective) -> "scaling": "weak"; time = max over ranks.
+         --shard: the database is partition-sharded over the ranks, every
+         rank matches the same batch against its partitions and the pairs go to
+         query owners over NCCL (tm_match_batch_sharded_device) -> "strong".
 --impl reference : the oracle (oracle/o2.c, the paper's CPU method) on the
          host cores, on a bounded sample of the same workload per step.
 """
@@ -41,6 +44,13 @@ SM_COUNT = 148
 # block test = and-not of both 32-bit halves + zero test = 3 ALU ops.
 OPS_PER_TILE_TEST = 3
 OPS_PER_PAIR_CHECK = 3
+
+
+class _CAI:
+    """__cuda_array_interface__ view of a library-owned device array (uint32)."""
+
+    def __init__(self, ptr, n, typestr="<u4"):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3}
 
 
 def measured_peaks():
@@ -174,7 +184,8 @@ def config_block(c, args, wl):
             "query_tags": "base set + 2..4 extra" if not c["total_tags"] else f"total {c['total_tags']}",
             "max_partition": c["max_partition"], "mode": "match-unique" if args.unique else "match",
             "tile_filter": ["alg4-prefix", "tile-and", "none"][args.tile_filter],
-            "parallelism": f"replicated-dp{args.gpus}" if args.gpus > 1 else "single",
+            "parallelism": (f"partition-sharded-{args.gpus} (NCCL exchange)" if args.shard else
+                            f"replicated-dp{args.gpus}") if args.gpus > 1 else "single",
             "l2": "flushed between timed steps (512 MiB write)", "bloom": "192 bits, k=7 (PAPER.md:106)"}
 
 
@@ -199,13 +210,20 @@ def run_ours(args):
         dist.barrier()
     import paper_conf_eurosys_rogorapkmcc17_b200 as tmb
 
-    wl, c = load_workload(args.config, rank)
+    sharded = args.shard and world > 1
+    # replicated mode: every rank its own batch; sharded mode: the same batch on every rank
+    wl, c = load_workload(args.config, 0 if sharded else rank)
     unique = bool(args.unique)
     Q = wl.queries.n_sets
     t0 = time.perf_counter()
     db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], device=dev,
-                      tile_filter=args.tile_filter)
+                      tile_filter=args.tile_filter, n_shards=world if sharded else 1, shard=rank if sharded else 0)
     build_s = time.perf_counter() - t0
+    if sharded:
+        from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as tmx
+        uid = [tmx.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
+        db.comm_init(uid[0], world, rank)
 
     # device-resident query batch (value) and pinned host copy (e2e)
     qarr = [np.ascontiguousarray(a) for a in (wl.queries.vocab_bytes, wl.queries.vocab_off.view(np.int64),
@@ -221,12 +239,31 @@ def run_ours(args):
     stream = torch.cuda.current_stream()
 
     def step_device():
+        if sharded:
+            return db.match_batch_sharded_device(dq, unique, stream.cuda_stream)
         return db.match_batch_device(dq, unique, stream.cuda_stream)
+
+    def step_e2e():
+        """Public API end to end: host queries in, host pairs out; returns D2H bytes."""
+        if not sharded:
+            p = db.match_batch_raw(hq, unique)
+            n = p.n
+            db.free_pairs(p)
+            return n * 8
+        for d, h in zip(dt_, pinned):          # H2D of the batch (every rank receives it)
+            d.copy_(h, non_blocking=True)
+        out = db.match_batch_sharded_device(dq, unique, stream.cuda_stream)
+        if out.n:                              # D2H of this rank's owner slice
+            host = torch.empty(2 * out.n, dtype=torch.int32, pin_memory=True)
+            qt = torch.as_tensor(_CAI(out.query, out.n), device=f"cuda:{dev}")
+            kt = torch.as_tensor(_CAI(out.key, out.n), device=f"cuda:{dev}")
+            host[:out.n].copy_(qt)
+            host[out.n:].copy_(kt)
+        return out.n * 8
 
     for _ in range(args.warmup):
         step_device()
-        p = db.match_batch_raw(hq, unique)
-        db.free_pairs(p)
+        step_e2e()
     torch.cuda.synchronize()
 
     # ---- value: device-resident inputs, per-step CUDA events, L2 flushed between steps
@@ -256,24 +293,25 @@ def run_ours(args):
         t = torch.tensor([t_local], device=f"cuda:{dev}", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         t_max = float(t.item())
-    value = world * Q * args.steps / t_max
+    value = (1 if sharded else world) * Q * args.steps / t_max
 
     # ---- e2e: host API, pinned inputs, H2D + D2H inside the timed region
     e2e_t, d2h = [], 0
     for i in range(args.steps):
         flush.zero_()
         torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
         t0 = time.perf_counter()
-        p = db.match_batch_raw(hq, unique)
+        d2h = step_e2e() + 8 * 2
+        torch.cuda.synchronize()
         e2e_t.append(time.perf_counter() - t0)
-        d2h = p.n * 8 + 8 * 2
-        db.free_pairs(p)
     e2e_local = sum(e2e_t)
     if world > 1:
         t = torch.tensor([e2e_local], device=f"cuda:{dev}", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_local = float(t.item())
-    e2e_value = world * Q * args.steps / e2e_local
+    e2e_value = (1 if sharded else world) * Q * args.steps / e2e_local
 
     if rank == 0:
         peaks, peak_src = measured_peaks()
@@ -293,7 +331,7 @@ def run_ours(args):
         line = {
             "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": statistics.mean(step_ms), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "u64",
             "data": "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)",
             "config": config_block(c, args, wl),
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
@@ -341,6 +379,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C2")
     ap.add_argument("--unique", action="store_true", help="match-unique instead of match")
+    ap.add_argument("--shard", action="store_true",
+                    help="N > 1: partition-sharded database + NCCL exchange (strong scaling) instead of replicas")
     ap.add_argument("--tile-filter", type=int, default=0, choices=[0, 1, 2])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-s", type=float, default=10.0, help="seconds of oracle work for cpu_baseline")

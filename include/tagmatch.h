@@ -209,6 +209,63 @@ tm_status tm_partitions(const tm_db *db, uint64_t *masks, uint64_t *sizes);
  * the tagset table's order (lexicographic). sig_out: sizes[p]*3. */
 tm_status tm_partition_sigs(const tm_db *db, uint64_t p, uint64_t *sig_out);
 
+/* ------------------------------------------------------------- shards --- */
+/*
+ * Partition sharding over G GPUs ("partition an extremely large
+ * tagset table on multiple GPUs"), one process per GPU.  Every rank
+ * calls tm_build on the same input with cfg.n_shards = G, cfg.shard = rank:
+ * all ranks compute the same Alg. 1 table and each keeps the partitions the
+ * deterministic plan (tm_shard_plan) assigns to it.  A call matches the whole
+ * batch against the local partitions; the pairs are then exchanged so that
+ * rank g owns queries [tm_owner_range(Q, G, g)) and returns that slice of the
+ * global sorted result (for match-unique, de-duplicated across shards).
+ * The exchange is NCCL (all-gather of counts + grouped send/recv over
+ * NVLink); libnccl.so.2 is loaded at run time (TM_NCCL_LIB overrides the path).
+ */
+
+/* Query owner ranges: owner g holds queries [floor(Q*g/G), floor(Q*(g+1)/G)). Host only. */
+tm_status tm_owner_range(uint64_t n_queries, uint32_t n_owners, uint32_t owner, uint64_t *lo, uint64_t *hi);
+
+/* Partition -> shard plan (host only, deterministic): greedy longest-processing-
+ * time over the estimated work |P| * 4^-|mask|.  masks: n_parts*3 words,
+ * sizes: n_parts set counts, owner_out: n_parts shard ids. */
+tm_status tm_shard_plan(const uint64_t *masks, const uint64_t *sizes, uint64_t n_parts, uint32_t n_shards,
+                        uint32_t *owner_out);
+
+/* Algorithm 1 on the host (test hook, no GPU): signatures sigs[n*3] (any
+ * order, duplicates allowed) are sorted and de-duplicated, then partitioned
+ * (readings R7/R8).  Outputs, each with capacity for n entries:
+ * masks_out[P*3], sizes_out[P], sigs_out[U*3] (may be NULL: the distinct
+ * signatures partition by partition, lexicographic inside), *n_parts_out = P,
+ * *n_unique_out = U. */
+tm_status tm_partition_host(const uint64_t *sigs, uint64_t n, uint32_t max_partition, uint64_t *masks_out,
+                            uint64_t *sizes_out, uint64_t *sigs_out, uint64_t *n_parts_out, uint64_t *n_unique_out);
+
+/* The last call's merged local result as sorted (query << 32 | key) uint64 in
+ * device memory (valid until the next call on the handle). */
+tm_status tm_last_result(const tm_db *db, const uint64_t **pairs, uint64_t *n);
+
+/* counts_out[g] (host) = pairs of the last local result owned by g, for
+ * n_owners contiguous owner ranges of the last call's batch. */
+tm_status tm_shard_counts(tm_db *db, uint32_t n_owners, uint64_t *counts_out);
+
+/* Owner-side merge: sort n device pairs (query << 32 | key) received from all
+ * shards, de-duplicate if unique, and return them split in device memory
+ * owned by the handle.  n_queries = the batch size (sort width). */
+tm_status tm_shard_merge(tm_db *db, const uint64_t *pairs, uint64_t n, uint64_t n_queries, int unique,
+                         tm_dev_pairs *out, void *stream);
+
+/* NCCL communicator of a shard handle.  id: 128 bytes from tm_nccl_unique_id
+ * on one rank, distributed by the caller (e.g. torch.distributed). */
+tm_status tm_nccl_unique_id(void *id_out, uint64_t len);
+tm_status tm_comm_init(tm_db *db, const void *id, uint64_t len, int nranks, int rank);
+
+/* match / match-unique of a batch resident in device memory (the same batch on
+ * every rank) against this rank's partitions, exchanged over NCCL: *out holds
+ * this rank's owner slice of the global sorted result (query ids global). */
+tm_status tm_match_batch_sharded_device(tm_db *db, const tm_tagsets *queries, int unique, tm_dev_pairs *out,
+                                        void *stream);
+
 #ifdef __cplusplus
 }
 #endif

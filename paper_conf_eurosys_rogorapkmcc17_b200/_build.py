@@ -20,6 +20,19 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
+def _nccl_include() -> str:
+    """nccl.h of the NCCL that torch uses (pip nvidia-nccl); the library dlopens libnccl at run time."""
+    try:
+        import nvidia.nccl
+        for d in nvidia.nccl.__path__:
+            inc = os.path.join(d, "include")
+            if os.path.exists(os.path.join(inc, "nccl.h")):
+                return inc
+    except Exception:
+        pass
+    return "/opt/prime-rl/.venv/lib/python3.12/site-packages/nvidia/nccl/include"
+
+
 def _sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")) + glob.glob(os.path.join(CSRC, "*.cpp")))
 
@@ -38,12 +51,10 @@ def needs_build() -> bool:
 
 def _compile(src: str, verbose_ptxas: bool) -> str:
     obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-    cmd = [NVCC, "-c", src, "-o", obj, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-I", INCLUDE, "-I", CSRC,
+    cmd = [NVCC, "-c", src, "-o", obj, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(),
            "-Xcompiler", "-fPIC,-O3,-Wall", "--expt-relaxed-constexpr", "-DNDEBUG"]
     if verbose_ptxas and src.endswith(".cu"):
         cmd += ["-Xptxas", "-v"]
-    if src.endswith(".cpp"):
-        cmd += ["-x", "cu"] if False else []
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")
@@ -59,7 +70,7 @@ def build(force: bool = False, verbose_ptxas: bool = False) -> str:
     with cf.ThreadPoolExecutor(max_workers=8) as ex:
         objs = list(ex.map(lambda s: _compile(s, verbose_ptxas), _sources()))
     tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, "-shared", *ARCH, "-o", tmp, *objs, "-Xcompiler", "-fPIC", "-lpthread"]
+    cmd = [NVCC, "-shared", *ARCH, "-o", tmp, *objs, "-Xcompiler", "-fPIC", "-lpthread", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")

@@ -18,72 +18,14 @@
 #include <string>
 #include <vector>
 
-#include "tm_internal.h"
+#include "tm_db.h"
 
 namespace tmb {
 
-static thread_local std::string g_err;
+thread_local std::string g_err;
 void set_error(const std::string &msg) { g_err = msg; }
 
-namespace {
 
-struct CudaFail {
-    cudaError_t e;
-    const char *what;
-    int line;
-};
-
-#define TMCK(call)                                                       \
-    do {                                                                 \
-        cudaError_t _e = (call);                                         \
-        if (_e != cudaSuccess) throw ::tmb::CudaFail{_e, #call, __LINE__}; \
-    } while (0)
-
-struct StatusFail {
-    tm_status s;
-    std::string msg;
-};
-
-[[noreturn]] void fail(tm_status s, const std::string &m) { throw StatusFail{s, m}; }
-
-struct DevBuf {
-    void *p = nullptr;
-    size_t cap = 0;
-    template <class T>
-    T *as() const { return static_cast<T *>(p); }
-    // grows (never shrinks); the caller guarantees the stream is idle w.r.t. the old contents
-    void ensure(size_t bytes) {
-        if (bytes <= cap) return;
-        if (p) TMCK(cudaFree(p));
-        p = nullptr;
-        cap = 0;
-        size_t want = std::max<size_t>(bytes + bytes / 4, 256);
-        cudaError_t e = cudaMalloc(&p, want);
-        if (e != cudaSuccess) {
-            cudaGetLastError();
-            p = nullptr;
-            if (e == cudaErrorMemoryAllocation) fail(TM_ENOMEM, "device allocation of " + std::to_string(want) + " bytes failed");
-            throw CudaFail{e, "cudaMalloc", __LINE__};
-        }
-        cap = want;
-    }
-    void release() {
-        if (p) cudaFree(p);
-        p = nullptr;
-        cap = 0;
-    }
-};
-
-struct DeviceGuard {
-    int prev = -1;
-    explicit DeviceGuard(int dev) {
-        cudaGetDevice(&prev);
-        if (dev >= 0 && dev != prev) TMCK(cudaSetDevice(dev));
-    }
-    ~DeviceGuard() {
-        if (prev >= 0) cudaSetDevice(prev);
-    }
-};
 
 // -------------------------------------------- pinned host result blocks --
 struct PinnedBlock {
@@ -174,41 +116,13 @@ int bits_for(uint64_t n) {  // bits needed to represent values < n
     return b;
 }
 
-}  // namespace
 }  // namespace tmb
 
 using namespace tmb;
 
 // ================================================================== tm_db ==
-struct tm_db {
-    int device = 0;
-    cudaStream_t stream = nullptr;
-    cudaEvent_t ev[6] = {};
-    tm_config cfg{};
-    int scan_grid = 0;
-    // database (device)
-    uint64_t n_sets = 0, n_entries = 0, n_unique = 0, n_rows = 0, n_parts = 0, n_parts_total = 0;
-    DevBuf planes;   // 3 x rows u64
-    DevBuf tand;     // 3 x (rows / 32) u64: AND of each tile's real rows
-    DevBuf key_off;  // rows + 1 u32
-    DevBuf keys;     // K u32
-    DevBuf masks;    // P x 3 u64
-    DevBuf part_row; // P + 1 u32
-    DevBuf part_n;   // P u32
-    std::vector<uint64_t> h_masks, h_sizes;
-    std::vector<uint32_t> h_part_row;
-    double build_ms = 0;
-    // per-call workspace
-    DevBuf in_bytes, in_voff, in_tidx, in_soff;  // host-API staging of the queries
-    DevBuf vsig, qplanes, bm, word_off, qidx, qoff, item_cnt, item_off, out, out_alt, res_q, res_k, tmp, ctr;
-    DevCounters *h_ctr = nullptr;  // pinned
-    unsigned long long *h_nuniq = nullptr;
-    unsigned long long cap_qidx = 0, cap_out = 0;
-    tm_stats_t st{};
-};
 
 namespace tmb {
-namespace {
 
 void *cub_tmp(tm_db *db, size_t bytes) {
     db->tmp.ensure(bytes);
@@ -222,6 +136,9 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
     const uint32_t P = (uint32_t)db->n_parts;
     std::memset(&st.n_queries, 0, sizeof(tm_stats_t) - offsetof(tm_stats_t, n_queries));
     st.n_queries = Q;
+    db->last_sorted = nullptr;
+    db->last_n = 0;
+    db->last_Q = Q;
     if (Q == 0 || P == 0) return 0;
     const uint64_t QW = (Q + 31) / 32;
     const uint64_t n_words = (uint64_t)P * QW;
@@ -354,6 +271,9 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         n = *db->h_nuniq;
         sorted = dst;
     }
+    db->last_sorted = sorted;
+    db->last_n = n;
+    db->last_Q = Q;
     db->res_q.ensure(std::max<uint64_t>(n, 1) * 4);
     db->res_k.ensure(std::max<uint64_t>(n, 1) * 4);
     TMCK(launch_split(sorted, n, db->res_q.as<uint32_t>(), db->res_k.as<uint32_t>(), s));
@@ -596,10 +516,15 @@ void destroy_db(tm_db *db) {
     cudaGetDevice(&prev);
     cudaSetDevice(db->device);
     if (db->stream) cudaStreamSynchronize(db->stream);
+    try {
+        shard_destroy(db);
+    } catch (...) {
+    }
     for (DevBuf *b : {&db->planes, &db->tand, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
                       &db->in_voff, &db->in_tidx, &db->in_soff, &db->vsig, &db->qplanes, &db->bm, &db->word_off,
                       &db->qidx, &db->qoff, &db->item_cnt, &db->item_off, &db->out, &db->out_alt, &db->res_q,
-                      &db->res_k, &db->tmp, &db->ctr})
+                      &db->res_k, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,
+                      &db->mk})
         b->release();
     for (auto &e : db->ev)
         if (e) cudaEventDestroy(e);
@@ -625,31 +550,9 @@ int check_device(int dev) {
     return dev;
 }
 
-}  // namespace
 }  // namespace tmb
 
 // ==================================================================== ABI ==
-#define TM_API_BEGIN \
-    try {            \
-        tmb::set_error("");
-#define TM_API_END                                                   \
-    }                                                                \
-    catch (const tmb::StatusFail &f) {                                \
-        tmb::set_error(f.msg);                                        \
-        return f.s;                                                  \
-    }                                                                \
-    catch (const tmb::CudaFail &f) {                                  \
-        return tmb::translate(f);                                     \
-    }                                                                \
-    catch (const std::bad_alloc &) {                                 \
-        tmb::set_error("host allocation failed");                    \
-        return TM_ENOMEM;                                            \
-    }                                                                \
-    catch (...) {                                                    \
-        tmb::set_error("unexpected exception");                      \
-        return TM_ESTATE;                                            \
-    }
-
 extern "C" {
 
 uint32_t tm_abi_version(void) { return TM_ABI_VERSION; }

@@ -1,0 +1,145 @@
+// tm_db.h -- the database handle and host-side error plumbing (internal).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "tm_internal.h"
+
+namespace tmb {
+
+struct CudaFail {
+    cudaError_t e;
+    const char *what;
+    int line;
+};
+
+#define TMCK(call)                                                       \
+    do {                                                                 \
+        cudaError_t _e = (call);                                         \
+        if (_e != cudaSuccess) throw ::tmb::CudaFail{_e, #call, __LINE__}; \
+    } while (0)
+
+struct StatusFail {
+    tm_status s;
+    std::string msg;
+};
+
+[[noreturn]] inline void fail(tm_status s, const std::string &m) { throw StatusFail{s, m}; }
+
+struct DevBuf {
+    void *p = nullptr;
+    size_t cap = 0;
+    template <class T>
+    T *as() const { return static_cast<T *>(p); }
+    // grows (never shrinks); the caller guarantees the stream is idle w.r.t. the old contents
+    void ensure(size_t bytes) {
+        if (bytes <= cap) return;
+        if (p) TMCK(cudaFree(p));
+        p = nullptr;
+        cap = 0;
+        size_t want = std::max<size_t>(bytes + bytes / 4, 256);
+        cudaError_t e = cudaMalloc(&p, want);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            p = nullptr;
+            if (e == cudaErrorMemoryAllocation) fail(TM_ENOMEM, "device allocation of " + std::to_string(want) + " bytes failed");
+            throw CudaFail{e, "cudaMalloc", __LINE__};
+        }
+        cap = want;
+    }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        cap = 0;
+    }
+};
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        cudaGetDevice(&prev);
+        if (dev >= 0 && dev != prev) TMCK(cudaSetDevice(dev));
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+extern thread_local std::string g_err;
+
+}  // namespace tmb
+
+using namespace tmb;
+
+struct tm_db {
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    cudaEvent_t ev[6] = {};
+    tm_config cfg{};
+    int scan_grid = 0;
+    // database (device)
+    uint64_t n_sets = 0, n_entries = 0, n_unique = 0, n_rows = 0, n_parts = 0, n_parts_total = 0;
+    DevBuf planes;   // 3 x rows u64
+    DevBuf tand;     // 3 x (rows / 32) u64: AND of each tile's real rows
+    DevBuf key_off;  // rows + 1 u32
+    DevBuf keys;     // K u32
+    DevBuf masks;    // P x 3 u64
+    DevBuf part_row; // P + 1 u32
+    DevBuf part_n;   // P u32
+    std::vector<uint64_t> h_masks, h_sizes;
+    std::vector<uint32_t> h_part_row;
+    double build_ms = 0;
+    // per-call workspace
+    DevBuf in_bytes, in_voff, in_tidx, in_soff;  // host-API staging of the queries
+    DevBuf vsig, qplanes, bm, word_off, qidx, qoff, item_cnt, item_off, out, out_alt, res_q, res_k, tmp, ctr;
+    DevCounters *h_ctr = nullptr;  // pinned
+    unsigned long long *h_nuniq = nullptr;
+    unsigned long long cap_qidx = 0, cap_out = 0;
+    // last call's merged result before the split (sorted (q<<32|key)), for the shard exchange
+    uint64_t *last_sorted = nullptr;
+    uint64_t last_n = 0, last_Q = 0;
+    // shard layer (tm_shard.cu)
+    void *nccl_comm = nullptr;
+    int nranks = 1, rank = 0;
+    DevBuf xcounts, xall, xrecv, xalt, mq, mk;
+    tm_stats_t st{};
+};
+
+namespace tmb {
+void *cub_tmp(tm_db *db, size_t bytes);
+uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s);
+void finish_timing(tm_db *db, cudaStream_t s);
+tm_status translate(const CudaFail &f);
+int check_device(int dev);
+void check_tagsets_device(const tm_tagsets *t);
+int bits_for(uint64_t n);
+std::vector<uint32_t> assign_shards(const std::vector<Partition> &parts, uint32_t n_shards);
+void shard_destroy(tm_db *db);
+}  // namespace tmb
+
+#define TM_API_BEGIN \
+    try {            \
+        tmb::set_error("");
+#define TM_API_END                                                   \
+    }                                                                \
+    catch (const tmb::StatusFail &f) {                                \
+        tmb::set_error(f.msg);                                        \
+        return f.s;                                                  \
+    }                                                                \
+    catch (const tmb::CudaFail &f) {                                  \
+        return tmb::translate(f);                                     \
+    }                                                                \
+    catch (const std::bad_alloc &) {                                 \
+        tmb::set_error("host allocation failed");                    \
+        return TM_ENOMEM;                                            \
+    }                                                                \
+    catch (...) {                                                    \
+        tmb::set_error("unexpected exception");                      \
+        return TM_ESTATE;                                            \
+    }
+

@@ -64,7 +64,9 @@ class tm_stats_t(ctypes.Structure):
 
 
 EXPORTS = ["tm_build", "tm_match_batch", "tm_match_batch_device", "tm_pairs_free", "tm_free", "tm_strerror",
-           "tm_last_error", "tm_abi_version", "tm_encode", "tm_stats", "tm_partitions", "tm_partition_sigs"]
+           "tm_last_error", "tm_abi_version", "tm_encode", "tm_stats", "tm_partitions", "tm_partition_sigs",
+           "tm_owner_range", "tm_shard_plan", "tm_partition_host", "tm_last_result", "tm_shard_counts",
+           "tm_shard_merge", "tm_nccl_unique_id", "tm_comm_init", "tm_match_batch_sharded_device"]
 
 _lib = None
 
@@ -99,6 +101,18 @@ def load(path: str = LIB_PATH):
     L.tm_partitions.argtypes = [vp, vp, vp]
     L.tm_partition_sigs.restype = ctypes.c_int
     L.tm_partition_sigs.argtypes = [vp, ctypes.c_uint64, vp]
+    u64, u32, i32 = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
+    for name, args in [("tm_owner_range", [u64, u32, u32, vp, vp]),
+                       ("tm_shard_plan", [vp, vp, u64, u32, vp]),
+                       ("tm_partition_host", [vp, u64, u32, vp, vp, vp, vp, vp]),
+                       ("tm_last_result", [vp, vp, vp]),
+                       ("tm_shard_counts", [vp, u32, vp]),
+                       ("tm_shard_merge", [vp, vp, u64, u64, i32, P(tm_dev_pairs), vp]),
+                       ("tm_nccl_unique_id", [vp, u64]),
+                       ("tm_comm_init", [vp, vp, u64, i32, i32]),
+                       ("tm_match_batch_sharded_device", [vp, P(tm_tagsets), i32, P(tm_dev_pairs), vp])]:
+        getattr(L, name).restype = ctypes.c_int
+        getattr(L, name).argtypes = args
     _lib = L
     return L
 
@@ -218,6 +232,35 @@ class Database:
             _check(load().tm_partition_sigs(self.h, p, _ptr(out)))
         return out
 
+    # ---- shard layer (include/tagmatch.h "shards")
+    def last_result(self) -> tuple[int, int]:
+        """(device pointer, n) of the last call's sorted (q<<32|key) pairs."""
+        ptr, n = ctypes.c_void_p(), ctypes.c_uint64()
+        _check(load().tm_last_result(self.h, ctypes.byref(ptr), ctypes.byref(n)))
+        return ptr.value or 0, n.value
+
+    def shard_counts(self, n_owners: int) -> np.ndarray:
+        out = np.zeros(n_owners, np.uint64)
+        _check(load().tm_shard_counts(self.h, n_owners, _ptr(out)))
+        return out
+
+    def shard_merge(self, pairs_ptr: int, n: int, n_queries: int, unique: bool, stream: int = 0) -> tm_dev_pairs:
+        out = tm_dev_pairs()
+        _check(load().tm_shard_merge(self.h, ctypes.c_void_p(pairs_ptr) if pairs_ptr else None, n, n_queries,
+                                     int(bool(unique)), ctypes.byref(out),
+                                     ctypes.c_void_p(stream) if stream else None))
+        return out
+
+    def comm_init(self, uid: bytes, nranks: int, rank: int):
+        buf = ctypes.create_string_buffer(uid, len(uid))
+        _check(load().tm_comm_init(self.h, buf, len(uid), nranks, rank))
+
+    def match_batch_sharded_device(self, dq: tm_tagsets, unique: bool, stream: int = 0) -> tm_dev_pairs:
+        out = tm_dev_pairs()
+        _check(load().tm_match_batch_sharded_device(self.h, ctypes.byref(dq), int(bool(unique)), ctypes.byref(out),
+                                                    ctypes.c_void_p(stream) if stream else None))
+        return out
+
     def close(self):
         if getattr(self, "h", None):
             load().tm_free(self.h)
@@ -248,3 +291,37 @@ def encode(sets, device: int = -1) -> np.ndarray:
 
 def abi_version() -> int:
     return int(load().tm_abi_version())
+
+
+# ------------------------------------------------------------ shard layer --
+def owner_range(n_queries: int, n_owners: int, owner: int) -> tuple[int, int]:
+    lo, hi = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(load().tm_owner_range(n_queries, n_owners, owner, ctypes.byref(lo), ctypes.byref(hi)))
+    return lo.value, hi.value
+
+
+def shard_plan(masks: np.ndarray, sizes: np.ndarray, n_shards: int) -> np.ndarray:
+    masks = np.ascontiguousarray(masks, dtype=np.uint64).reshape(-1, 3)
+    sizes = np.ascontiguousarray(sizes, dtype=np.uint64)
+    out = np.zeros(masks.shape[0], np.uint32)
+    _check(load().tm_shard_plan(_ptr(masks), _ptr(sizes), masks.shape[0], n_shards, _ptr(out)))
+    return out
+
+
+def partition_host(sigs: np.ndarray, max_partition: int = 0):
+    """Algorithm 1 on the host (no GPU): (masks [P,3], sizes [P], distinct sigs [U,3] partition by partition)."""
+    sigs = np.ascontiguousarray(sigs, dtype=np.uint64).reshape(-1, 3)
+    n = max(sigs.shape[0], 1)
+    masks = np.zeros((n, 3), np.uint64)
+    sizes = np.zeros(n, np.uint64)
+    out = np.zeros((n, 3), np.uint64)
+    P, U = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(load().tm_partition_host(_ptr(sigs), sigs.shape[0], max_partition, _ptr(masks), _ptr(sizes), _ptr(out),
+                                    ctypes.byref(P), ctypes.byref(U)))
+    return masks[:P.value], sizes[:P.value], out[:U.value]
+
+
+def nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(load().tm_nccl_unique_id(buf, 128))
+    return buf.raw
