@@ -21,7 +21,7 @@ constexpr int kHashes = 7;
 constexpr int kTile = 32;  // rows per warp tile (= one warp, Alg. 4 "thread block")
 
 // Scan-kernel geometry.
-constexpr int kScanWarps = 8;      // warps per CTA
+constexpr int kScanWarps = 4;      // warps per CTA
 constexpr int kChunk = 512;        // queries per work item (per-partition batch)
 constexpr int kRangeRows = 8192;    // rows per work item (multiple of 256)
 

@@ -189,6 +189,12 @@ struct ScanSmem {
     unsigned int unit_ctr;
 };
 
+__device__ __forceinline__ uint4 lds128(uint32_t addr) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
+    return v;
+}
+
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
     return __shfl_sync(0xffffffffu, v, src);
 }
@@ -288,6 +294,7 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
     uint16_t *sa = sm.sa[warp];
     ulonglong2 *sb01 = sm.sb01[warp];
     uint16_t *sbi = sm.sbi[warp];
+    const uint32_t sb01_addr = (uint32_t)__cvta_generic_to_shared(sb01);
 
     for (;;) {
         if (threadIdx.x == 0) {
@@ -429,10 +436,8 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                     __syncwarp();
                     // ---- Alg. 3: blocks 0-1 of every survivor, 4 at a time; block 2 on a hit
                     for (uint32_t k = 0; k < nb; k += 4) {
-                        const uint4 v0 = reinterpret_cast<const uint4 *>(sb01)[k];
-                        const uint4 v1 = reinterpret_cast<const uint4 *>(sb01)[k + 1];
-                        const uint4 v2 = reinterpret_cast<const uint4 *>(sb01)[k + 2];
-                        const uint4 v3 = reinterpret_cast<const uint4 *>(sb01)[k + 3];
+                        const uint32_t a = sb01_addr + k * 16;
+                        const uint4 v0 = lds128(a), v1 = lds128(a + 16), v2 = lds128(a + 32), v3 = lds128(a + 48);
                         const bool h0 = ((a0l & ~v0.x) | (a0h & ~v0.y) | (a1l & ~v0.z) | (a1h & ~v0.w)) == 0;
                         const bool h1 = ((a0l & ~v1.x) | (a0h & ~v1.y) | (a1l & ~v1.z) | (a1h & ~v1.w)) == 0;
                         const bool h2 = ((a0l & ~v2.x) | (a0h & ~v2.y) | (a1l & ~v2.z) | (a1h & ~v2.w)) == 0;
