@@ -117,9 +117,11 @@ def load_workload(name: str, rank: int = 0):
     """BASELINE config `name`; rank r > 0 matches its own query batch (query seed + 7919 r)."""
     import tmgen
     c = dict(tmgen.CONFIGS[name])
+    if getattr(load_workload, "max_partition", 0):
+        c["max_partition"] = load_workload.max_partition
     wl = tmgen.generate(c["n_sets"], c["n_queries"], c["seed"], total_tags=c["total_tags"],
                         max_partition=c["max_partition"], name=name,
-                        query_seed=c["seed"] + (1 << 32) + 7919 * rank)
+                        query_seed=(c.get("query_seed") or c["seed"] + (1 << 32)) + 7919 * rank)
     return wl, c
 
 
@@ -131,18 +133,36 @@ def oracle_rate(wl, c, unique: bool, target_s: float = 8.0, max_q: int | None = 
     db_sig = o2.encode(wl.db)
     q_sig = o2.encode(wl.queries)
     t0 = time.perf_counter()
-    ix = o2.Index(db_sig, c["max_partition"])
+    if c["n_sets"] <= 20_000_000:
+        ix = o2.Index(db_sig, c["max_partition"])
+    else:
+        # O2's single-threaded Alg. 1 takes minutes beyond ~20M sets (213 s at 100M):
+        # the baseline is then O2's brute-force scan on all cores
+        ix = _BruteOracle(db_sig)
     build_s = time.perf_counter() - t0
     nq = q_sig.shape[0]
-    n = min(nq, 256)
+    n = min(nq, 256 if isinstance(ix, o2.Index) else 32)
     t0 = time.perf_counter()
     ix.match(wl.key_off, wl.keys, q_sig[:n], unique)
     dt = max(time.perf_counter() - t0, 1e-6)
     per_q = dt / n
-    size = int(min(nq, max(256, target_s / per_q)))
+    size = int(min(nq, max(n, target_s / per_q)))
     if max_q:
         size = min(size, max_q)
     return ix, q_sig, size, build_s
+
+
+class _BruteOracle:
+    """O2 brute force with the Index.match signature."""
+    kind = "brute force"
+
+    def __init__(self, db_sig):
+        self.db = db_sig
+
+    def match(self, key_off, keys, q_sig, unique, qid=None):
+        from oracle import o2
+        q, k = o2.match_brute(self.db, key_off, keys, q_sig, unique, qid=qid)
+        return q, k, (0, 0)
 
 
 def run_reference(args):
@@ -172,9 +192,10 @@ def run_reference(args):
             "data": "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)",
             "config": config_block(c, args, wl),
             "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
-                             "sample": f"{size} of {q_sig.shape[0]} queries per step (O2: Alg.1 MAX_P="
-                                       f"{c['max_partition']} + Alg.2 + linear scan; Alg.1 build {build_s:.1f} s "
-                                       f"excluded)"},
+                             "sample": f"{size} of {q_sig.shape[0]} queries per step ("
+                                       + (f"O2 brute force over {c['n_sets']} sets" if isinstance(ix, _BruteOracle)
+                                          else f"O2: Alg.1 MAX_P={c['max_partition']} + Alg.2 + linear scan; "
+                                               f"Alg.1 build {build_s:.1f} s excluded") + ")"},
             "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -197,9 +218,15 @@ def run_ours(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # control-plane process group (barriers, max-over-ranks timing): NCCL, one GPU per
+    # rank; TM_BENCH_PG=gloo allows a functional multi-rank run on a single GPU
+    pg = os.environ.get("TM_BENCH_PG", "nccl")
     if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        torch.cuda.set_device(local % torch.cuda.device_count())
+        if pg == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(pg)
     else:
         torch.cuda.set_device(0)
     dev = torch.cuda.current_device()
@@ -290,7 +317,7 @@ def run_ours(args):
     t_local = sum(step_ms) / 1000.0
     t_max = t_local
     if world > 1:
-        t = torch.tensor([t_local], device=f"cuda:{dev}", dtype=torch.float64)
+        t = torch.tensor([t_local], device=f"cuda:{dev}" if pg == "nccl" else "cpu", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         t_max = float(t.item())
     value = (1 if sharded else world) * Q * args.steps / t_max
@@ -308,7 +335,7 @@ def run_ours(args):
         e2e_t.append(time.perf_counter() - t0)
     e2e_local = sum(e2e_t)
     if world > 1:
-        t = torch.tensor([e2e_local], device=f"cuda:{dev}", dtype=torch.float64)
+        t = torch.tensor([e2e_local], device=f"cuda:{dev}" if pg == "nccl" else "cpu", dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_local = float(t.item())
     e2e_value = (1 if sharded else world) * Q * args.steps / e2e_local
@@ -361,9 +388,11 @@ def run_ours(args):
             dt = time.perf_counter() - t0
             line["cpu_baseline"] = {"value": size / dt, "unit": "queries/s", "cores": o2.threads(0),
                                     "kind": "oracle",
-                                    "sample": f"{size} of {Q} queries (O2: Alg.1 MAX_P={c['max_partition']} + "
-                                              f"Alg.2 + linear scan, {o2.threads(0)} threads; Alg.1 build "
-                                              f"{obuild:.1f} s excluded)"}
+                                    "sample": f"{size} of {Q} queries (" +
+                                              (f"O2 brute force over {c['n_sets']} sets, {o2.threads(0)} threads"
+                                               if isinstance(ix, _BruteOracle) else
+                                               f"O2: Alg.1 MAX_P={c['max_partition']} + Alg.2 + linear scan, "
+                                               f"{o2.threads(0)} threads; Alg.1 build {obuild:.1f} s excluded") + ")"}
         print(json.dumps(line), flush=True)
     db.close()
     if world > 1:
@@ -382,12 +411,15 @@ def main():
     ap.add_argument("--shard", action="store_true",
                     help="N > 1: partition-sharded database + NCCL exchange (strong scaling) instead of replicas")
     ap.add_argument("--tile-filter", type=int, default=0, choices=[0, 1, 2])
+    ap.add_argument("--max-partition", type=int, default=0,
+                    help="override the config's MAX_P (PAPER.md:361-371 sweep); 0 = config value")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-s", type=float, default=10.0, help="seconds of oracle work for cpu_baseline")
     ap.add_argument("--ref-step-s", type=float, default=8.0, help="seconds per --impl reference step")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    load_workload.max_partition = args.max_partition
     if args.impl == "reference":
         run_reference(args)
     else:

@@ -183,7 +183,7 @@ struct ScanSmem {
     uint64_t q0[kChunk], q1[kChunk], q2[kChunk];  // the item's query batch (SoA)
     uint32_t qid[kChunk];                          // batch slot -> query index in the call
     uint16_t sa[kScanWarps][kChunk];               // per-warp level-A survivors (slots)
-    ulonglong2 sb01[kScanWarps][kSubB];            // per-warp level-B survivors: blocks 0 and 1
+    uint4 sbuf[kScanWarps][kSubB];                 // per-warp level-B survivors (see SurvivorLayout)
     uint16_t sbi[kScanWarps][kSubB];               // per-warp level-B survivors: slots
     unsigned long long item;
     unsigned int unit_ctr;
@@ -282,6 +282,11 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // check "amounts to a simple operation on each Bloom-filter block").
 // Filters: 0 = Alg. 4 common prefix of first/last row; 1 = AND of the rows
 // (precomputed per tile at build); 2 = none.
+// Survivor layout: FULL3 = false: one 16-B entry (blocks 0, 1) per survivor, up to
+// kSubB per pass, block 2 checked on a hit; FULL3 = true: two 16-B entries
+// (blocks 0, 1 | block 2, slot) per survivor, up to kSubB / 2 per pass, all
+// three blocks checked in the main loop.  U = survivors per loop iteration.
+template <int U, bool FULL3>
 __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     ScanSmem &sm = *reinterpret_cast<ScanSmem *>(smem_raw);
@@ -292,9 +297,10 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
     if (blockIdx.x == 0 && threadIdx.x == 0) p.ctr->n_items = n_items;
     if (p.ctr->routed > p.qcap) return;  // query lists truncated: the host grows qidx and re-runs
     uint16_t *sa = sm.sa[warp];
-    ulonglong2 *sb01 = sm.sb01[warp];
+    uint4 *sbuf = sm.sbuf[warp];
     uint16_t *sbi = sm.sbi[warp];
-    const uint32_t sb01_addr = (uint32_t)__cvta_generic_to_shared(sb01);
+    const uint32_t sb_addr = (uint32_t)__cvta_generic_to_shared(sbuf);
+    constexpr uint32_t kPiece = FULL3 ? kSubB / 2 : kSubB;   // level-B survivors per pass
 
     for (;;) {
         if (threadIdx.x == 0) {
@@ -400,56 +406,91 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                     g1 = __ldg(p.t1 + row0 / kTile);
                     g2 = __ldg(p.t2 + row0 / kTile);
                 }
-                // 32-bit halves of blocks 0-1 (invalid lanes: all ones, never pass)
+                // 32-bit halves of the lane's set (invalid lanes: all ones, never pass)
                 const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
                 const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
-                for (uint32_t pb = 0; pb < na; pb += kSubB) {
-                    const uint32_t pe = min(na, pb + (uint32_t)kSubB);
+                const uint32_t a2l = valid ? (uint32_t)s2 : ~0u, a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
+                for (uint32_t pb = 0; pb < na; pb += kPiece) {
+                    const uint32_t pe = min(na, pb + kPiece);
                     // ---- level B: level-A survivors that contain the tile's mask
                     uint32_t nb = 0;
                     for (uint32_t j = pb; j < pe; j += 32) {
                         const uint32_t jj = j + lane;
                         bool ok = false;
-                        uint64_t a0 = 0, a1 = 0;
+                        uint64_t a0 = 0, a1 = 0, a2 = 0;
                         uint32_t i = 0;
                         if (jj < pe) {
                             i = sa[jj];
                             a0 = sm.q0[i];
                             a1 = sm.q1[i];
-                            ok = ((g0 & ~a0) | (g1 & ~a1)) == 0 && (g2 == 0 || (g2 & ~sm.q2[i]) == 0);
+                            a2 = sm.q2[i];
+                            ok = ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
                         }
                         const uint32_t b = __ballot_sync(0xffffffffu, ok);
                         if (ok) {
                             const uint32_t k = nb + __popc(b & lt_mask);
-                            sb01[k] = make_ulonglong2(a0, a1);
-                            sbi[k] = (uint16_t)i;
+                            if (FULL3) {
+                                sbuf[2 * k] = make_uint4((uint32_t)a0, (uint32_t)(a0 >> 32), (uint32_t)a1,
+                                                         (uint32_t)(a1 >> 32));
+                                sbuf[2 * k + 1] = make_uint4((uint32_t)a2, (uint32_t)(a2 >> 32), i, 0u);
+                            } else {
+                                sbuf[k] = make_uint4((uint32_t)a0, (uint32_t)(a0 >> 32), (uint32_t)a1,
+                                                     (uint32_t)(a1 >> 32));
+                                sbi[k] = (uint16_t)i;
+                            }
                         }
                         nb += __popc(b);
                     }
                     st_tests += pe - pb;
                     st_checks += (unsigned long long)nb * nvalid;
-                    // pad to a multiple of 4 with zeros (masked by k < nb below)
-                    if ((uint32_t)lane < ((4 - (nb & 3)) & 3)) {
-                        sb01[nb + lane] = make_ulonglong2(0, 0);
-                        sbi[nb + lane] = 0;
+                    // pad to a multiple of U with zeros (masked by k < nb below)
+                    if ((uint32_t)lane < ((U - (nb % U)) % U)) {
+                        if (FULL3) {
+                            sbuf[2 * (nb + lane)] = make_uint4(0, 0, 0, 0);
+                            sbuf[2 * (nb + lane) + 1] = make_uint4(0, 0, 0, 0);
+                        } else {
+                            sbuf[nb + lane] = make_uint4(0, 0, 0, 0);
+                            sbi[nb + lane] = 0;
+                        }
                     }
                     __syncwarp();
-                    // ---- Alg. 3: blocks 0-1 of every survivor, 4 at a time; block 2 on a hit
-                    for (uint32_t k = 0; k < nb; k += 4) {
-                        const uint32_t a = sb01_addr + k * 16;
-                        const uint4 v0 = lds128(a), v1 = lds128(a + 16), v2 = lds128(a + 32), v3 = lds128(a + 48);
-                        const bool h0 = ((a0l & ~v0.x) | (a0h & ~v0.y) | (a1l & ~v0.z) | (a1h & ~v0.w)) == 0;
-                        const bool h1 = ((a0l & ~v1.x) | (a0h & ~v1.y) | (a1l & ~v1.z) | (a1h & ~v1.w)) == 0;
-                        const bool h2 = ((a0l & ~v2.x) | (a0h & ~v2.y) | (a1l & ~v2.z) | (a1h & ~v2.w)) == 0;
-                        const bool h3 = ((a0l & ~v3.x) | (a0h & ~v3.y) | (a1l & ~v3.z) | (a1h & ~v3.w)) == 0;
-                        if (__any_sync(0xffffffffu, h0 | h1 | h2 | h3)) {
-                            if (__any_sync(0xffffffffu, h0)) check_block2(h0, sbi[k], s2, row, sm, p, lane, st_matched);
-                            if (k + 1 < nb && __any_sync(0xffffffffu, h1))
-                                check_block2(h1, sbi[k + 1], s2, row, sm, p, lane, st_matched);
-                            if (k + 2 < nb && __any_sync(0xffffffffu, h2))
-                                check_block2(h2, sbi[k + 2], s2, row, sm, p, lane, st_matched);
-                            if (k + 3 < nb && __any_sync(0xffffffffu, h3))
-                                check_block2(h3, sbi[k + 3], s2, row, sm, p, lane, st_matched);
+                    // ---- Alg. 3: U survivors per iteration against the warp's 32 sets
+                    for (uint32_t k = 0; k < nb; k += U) {
+                        bool h[U];
+                        uint32_t slot[U];
+#pragma unroll
+                        for (int j = 0; j < U; ++j) {
+                            if (FULL3) {
+                                const uint32_t a = sb_addr + (k + j) * 32;
+                                const uint4 v = lds128(a), w = lds128(a + 16);
+                                h[j] = ((a0l & ~v.x) | (a0h & ~v.y) | (a1l & ~v.z) | (a1h & ~v.w) | (a2l & ~w.x) |
+                                        (a2h & ~w.y)) == 0;
+                                slot[j] = w.z;
+                            } else {
+                                const uint4 v = lds128(sb_addr + (k + j) * 16);
+                                h[j] = ((a0l & ~v.x) | (a0h & ~v.y) | (a1l & ~v.z) | (a1h & ~v.w)) == 0;
+                                slot[j] = 0;
+                            }
+                        }
+                        bool any = false;
+#pragma unroll
+                        for (int j = 0; j < U; ++j) any |= h[j];
+                        if (__any_sync(0xffffffffu, any)) {
+#pragma unroll
+                            for (int j = 0; j < U; ++j) {
+                                if (k + j < nb && __any_sync(0xffffffffu, h[j])) {
+                                    if (FULL3) {
+                                        const bool m = h[j] && valid;
+                                        const uint32_t bm = __ballot_sync(0xffffffffu, m);
+                                        if (bm) {
+                                            st_matched += __popc(bm);
+                                            emit_keys(m, row, sm.qid[slot[j]], p, lane);
+                                        }
+                                    } else {
+                                        check_block2(h[j], sbi[k + j], s2, row, sm, p, lane, st_matched);
+                                    }
+                                }
+                            }
                         }
                     }
                     __syncwarp();
@@ -546,18 +587,39 @@ cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const 
     return cudaGetLastError();
 }
 
+namespace {
+using ScanFn = void (*)(const ScanParams);
+ScanFn scan_fn(int variant) {
+    switch (variant) {
+        case 1: return k_scan<8, false>;
+        case 2: return k_scan<4, true>;
+        case 3: return k_scan<8, true>;
+        default: return k_scan<4, false>;
+    }
+}
+}  // namespace
+
+int scan_variant() {
+    // scan-kernel variant: 0 = 4 survivors/iteration, blocks 0-1 first (default);
+    // 1 = 8, blocks 0-1; 2 = 4, all three blocks; 3 = 8, all three blocks.  TM_SCAN_VARIANT overrides.
+    const char *e = getenv("TM_SCAN_VARIANT");
+    const int v = e ? atoi(e) : 0;
+    return (v >= 0 && v <= 3) ? v : 0;
+}
+
 int scan_grid(int device) {
     int sms = 0, per = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    cudaFuncSetAttribute(k_scan, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScanSmem));
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_scan, kScanWarps * 32, sizeof(ScanSmem));
+    ScanFn f = scan_fn(scan_variant());
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScanSmem));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, kScanWarps * 32, sizeof(ScanSmem));
     if (per < 1) per = 1;
     if (sms < 1) sms = 1;
     return sms * per;
 }
 
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s) {
-    k_scan<<<grid, kScanWarps * 32, sizeof(ScanSmem), s>>>(p);
+    scan_fn(scan_variant())<<<grid, kScanWarps * 32, sizeof(ScanSmem), s>>>(p);
     return cudaGetLastError();
 }
 

@@ -1,0 +1,62 @@
+"""Parity at BASELINE.json's full sizes (C3: 100M tag sets x 1M queries; C4:
+300M x 1M) in the configuration bench.py times, checked on a seeded sample of
+queries that the oracle (O2, brute force over the whole database) computes
+one by one.  Plus size-independent properties of the whole output.
+
+These need minutes of generation and a B200; they run when TM_FULL_SIZE is set
+(`TM_FULL_SIZE=C3 pytest -m gpu tests/test_gpu_full.py`), C3 by default.
+"""
+import os
+import time
+
+import numpy as np
+import pytest
+
+import tmgen
+from oracle import o2
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow,
+              pytest.mark.skipif(not os.environ.get("TM_FULL_SIZE"), reason="set TM_FULL_SIZE=C3|C4")]
+tmb = pytest.importorskip("paper_conf_eurosys_rogorapkmcc17_b200")
+
+
+@pytest.fixture(scope="module")
+def full():
+    name = os.environ.get("TM_FULL_SIZE", "C3")
+    name = name if name in tmgen.CONFIGS else "C3"
+    t = time.time()
+    wl = tmgen.config(name)
+    print(f"\n{name}: generated {wl.db.n_sets} sets, {wl.queries.n_sets} queries in {time.time() - t:.1f} s")
+    t = time.time()
+    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition)
+    st = db.stats()
+    print(f"{name}: built in {time.time() - t:.1f} s: {st['n_partitions']} partitions, {st['n_unique']} rows")
+    yield name, wl, db
+    db.close()
+
+
+@pytest.mark.parametrize("unique", [False, True])
+def test_full_size_sampled_parity(full, unique):
+    name, wl, db = full
+    t = time.time()
+    gq, gk = db.match_batch(wl.queries, unique)
+    st = db.stats()
+    print(f"{name} unique={unique}: {gq.size} pairs in {time.time() - t:.2f} s (scan {st['scan_ms']:.1f} ms, "
+          f"{st['candidate_pairs']:.3e} candidate pairs, {st['pair_checks']:.3e} checks)")
+    # properties of the whole output: sorted, query ids in range, every query matches its base
+    key = (gq.astype(np.uint64) << np.uint64(32)) | gk.astype(np.uint64)
+    assert np.all(key[1:] >= key[:-1])
+    if unique:
+        assert np.all(key[1:] != key[:-1])
+    assert gq.size == 0 or gq.max() < wl.queries.n_sets
+    assert np.unique(gq).size == wl.queries.n_sets
+    # sampled bit-exact parity against brute force over the whole database
+    rng = np.random.default_rng(2024 + unique)
+    qsel = np.sort(rng.choice(wl.queries.n_sets, 192, replace=False))
+    t = time.time()
+    db_sig = o2.encode(wl.db)
+    qs = o2.encode(wl.queries.subset(qsel))
+    wq, wk = o2.match_brute(db_sig, wl.key_off, wl.keys, qs, unique, qid=qsel.astype(np.uint32))
+    print(f"oracle sample: {time.time() - t:.1f} s")
+    keep = np.isin(gq, qsel)
+    assert np.array_equal(gq[keep], wq) and np.array_equal(gk[keep], wk)

@@ -31,8 +31,9 @@ CONFIGS = {
     "C3": dict(n_sets=100_000_000, n_queries=1_000_000, seed=3, max_partition=200_000, total_tags=0),
     "C4": dict(n_sets=300_000_000, n_queries=1_000_000, seed=4, max_partition=200_000, total_tags=0),
 }
+# C5: one 100M-set database (seed 500), query batches of exactly t tags (query seed 500 + t)
 for _t in range(2, 21, 2):
-    CONFIGS[f"C5t{_t}"] = dict(n_sets=100_000_000, n_queries=100_000, seed=500 + _t,
+    CONFIGS[f"C5t{_t}"] = dict(n_sets=100_000_000, n_queries=100_000, seed=500, query_seed=500 + _t,
                                max_partition=200_000, total_tags=_t)
 
 
@@ -126,9 +127,18 @@ def tag_strings(ids: np.ndarray) -> tuple[np.ndarray, np.ndarray]:
 
 def intern(set_off: np.ndarray, tags: np.ndarray) -> TagSets:
     """CSR of global tag ids -> interned form with a compact vocabulary."""
-    uniq, inv = np.unique(tags, return_inverse=True)
+    tags = np.ascontiguousarray(tags, dtype=np.uint32)
+    if tags.size == 0:
+        uniq, inv = np.zeros(0, np.uint32), np.zeros(0, np.uint32)
+    else:
+        # dense remap (ids are < 8*2^20 + publishers): O(n), no sort
+        present = np.zeros(int(tags.max()) + 1, dtype=bool)
+        present[tags] = True
+        uniq = np.flatnonzero(present).astype(np.uint32)
+        remap = np.cumsum(present, dtype=np.int64) - 1
+        inv = remap[tags].astype(np.uint32)
     vb, vo = tag_strings(uniq)
-    return TagSets(vb, vo, inv.astype(np.uint32), np.ascontiguousarray(set_off, dtype=np.uint64))
+    return TagSets(vb, vo, inv, np.ascontiguousarray(set_off, dtype=np.uint64))
 
 
 @dataclass
@@ -181,4 +191,36 @@ def config(name: str, **overrides) -> Workload:
     c = dict(CONFIGS[name])
     c.update(overrides)
     return generate(c["n_sets"], c["n_queries"], c["seed"], total_tags=c["total_tags"],
-                    max_partition=c["max_partition"], name=name)
+                    max_partition=c["max_partition"], name=name, query_seed=c.get("query_seed"))
+
+
+def generate_sweep(n_sets: int, seed: int, n_queries: int, totals, query_seed_base: int,
+                   max_partition: int = 200_000, nthreads: int = 0):
+    """One database and one query batch per total tag count t (C5):
+    returns (Workload with the t = totals[0] batch, {t: TagSets}, {t: base indices})."""
+    L = lib()
+    h = L.tg_db_generate(seed, n_sets, nthreads)
+    try:
+        n, nt, nk = L.tg_db_n_sets(h), L.tg_db_n_tags(h), L.tg_db_n_keys(h)
+        set_off = np.zeros(n + 1, np.uint64)
+        tags = np.zeros(nt, np.uint32)
+        key_off = np.zeros(n + 1, np.uint64)
+        keys = np.zeros(nk, np.uint32)
+        L.tg_db_copy(h, _p(set_off), _p(tags), _p(key_off), _p(keys), None)
+        batches, bases = {}, {}
+        for t in totals:
+            qh = L.tg_queries_generate(h, query_seed_base + t, n_queries, 0, 0, t, nthreads)
+            try:
+                nq, nqt = L.tg_q_n(qh), L.tg_q_n_tags(qh)
+                q_off = np.zeros(nq + 1, np.uint64)
+                q_tags = np.zeros(nqt, np.uint32)
+                base = np.zeros(nq, np.uint64)
+                L.tg_q_copy(qh, _p(q_off), _p(q_tags), _p(base))
+            finally:
+                L.tg_q_free(qh)
+            batches[t], bases[t] = intern(q_off, q_tags), base
+    finally:
+        L.tg_db_free(h)
+    t0 = list(totals)[0]
+    wl = Workload(f"sweep{n_sets}", intern(set_off, tags), key_off, keys, batches[t0], bases[t0], max_partition)
+    return wl, batches, bases
