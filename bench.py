@@ -205,6 +205,7 @@ def config_block(c, args, wl):
             "query_tags": "base set + 2..4 extra" if not c["total_tags"] else f"total {c['total_tags']}",
             "max_partition": c["max_partition"], "mode": "match-unique" if args.unique else "match",
             "tile_filter": ["alg4-prefix", "tile-and", "none"][args.tile_filter],
+            "row_order": ["lexicographic", "balanced-splits"][args.row_order],
             "parallelism": (f"partition-sharded-{args.gpus} (NCCL exchange)" if args.shard else
                             f"replicated-dp{args.gpus}") if args.gpus > 1 else "single",
             "l2": "flushed between timed steps (512 MiB write)", "bloom": "192 bits, k=7 (PAPER.md:106)"}
@@ -244,7 +245,7 @@ def run_ours(args):
     Q = wl.queries.n_sets
     t0 = time.perf_counter()
     db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], device=dev,
-                      tile_filter=args.tile_filter, n_shards=world if sharded else 1, shard=rank if sharded else 0)
+                      tile_filter=args.tile_filter, row_order=args.row_order, n_shards=world if sharded else 1, shard=rank if sharded else 0)
     build_s = time.perf_counter() - t0
     if sharded:
         from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as tmx
@@ -410,7 +411,11 @@ def main():
     ap.add_argument("--unique", action="store_true", help="match-unique instead of match")
     ap.add_argument("--shard", action="store_true",
                     help="N > 1: partition-sharded database + NCCL exchange (strong scaling) instead of replicas")
-    ap.add_argument("--tile-filter", type=int, default=0, choices=[0, 1, 2])
+    # default layout = the B200 one (R18): balanced splits inside partitions +
+    # tile AND masks; --tile-filter 0 --row-order 0 is the paper's lexicographic order + Alg. 4 prefix
+    ap.add_argument("--tile-filter", type=int, default=1, choices=[0, 1, 2])
+    ap.add_argument("--row-order", type=int, default=1, choices=[0, 1],
+                    help="1: balanced-split order inside partitions (DESIGN.md R18; needs --tile-filter 1)")
     ap.add_argument("--max-partition", type=int, default=0,
                     help="override the config's MAX_P (PAPER.md:361-371 sweep); 0 = config value")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -419,6 +424,8 @@ def main():
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    if args.row_order == 1 and args.tile_filter == 0:
+        args.row_order = 0   # the first/last prefix needs lexicographic order
     load_workload.max_partition = args.max_partition
     if args.impl == "reference":
         run_reference(args)

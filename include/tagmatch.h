@@ -106,7 +106,13 @@ typedef struct {
     uint32_t tile_filter;   /* 0 = Alg. 4 common prefix of each 32-set tile (default);
                                1 = AND of the tile's signatures (lossless strengthening);
                                2 = no pre-filter (plain Alg. 3 scan)                   */
-    uint32_t reserved[3];   /* must be 0                                               */
+    uint32_t row_order;     /* order of the sets inside a partition:
+                               0 = lexicographic (default);
+                               1 = Alg. 1's balanced splits continued inside the partition
+                                   down to groups of <= 8 sets, depth-first (R18);
+                                   requires tile_filter 1 or 2 (Alg. 4's first/last prefix
+                                   is only sound for lexicographic order)            */
+    uint32_t reserved[2];   /* must be 0                                               */
 } tm_config;
 
 /* Result pairs in host memory, allocated by the library (pinned), released by

@@ -429,6 +429,7 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
     std::vector<uint32_t> order;
     std::vector<Partition> parts;
     alg1_partition(usig.data(), U, db->cfg.max_partition, order, parts);
+    if (db->cfg.row_order == 1) refine_order(usig.data(), order, parts, 8);
     db->n_parts_total = parts.size();
     const std::vector<uint32_t> owner = assign_shards(parts, std::max(1u, db->cfg.n_shards));
 
@@ -581,7 +582,10 @@ tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32
     if (cfg) {
         if (cfg->n_shards > 1 && cfg->shard >= cfg->n_shards) fail(TM_EINVAL, "shard >= n_shards");
         if (cfg->tile_filter > 2) fail(TM_EINVAL, "tile_filter must be 0, 1 or 2");
-        if (cfg->reserved[0] | cfg->reserved[1] | cfg->reserved[2]) fail(TM_EINVAL, "reserved fields must be 0");
+        if (cfg->row_order > 1) fail(TM_EINVAL, "row_order must be 0 or 1");
+        if (cfg->row_order == 1 && cfg->tile_filter == 0)
+            fail(TM_EINVAL, "row_order 1 needs tile_filter 1 or 2 (the first/last prefix needs lexicographic order)");
+        if (cfg->reserved[0] | cfg->reserved[1]) fail(TM_EINVAL, "reserved fields must be 0");
     }
     const int dev = check_device(cfg ? cfg->device : -1);
     DeviceGuard g(dev);

@@ -106,6 +106,14 @@ struct Partition {
 void alg1_partition(const Sig *sigs, uint64_t n, uint32_t max_p, std::vector<uint32_t> &order,
                     std::vector<Partition> &parts);
 
+// Reading R18: inside every partition, continue Alg. 1's balanced splits (pivot =
+// unused bit with frequency closest to 50%) depth-first down to groups of <= leaf
+// sets, rewriting `order` within each partition's range (P0 before P1; members
+// of a group stay lexicographic).  Rows sharing a deep path share many bits,
+// which strengthens the tile AND masks.
+void refine_order(const Sig *sigs, std::vector<uint32_t> &order, const std::vector<Partition> &parts,
+                  uint32_t leaf);
+
 void set_error(const std::string &msg);
 
 }  // namespace tmb

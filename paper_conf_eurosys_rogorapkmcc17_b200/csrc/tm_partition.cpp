@@ -8,6 +8,7 @@
 // order (what Alg. 4 needs).  Readings R7/R8 fix
 // the cases the paper leaves open.
 #include <algorithm>
+#include <atomic>
 #include <cstring>
 #include <deque>
 #include <thread>
@@ -153,6 +154,67 @@ void alg1_partition(const Sig *sigs, uint64_t n, uint32_t max_p, std::vector<uin
         Q.push_back(a);  // (mask -> P0, used_bits)
         Q.push_back(b);  // (mask u {pivot} -> P1, used_bits)
     }
+}
+
+namespace {
+
+// DFS refinement of one partition's range [lo, hi) of `order` (single thread).
+void refine_range(const Sig *sigs, uint32_t *idx, uint64_t n, uint32_t leaf, uint32_t *scratch) {
+    struct R {
+        uint64_t lo, hi;
+    };
+    std::vector<R> st;
+    st.push_back({0, n});
+    uint64_t freq[kBits];
+    while (!st.empty()) {
+        const R r = st.back();
+        st.pop_back();
+        const uint64_t cnt = r.hi - r.lo;
+        if (cnt <= leaf) continue;
+        std::memset(freq, 0, sizeof freq);
+        histogram_range(sigs, idx + r.lo, cnt, freq);
+        int pivot = -1;
+        uint64_t best = 0;
+        for (int p = 0; p < kBits; ++p) {
+            if (freq[p] == 0 || freq[p] == cnt) continue;
+            const uint64_t d = 2 * freq[p] > cnt ? 2 * freq[p] - cnt : cnt - 2 * freq[p];
+            if (pivot < 0 || d < best) {
+                pivot = p;
+                best = d;
+            }
+        }
+        if (pivot < 0) continue;  // identical signatures
+        uint64_t n0 = 0;
+        for (uint64_t i = r.lo; i < r.hi; ++i)
+            if (!pos_set(sigs[idx[i]], pivot)) scratch[n0++] = idx[i];
+        uint64_t k = n0;
+        for (uint64_t i = r.lo; i < r.hi; ++i)
+            if (pos_set(sigs[idx[i]], pivot)) scratch[k++] = idx[i];
+        std::memcpy(idx + r.lo, scratch, cnt * sizeof(uint32_t));
+        st.push_back({r.lo + n0, r.hi});  // P1 after P0 (stack: push P1 first)
+        st.push_back({r.lo, r.lo + n0});
+    }
+}
+
+}  // namespace
+
+void refine_order(const Sig *sigs, std::vector<uint32_t> &order, const std::vector<Partition> &parts,
+                  uint32_t leaf) {
+    const unsigned T = hw_threads();
+    std::atomic<size_t> next{0};
+    auto work = [&]() {
+        std::vector<uint32_t> scratch;
+        for (;;) {
+            const size_t i = next.fetch_add(1);
+            if (i >= parts.size()) break;
+            const uint64_t n = parts[i].end - parts[i].begin;
+            if (scratch.size() < n) scratch.resize(n);
+            refine_range(sigs, order.data() + parts[i].begin, n, leaf, scratch.data());
+        }
+    };
+    std::vector<std::thread> th;
+    for (unsigned t = 0; t < T; ++t) th.emplace_back(work);
+    for (auto &x : th) x.join();
 }
 
 }  // namespace tmb

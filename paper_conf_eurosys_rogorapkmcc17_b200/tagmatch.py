@@ -37,7 +37,8 @@ class tm_tagsets(ctypes.Structure):
 
 class tm_config(ctypes.Structure):
     _fields_ = [("max_partition", ctypes.c_uint32), ("device", ctypes.c_int32), ("n_shards", ctypes.c_uint32),
-                ("shard", ctypes.c_uint32), ("tile_filter", ctypes.c_uint32), ("reserved", ctypes.c_uint32 * 3)]
+                ("shard", ctypes.c_uint32), ("tile_filter", ctypes.c_uint32), ("row_order", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32 * 2)]
 
 
 class tm_pairs(ctypes.Structure):
@@ -152,13 +153,14 @@ def device_tagsets(vocab_bytes_ptr, vocab_off_ptr, tag_idx_ptr, set_off_ptr, n_b
                       n_bytes, n_vocab, n_tags, n_sets)
 
 
-def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0) -> tm_config:
+def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0, row_order=0) -> tm_config:
     c = tm_config()
     c.max_partition = max_partition
     c.device = device
     c.n_shards = n_shards
     c.shard = shard
     c.tile_filter = tile_filter
+    c.row_order = row_order
     return c
 
 
@@ -166,12 +168,12 @@ class Database:
     """A tm_db handle: tm_build on construction, tm_free on close()."""
 
     def __init__(self, sets, key_off=None, keys=None, max_partition=0, device=-1, n_shards=1, shard=0,
-                 tile_filter=0):
+                 tile_filter=0, row_order=0):
         L = load()
         self._sets = sets if isinstance(sets, HostTagSets) else HostTagSets.of(sets)
         self._ko = None if key_off is None else np.ascontiguousarray(key_off, dtype=np.uint64)
         self._ks = np.ascontiguousarray(keys if keys is not None else np.zeros(0), dtype=np.uint32)
-        cfg = make_config(max_partition, device, n_shards, shard, tile_filter)
+        cfg = make_config(max_partition, device, n_shards, shard, tile_filter, row_order)
         h = ctypes.c_void_p()
         _check(L.tm_build(ctypes.byref(self._sets.c), _ptr(self._ko), _ptr(self._ks) if self._ks.size else None,
                           ctypes.byref(cfg), ctypes.byref(h)))

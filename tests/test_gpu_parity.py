@@ -93,6 +93,24 @@ def test_c1_single_partition(c1, unique, tile_filter):
         assert st["pair_checks"] == st["candidate_pairs"]
 
 
+@pytest.mark.parametrize("unique", [False, True])
+@pytest.mark.parametrize("tile_filter", [1, 2])
+def test_c1_balanced_row_order(c1, unique, tile_filter):
+    """Row order 1 (reading R18: balanced splits inside partitions) with AND
+    masks: same result (the order inside a partition is lossless)."""
+    want = oracle_pairs(c1, unique)
+    for max_p in (0xFFFFFFFF, 2000):
+        with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=max_p, tile_filter=tile_filter,
+                          row_order=1) as db:
+            got = db.match_batch(c1.queries, unique)
+        assert_pairs_equal(got, want, f"C1 row_order=1 MAX_P={max_p}")
+
+
+def test_row_order_needs_and_masks(c1):
+    with pytest.raises(tmb.TagMatchError):
+        tmb.Database(c1.db, c1.key_off, c1.keys, tile_filter=0, row_order=1)
+
+
 @pytest.mark.parametrize("max_p", [200_000, 1000, 64, 1])
 def test_c1_metamorphic_max_partition(c1, max_p):
     """The result is invariant under MAX_P (partitioning is lossless)."""
@@ -121,23 +139,34 @@ def test_partition_table_matches_oracle_alg1(c1, max_p):
             assert np.array_equal(got, want), p  # members, lexicographically sorted
 
 
-def test_c2_full_parity():
+@pytest.fixture(scope="module")
+def c2():
+    return tmgen.config("C2")
+
+
+@pytest.fixture(scope="module")
+def c2_oracle(c2):
+    return {u: oracle_pairs(c2, u, brute=False, max_p=50_000) for u in (False, True)}
+
+
+@pytest.mark.parametrize("layout", [(0, 0), (1, 1)], ids=["paper", "balanced"])
+def test_c2_full_parity(c2, c2_oracle, layout):
     """BASELINE config 1: 1M sets, 100k queries, MAX_P = 200K; the oracle
-    uses MAX_P = 50K so no partitioning misreading can hide."""
-    wl = tmgen.config("C2")
-    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition) as db:
+    uses MAX_P = 50K so no partitioning misreading can hide.  Both layouts:
+    lexicographic + Alg. 4 prefix, and balanced splits + AND masks."""
+    wl = c2
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=layout[0],
+                      row_order=layout[1]) as db:
         for unique in (False, True):
             got = db.match_batch(wl.queries, unique)
-            want = oracle_pairs(wl, unique, brute=False, max_p=50_000)
-            assert_pairs_equal(got, want, f"C2 unique={unique}")
-        st = db.stats()
+            assert_pairs_equal(got, c2_oracle[unique], f"C2 unique={unique}")
     # every query matches at least its base set (PAPER.md:282)
     assert np.unique(got[0]).size == wl.queries.n_sets
 
 
-def test_c2_sampled_against_brute_force():
+def test_c2_sampled_against_brute_force(c2):
     """The partitioned oracle is itself pinned to brute force on a query sample."""
-    wl = tmgen.config("C2")
+    wl = c2
     rnd = np.random.default_rng(12)
     qsel = np.sort(rnd.choice(wl.queries.n_sets, 512, replace=False))
     want = oracle_pairs(wl, False, qsel=qsel, brute=True)
