@@ -178,6 +178,7 @@ __global__ void k_items(const unsigned long long *__restrict__ word_off, uint32_
 constexpr int kBlockTiles = 8;   // tiles per level-A block (256 rows)
 constexpr int kSubB = 128;       // level-B survivors buffered per pass
 constexpr int kQSub = 128;       // queries per unit
+constexpr int kSmallBatch = 8;   // batches up to this size take the unfiltered streaming path
 
 struct ScanSmem {
     uint64_t q0[kChunk], q1[kChunk], q2[kChunk];  // the item's query batch (SoA)
@@ -337,6 +338,51 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
             sm.q2[i] = __ldg(p.q2 + q);
         }
         __syncthreads();
+
+        if (nq <= (uint32_t)kSmallBatch) {
+            // Small batch (a lightly loaded partition, a latency-bound call, the HBM sweep):
+            // the pre-filter cannot pay off, so each warp streams 64-row units (two rows per
+            // lane, all loads issued up front) and checks every row against every query on all
+            // three blocks -- the HBM-bound regime of the scan.
+            const uint32_t vend = min(real_end, rhi);
+            const uint32_t nunit = (rhi - rlo + 63) / 64;
+            for (;;) {
+                uint32_t u = 0;
+                if (lane == 0) u = atomicAdd(&sm.unit_ctr, 1u);
+                u = __shfl_sync(0xffffffffu, u, 0);
+                if (u >= nunit) break;
+                const uint32_t ra = rlo + u * 64 + lane, rb = ra + 32;
+                uint64_t a0 = __ldg(p.w0 + ra), a1 = __ldg(p.w1 + ra), a2 = __ldg(p.w2 + ra);
+                uint64_t b0 = ~0ULL, b1 = ~0ULL, b2 = ~0ULL;
+                if (rb < rhi) {
+                    b0 = __ldg(p.w0 + rb);
+                    b1 = __ldg(p.w1 + rb);
+                    b2 = __ldg(p.w2 + rb);
+                }
+                const bool va = ra < vend, vb = rb < vend;
+                for (uint32_t j = 0; j < nq; ++j) {
+                    const uint64_t q0 = sm.q0[j], q1 = sm.q1[j], q2 = sm.q2[j];
+                    const bool ha = va && ((a0 & ~q0) | (a1 & ~q1) | (a2 & ~q2)) == 0;
+                    const bool hb = vb && ((b0 & ~q0) | (b1 & ~q1) | (b2 & ~q2)) == 0;
+                    if (__any_sync(0xffffffffu, ha || hb)) {
+                        const uint32_t ba = __ballot_sync(0xffffffffu, ha);
+                        if (ba) {
+                            st_matched += __popc(ba);
+                            emit_keys(ha, ra, sm.qid[j], p, lane);
+                        }
+                        const uint32_t bb = __ballot_sync(0xffffffffu, hb);
+                        if (bb) {
+                            st_matched += __popc(bb);
+                            emit_keys(hb, rb, sm.qid[j], p, lane);
+                        }
+                    }
+                }
+                const uint32_t u0 = rlo + u * 64;
+                st_checks += (unsigned long long)nq * (vend > u0 ? min(64u, vend - u0) : 0u);
+            }
+            __syncthreads();
+            continue;
+        }
 
         const uint32_t ntile = (rhi - rlo) / kTile;
         const uint32_t nblock = (ntile + kBlockTiles - 1) / kBlockTiles;

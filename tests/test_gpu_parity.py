@@ -111,6 +111,20 @@ def test_row_order_needs_and_masks(c1):
         tmb.Database(c1.db, c1.key_off, c1.keys, tile_filter=0, row_order=1)
 
 
+@pytest.mark.parametrize("nq", [1, 3, 8, 9, 40])
+@pytest.mark.parametrize("max_p", [0xFFFFFFFF, 500])
+def test_small_batches(c1, nq, max_p):
+    """Batches of <= 8 routed queries take the unfiltered streaming path; 9 and
+    40 straddle it (per partition)."""
+    qsel = np.arange(0, c1.queries.n_sets, c1.queries.n_sets // nq)[:nq]
+    q = c1.queries.subset(qsel)
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=max_p) as db:
+        for unique in (False, True):
+            got = db.match_batch(q, unique)
+            want = o2.match_brute(o2.encode(c1.db), c1.key_off, c1.keys, o2.encode(q), unique)
+            assert_pairs_equal(got, want, f"nq={nq}")
+
+
 @pytest.mark.parametrize("max_p", [200_000, 1000, 64, 1])
 def test_c1_metamorphic_max_partition(c1, max_p):
     """The result is invariant under MAX_P (partitioning is lossless)."""
