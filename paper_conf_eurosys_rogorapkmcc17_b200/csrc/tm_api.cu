@@ -340,6 +340,12 @@ std::vector<uint32_t> assign_shards(const std::vector<Partition> &parts, uint32_
 
 void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys) {
     auto t0 = std::chrono::steady_clock::now();
+    const bool trace = getenv("TM_TRACE_BUILD") != nullptr;
+    auto mark = [&](const char *what) {
+        if (trace)
+            fprintf(stderr, "[tm_build] %-28s %9.1f ms\n", what,
+                    std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    };
     cudaStream_t s = db->stream;
     const uint64_t N = sets->n_sets;
     // keys
@@ -406,6 +412,13 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
         d_sorted.ensure(N * 24);
         uint64_t *s0 = d_sorted.as<uint64_t>(), *s1 = s0 + N, *s2 = s1 + N;
         TMCK(launch_gather_planes(w0, w1, w2, d_idx.as<uint32_t>(), N, s0, s1, s2, s));
+        if (!getenv("TM_BUILD_HOST")) {  // consolidate on the GPU (default)
+            d_planes.release();
+            build_gpu(db, N, s0, s1, s2, d_idx.as<uint32_t>(), key_off, keys, mark);
+            mark("done");
+            db->build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+            return;
+        }
         std::vector<uint64_t> hs(3 * N);
         TMCK(cudaMemcpyAsync(hs.data(), d_sorted.p, N * 24, cudaMemcpyDeviceToHost, s));
         TMCK(cudaMemcpyAsync(h_idx.data(), d_idx.p, N * 4, cudaMemcpyDeviceToHost, s));
@@ -425,11 +438,14 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
     const uint64_t U = usig.size();
     db->n_unique = U;
 
+    mark("encode+sort+unique");
     // S0c: Algorithm 1 over the distinct signatures
     std::vector<uint32_t> order;
     std::vector<Partition> parts;
     alg1_partition(usig.data(), U, db->cfg.max_partition, order, parts);
+    mark("alg1");
     if (db->cfg.row_order == 1) refine_order(usig.data(), order, parts, 8);
+    mark("row order");
     db->n_parts_total = parts.size();
     const std::vector<uint32_t> owner = assign_shards(parts, std::max(1u, db->cfg.n_shards));
 
@@ -483,6 +499,7 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
             for (int w = 0; w < 3; ++w) ht[w * ntiles + rr / kTile] &= hp[w * rows + rr];
     }
 
+    mark("layout");
     db->planes.ensure(std::max<uint64_t>(rows, 1) * 24);
     db->tand.ensure(std::max<uint64_t>(ntiles, 1) * 24);
     if (ntiles) TMCK(cudaMemcpyAsync(db->tand.p, ht.data(), ntiles * 24, cudaMemcpyHostToDevice, s));
@@ -500,6 +517,7 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
     }
     TMCK(cudaMemcpyAsync(db->part_row.p, db->h_part_row.data(), (P + 1) * 4, cudaMemcpyHostToDevice, s));
     TMCK(cudaStreamSynchronize(s));
+    mark("upload");
     db->build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
 }
 

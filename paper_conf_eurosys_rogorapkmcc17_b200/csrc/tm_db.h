@@ -4,6 +4,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <functional>
 #include <new>
 #include <string>
 #include <vector>
@@ -120,6 +121,10 @@ void check_tagsets_device(const tm_tagsets *t);
 int bits_for(uint64_t n);
 std::vector<uint32_t> assign_shards(const std::vector<Partition> &parts, uint32_t n_shards);
 void shard_destroy(tm_db *db);
+// consolidate() on the GPU (tm_build.cu): distinct signatures, Alg. 1, row order, table, masks, keys
+void build_gpu(tm_db *db, uint64_t N, const uint64_t *s0, const uint64_t *s1, const uint64_t *s2,
+               const uint32_t *idx, const uint64_t *h_key_off, const uint32_t *h_keys,
+               const std::function<void(const char *)> &mark);
 }  // namespace tmb
 
 #define TM_API_BEGIN \

@@ -163,6 +163,32 @@ def c2_oracle(c2):
     return {u: oracle_pairs(c2, u, brute=False, max_p=50_000) for u in (False, True)}
 
 
+@pytest.mark.parametrize("max_p,row_order", [(500, 0), (2000, 1), (1, 0), (0xFFFFFFFF, 1), (64, 1)])
+def test_gpu_build_equals_host_build(c1, max_p, row_order, monkeypatch):
+    """consolidate() on the GPU (tm_build.cu, depth-synchronous Alg. 1) builds the
+    same table as the host implementation (FIFO queue): partitions in the same
+    order, same masks, same rows in the same order."""
+    def table(host):
+        if host:
+            monkeypatch.setenv("TM_BUILD_HOST", "1")
+        else:
+            monkeypatch.delenv("TM_BUILD_HOST", raising=False)
+        with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=max_p, tile_filter=1,
+                          row_order=row_order) as db:
+            masks, sizes = db.partitions()
+            sigs = [db.partition_sigs(p, int(sizes[p])) for p in range(sizes.size)]
+            st = db.stats()
+            q, k = db.match_batch(c1.queries, False)
+        return masks, sizes, sigs, st, q, k
+    gm, gs, gsig, gst, gq, gk = table(False)
+    hm, hs, hsig, hst, hq, hk = table(True)
+    assert np.array_equal(gm, hm) and np.array_equal(gs, hs)
+    assert all(np.array_equal(a, b) for a, b in zip(gsig, hsig))
+    for k_ in ("n_unique", "n_rows", "n_entries", "n_partitions"):
+        assert gst[k_] == hst[k_], k_
+    assert np.array_equal(gq, hq) and np.array_equal(gk, hk)
+
+
 @pytest.mark.parametrize("layout", [(0, 0), (1, 1)], ids=["paper", "balanced"])
 def test_c2_full_parity(c2, c2_oracle, layout):
     """BASELINE config 1: 1M sets, 100k queries, MAX_P = 200K; the oracle
