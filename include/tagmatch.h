@@ -272,6 +272,52 @@ tm_status tm_comm_init(tm_db *db, const void *id, uint64_t len, int nranks, int 
 tm_status tm_match_batch_sharded_device(tm_db *db, const tm_tagsets *queries, int unique, tm_dev_pairs *out,
                                         void *stream);
 
+/* ----------------------------------------------------------- streaming --- */
+/*
+ * Streaming front-end with batch timeout: queries are
+ * submitted one at a time; a dispatcher thread closes the open batch when it
+ * holds max_batch queries or its oldest query has waited timeout_us (0 = no
+ * timeout), runs it through tm_match_batch while the next batch fills, and
+ * publishes per-batch results.  One stream per tm_db; the stream owns the
+ * handle's calls while open (do not call tm_match_batch* concurrently).
+ */
+typedef struct tm_stream tm_stream;
+
+typedef struct {
+    uint32_t max_batch;  /* dispatch when this many queries are waiting (> 0)        */
+    uint32_t timeout_us; /* dispatch when the oldest has waited this long (0 = never) */
+    int32_t unique;      /* 0 = match, 1 = match-unique                               */
+    uint32_t reserved;   /* must be 0                                                 */
+} tm_stream_config;
+
+/* One dispatched batch: query i of the batch has ticket tickets[i] and keys
+ * keys[key_off[i] .. key_off[i+1]) (sorted); times are steady-clock ns.
+ * Owned by the library until tm_stream_result_free. */
+typedef struct {
+    uint64_t n_queries;
+    const uint64_t *tickets;
+    const uint64_t *submit_ns;
+    const uint64_t *key_off;
+    const uint32_t *keys;
+    uint64_t dispatch_ns, done_ns;
+    void *priv_;
+} tm_stream_result;
+
+tm_status tm_stream_open(tm_db *db, const tm_stream_config *cfg, tm_stream **out);
+/* one query: n_tags tag strings bytes[tag_off[t] .. tag_off[t+1]); *ticket = its id */
+tm_status tm_stream_submit(tm_stream *st, const uint8_t *bytes, const uint64_t *tag_off, uint64_t n_tags,
+                           uint64_t *ticket);
+/* next completed batch (n_queries = 0 if none); wait = 1 blocks until one is ready
+ * or nothing is in flight.  Errors of a failed batch are returned here. */
+tm_status tm_stream_poll(tm_stream *st, int wait, tm_stream_result *out);
+void tm_stream_result_free(tm_stream_result *r);
+/* dispatch the open batch now and wait until every submitted query is published */
+tm_status tm_stream_flush(tm_stream *st);
+/* open-loop load generator (test / experiment hook): submits query i of q (host
+ * arrays) at arrival_ns[i] after the call starts; returns when all are submitted */
+tm_status tm_stream_replay(tm_stream *st, const tm_tagsets *q, const uint64_t *arrival_ns);
+void tm_stream_close(tm_stream *st); /* dispatches what is open, joins the thread, frees */
+
 #ifdef __cplusplus
 }
 #endif

@@ -7,7 +7,7 @@
 // Algorithm 1 is processed level by level: the FIFO queue of PAPER.md:120 visits
 // the nodes of each tree depth in order, children pushed as (P0, P1), so
 // processing a whole depth at once accepts partitions in exactly the FIFO order
-// (tested against oracle/o2.c's literal FIFO implementation).  Each node is a
+// (the tests compare it with a literal FIFO implementation).  Each node is a
 // contiguous range of a permutation that is split stably, so members stay in
 // lexicographic order unless the row-order refinement reorders them.
 #include <cub/cub.cuh>

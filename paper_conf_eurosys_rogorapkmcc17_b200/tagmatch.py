@@ -50,6 +50,18 @@ class tm_dev_pairs(ctypes.Structure):
     _fields_ = [("n", ctypes.c_uint64), ("query", ctypes.c_void_p), ("key", ctypes.c_void_p)]
 
 
+class tm_stream_config(ctypes.Structure):
+    _fields_ = [("max_batch", ctypes.c_uint32), ("timeout_us", ctypes.c_uint32), ("unique", ctypes.c_int32),
+                ("reserved", ctypes.c_uint32)]
+
+
+class tm_stream_result(ctypes.Structure):
+    _fields_ = [("n_queries", ctypes.c_uint64), ("tickets", ctypes.POINTER(ctypes.c_uint64)),
+                ("submit_ns", ctypes.POINTER(ctypes.c_uint64)), ("key_off", ctypes.POINTER(ctypes.c_uint64)),
+                ("keys", ctypes.POINTER(ctypes.c_uint32)), ("dispatch_ns", ctypes.c_uint64),
+                ("done_ns", ctypes.c_uint64), ("priv_", ctypes.c_void_p)]
+
+
 class tm_stats_t(ctypes.Structure):
     _fields_ = [(n, ctypes.c_uint64) for n in
                 ("n_sets", "n_entries", "n_unique", "n_rows", "n_partitions", "n_partitions_total")] + \
@@ -67,7 +79,9 @@ class tm_stats_t(ctypes.Structure):
 EXPORTS = ["tm_build", "tm_match_batch", "tm_match_batch_device", "tm_pairs_free", "tm_free", "tm_strerror",
            "tm_last_error", "tm_abi_version", "tm_encode", "tm_stats", "tm_partitions", "tm_partition_sigs",
            "tm_owner_range", "tm_shard_plan", "tm_partition_host", "tm_last_result", "tm_shard_counts",
-           "tm_shard_merge", "tm_nccl_unique_id", "tm_comm_init", "tm_match_batch_sharded_device"]
+           "tm_shard_merge", "tm_nccl_unique_id", "tm_comm_init", "tm_match_batch_sharded_device",
+           "tm_stream_open", "tm_stream_submit", "tm_stream_poll", "tm_stream_result_free", "tm_stream_flush",
+           "tm_stream_replay", "tm_stream_close"]
 
 _lib = None
 
@@ -114,6 +128,15 @@ def load(path: str = LIB_PATH):
                        ("tm_match_batch_sharded_device", [vp, P(tm_tagsets), i32, P(tm_dev_pairs), vp])]:
         getattr(L, name).restype = ctypes.c_int
         getattr(L, name).argtypes = args
+    for name, args in [("tm_stream_open", [vp, P(tm_stream_config), P(vp)]),
+                       ("tm_stream_submit", [vp, vp, vp, u64, P(ctypes.c_uint64)]),
+                       ("tm_stream_poll", [vp, i32, P(tm_stream_result)]),
+                       ("tm_stream_flush", [vp]),
+                       ("tm_stream_replay", [vp, P(tm_tagsets), vp])]:
+        getattr(L, name).restype = ctypes.c_int
+        getattr(L, name).argtypes = args
+    L.tm_stream_result_free.argtypes = [P(tm_stream_result)]
+    L.tm_stream_close.argtypes = [vp]
     _lib = L
     return L
 
@@ -327,3 +350,62 @@ def nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(load().tm_nccl_unique_id(buf, 128))
     return buf.raw
+
+
+# -------------------------------------------------------------- streaming --
+class Stream:
+    """tm_stream: one-query submissions batched by size or timeout."""
+
+    def __init__(self, db: Database, max_batch: int, timeout_us: int, unique: bool):
+        cfg = tm_stream_config(max_batch, timeout_us, int(bool(unique)), 0)
+        h = ctypes.c_void_p()
+        _check(load().tm_stream_open(db.h, ctypes.byref(cfg), ctypes.byref(h)))
+        self.h = h
+        self._db = db
+
+    def submit(self, tags: list[bytes]) -> int:
+        b = b"".join(tags)
+        off = np.zeros(len(tags) + 1, np.uint64)
+        off[1:] = np.cumsum([len(t) for t in tags]) if tags else []
+        buf = np.frombuffer(b, np.uint8) if b else np.zeros(1, np.uint8)
+        t = ctypes.c_uint64()
+        _check(load().tm_stream_submit(self.h, _ptr(buf), _ptr(off), len(tags), ctypes.byref(t)))
+        return t.value
+
+    def replay(self, queries, arrival_ns: np.ndarray):
+        q = queries if isinstance(queries, HostTagSets) else HostTagSets.of(queries)
+        arr = np.ascontiguousarray(arrival_ns, dtype=np.uint64)
+        _check(load().tm_stream_replay(self.h, ctypes.byref(q.c), _ptr(arr)))
+
+    def flush(self):
+        _check(load().tm_stream_flush(self.h))
+
+    def poll(self, wait: bool = True):
+        """Next completed batch as a dict of numpy arrays, or None."""
+        r = tm_stream_result()
+        _check(load().tm_stream_poll(self.h, int(bool(wait)), ctypes.byref(r)))
+        if r.n_queries == 0:
+            return None
+        n = r.n_queries
+        try:
+            ko = np.ctypeslib.as_array(r.key_off, shape=(n + 1,)).copy()
+            out = {"tickets": np.ctypeslib.as_array(r.tickets, shape=(n,)).copy(),
+                   "submit_ns": np.ctypeslib.as_array(r.submit_ns, shape=(n,)).copy(),
+                   "key_off": ko,
+                   "keys": np.ctypeslib.as_array(r.keys, shape=(int(ko[-1]),)).copy() if ko[-1] else
+                   np.zeros(0, np.uint32),
+                   "dispatch_ns": r.dispatch_ns, "done_ns": r.done_ns}
+        finally:
+            load().tm_stream_result_free(ctypes.byref(r))
+        return out
+
+    def close(self):
+        if getattr(self, "h", None):
+            load().tm_stream_close(self.h)
+            self.h = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

@@ -300,3 +300,47 @@ def test_device_entry_point_matches_host(c1):
             gq = torch.as_tensor(_CAI(out.query, out.n), device="cuda").cpu().numpy().view(np.uint32)
             gk = torch.as_tensor(_CAI(out.key, out.n), device="cuda").cpu().numpy().view(np.uint32)
             assert_pairs_equal((gq, gk), (hq, hk), f"device API unique={unique}")
+
+
+# ------------------------------------------------------------- streaming --
+@pytest.mark.parametrize("max_batch,timeout_us", [(64, 200), (1_000_000, 500), (7, 0)])
+def test_stream_one_query_at_a_time(c1, max_batch, timeout_us):
+    """tm_stream: one-query submissions, batches closed by size or
+    timeout; every query's keys equal the oracle's."""
+    from paper_conf_eurosys_rogorapkmcc17_b200.tagmatch import Stream
+    want_q, want_k = oracle_pairs(c1, True)
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=200_000) as db:
+        with Stream(db, max_batch, timeout_us, unique=True) as st:
+            tickets = [st.submit(c1.queries.strings(j)) for j in range(300)]
+            st.flush()
+            got = {}
+            while True:
+                r = st.poll(wait=False)
+                if r is None:
+                    break
+                assert r["n_queries"] if "n_queries" in r else True
+                for i, t in enumerate(r["tickets"]):
+                    got[int(t)] = r["keys"][r["key_off"][i]:r["key_off"][i + 1]]
+                assert r["done_ns"] >= r["dispatch_ns"] >= r["submit_ns"].max()
+                if max_batch < 300:
+                    assert r["tickets"].size <= max_batch
+    assert sorted(got) == tickets
+    for j in range(300):
+        assert np.array_equal(got[j], want_k[want_q == j])
+
+
+def test_stream_replay_open_loop(c1):
+    from paper_conf_eurosys_rogorapkmcc17_b200.tagmatch import Stream
+    want_q, want_k = oracle_pairs(c1, False)
+    arrivals = np.cumsum(np.random.default_rng(3).exponential(20_000, c1.queries.n_sets)).astype(np.uint64)
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=200_000) as db:
+        with Stream(db, 128, 1000, unique=False) as st:
+            st.replay(c1.queries, arrivals)
+            st.flush()
+            got = {}
+            while (r := st.poll(wait=False)) is not None:
+                for i, t in enumerate(r["tickets"]):
+                    got[int(t)] = r["keys"][r["key_off"][i]:r["key_off"][i + 1]]
+    assert sorted(got) == list(range(c1.queries.n_sets))
+    for j in range(c1.queries.n_sets):
+        assert np.array_equal(got[j], want_k[want_q == j])
