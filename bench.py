@@ -206,6 +206,7 @@ def config_block(c, args, wl):
             "max_partition": c["max_partition"], "mode": "match-unique" if args.unique else "match",
             "tile_filter": ["alg4-prefix", "tile-and", "none"][args.tile_filter],
             "row_order": ["lexicographic", "balanced-splits"][args.row_order],
+            "exact_check": bool(args.exact),
             "parallelism": (f"partition-sharded-{args.gpus} (NCCL exchange)" if args.shard else
                             f"replicated-dp{args.gpus}") if args.gpus > 1 else "single",
             "l2": "flushed between timed steps (512 MiB write)", "bloom": "192 bits, k=7 (PAPER.md:106)"}
@@ -245,7 +246,8 @@ def run_ours(args):
     Q = wl.queries.n_sets
     t0 = time.perf_counter()
     db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], device=dev,
-                      tile_filter=args.tile_filter, row_order=args.row_order, n_shards=world if sharded else 1, shard=rank if sharded else 0)
+                      tile_filter=args.tile_filter, row_order=args.row_order, exact=int(args.exact),
+                      n_shards=world if sharded else 1, shard=rank if sharded else 0)
     build_s = time.perf_counter() - t0
     if sharded:
         from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as tmx
@@ -377,7 +379,7 @@ def run_ours(args):
                           ("encode_ms", "route_ms", "scan_ms", "merge_ms", "total_ms")},
             "path_stats": {k: last[k] for k in ("n_partitions", "routed", "candidate_pairs", "tile_tests",
                                                 "pair_checks", "matched_sets", "emitted_pairs", "result_pairs",
-                                                "work_items")},
+                                                "work_items", "exact_checked", "exact_kept")},
             "build_s": build_s,
         }
         if not args.no_cpu_baseline and world == 1:
@@ -414,6 +416,8 @@ def main():
     # default layout = the B200 one (R18): balanced splits inside partitions +
     # tile AND masks; --tile-filter 0 --row-order 0 is the paper's lexicographic order + Alg. 4 prefix
     ap.add_argument("--tile-filter", type=int, default=1, choices=[0, 1, 2])
+    ap.add_argument("--exact", action="store_true",
+                    help="exact subset post-check (PAPER.md:106; removes Bloom false positives)")
     ap.add_argument("--row-order", type=int, default=1, choices=[0, 1],
                     help="1: balanced-split order inside partitions (DESIGN.md R18; needs --tile-filter 1)")
     ap.add_argument("--max-partition", type=int, default=0,

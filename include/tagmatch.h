@@ -47,7 +47,7 @@
 extern "C" {
 #endif
 
-#define TM_ABI_VERSION 1u
+#define TM_ABI_VERSION 2u
 /* Bloom filter width and number of hash functions. */
 #define TM_SIG_BITS 192u
 #define TM_SIG_WORDS 3u
@@ -112,7 +112,12 @@ typedef struct {
                                    down to groups of <= 8 sets, depth-first (R18);
                                    requires tile_filter 1 or 2 (Alg. 4's first/last prefix
                                    is only sound for lexicographic order)            */
-    uint32_t reserved[2];   /* must be 0                                               */
+    uint32_t exact;         /* 1 = exact subset post-check ("the system ...
+                               can perform an additional exact subset check"): a pair is
+                               kept only if every tag string of the entry's set occurs in
+                               the query, which removes Bloom false positives; 0 = the
+                               Bloom result (default)                                  */
+    uint32_t reserved;      /* must be 0                                               */
 } tm_config;
 
 /* Result pairs in host memory, allocated by the library (pinned), released by
@@ -200,7 +205,9 @@ typedef struct {
     uint64_t retries;          /* capacity-overflow re-runs in the last call          */
     double encode_ms, route_ms, scan_ms, merge_ms, total_ms; /* CUDA-event stage times */
     uint32_t scan_launches;    /* scan-kernel launches in the last call               */
-    uint32_t kernel_launches;  /* all library kernel launches in the last call (incl. CUB) */
+    uint32_t kernel_launches;  /* library kernel launches in the last call (CUB excluded) */
+    uint64_t exact_checked;    /* exact mode: (query, entry) Bloom matches checked      */
+    uint64_t exact_kept;       /* exact mode: ... that are exact subsets                  */
 } tm_stats_t;
 
 tm_status tm_stats(const tm_db *db, tm_stats_t *out);

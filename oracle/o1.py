@@ -146,6 +146,25 @@ def match_numpy(db_w, key_off, keys, q_w, unique: bool, qids=None):
     return np.concatenate(oq), np.concatenate(ok)
 
 
+def match_exact(db_sets: Sequence[Iterable[bytes]], key_lists: Sequence[Sequence[int]],
+                queries: Sequence[Iterable[bytes]], unique: bool) -> list[tuple[int, int]]:
+    """Exact subset matching on the tag strings themselves (s_i
+    subset of q; "an additional exact subset check"): for query j, every
+    key of every entry whose tag set is contained in the query's tag set.
+    Brute force over Python sets."""
+    sets = [frozenset(s) for s in db_sets]
+    out = []
+    for j, q in enumerate(queries):
+        qs = frozenset(q)
+        ks = []
+        for s, kl in zip(sets, key_lists):
+            if s <= qs:
+                ks.extend(kl)
+        ks = sorted(set(ks)) if unique else sorted(ks)
+        out.extend((j, k) for k in ks)
+    return out
+
+
 # ------------------------------------------------- Algorithm 1 (PAPER.md:120) --
 def alg1(sigs: Sequence[int], max_p: int) -> list[tuple[int, list[int]]]:
     """Balanced partitioning, Algorithm 1, as written, with

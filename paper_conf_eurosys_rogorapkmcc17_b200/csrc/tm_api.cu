@@ -246,6 +246,10 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         break;
     }
     uint64_t n = st.emitted_pairs;
+    if (db->cfg.exact) {  // S7': exact subset check of the (query, set) candidates, then keys
+        n = exact_filter(db, q, n, s);
+        launches += 5;
+    }
     // S8: canonical order (sort by (query, key)), merge (unique for match-unique)
     db->out_alt.ensure(std::max<uint64_t>(n, 1) * 8);
     uint64_t *sorted = db->out.as<uint64_t>();
@@ -412,9 +416,15 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
         d_sorted.ensure(N * 24);
         uint64_t *s0 = d_sorted.as<uint64_t>(), *s1 = s0 + N, *s2 = s1 + N;
         TMCK(launch_gather_planes(w0, w1, w2, d_idx.as<uint32_t>(), N, s0, s1, s2, s));
-        if (!getenv("TM_BUILD_HOST")) {  // consolidate on the GPU (default)
+        if (!getenv("TM_BUILD_HOST") || db->cfg.exact) {  // consolidate on the GPU (default)
             d_planes.release();
             build_gpu(db, N, s0, s1, s2, d_idx.as<uint32_t>(), key_off, keys, mark);
+            if (db->cfg.exact) {
+                exact_build(db, d_bytes.as<uint8_t>(), sets->n_bytes, d_voff.as<uint64_t>(), sets->n_vocab,
+                            (sets->tag_idx && sets->n_tags) ? d_tidx.as<uint32_t>() : nullptr, d_soff.as<uint64_t>(),
+                            N, sets->n_tags, key_off, keys);
+                mark("exact tables");
+            }
             mark("done");
             db->build_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
             return;
@@ -543,7 +553,9 @@ void destroy_db(tm_db *db) {
                       &db->in_voff, &db->in_tidx, &db->in_soff, &db->vsig, &db->qplanes, &db->bm, &db->word_off,
                       &db->qidx, &db->qoff, &db->item_cnt, &db->item_off, &db->out, &db->out_alt, &db->res_q,
                       &db->res_k, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,
-                      &db->mk})
+                      &db->mk, &db->xv_bytes, &db->xv_off, &db->xv_hash, &db->xv_pos, &db->xv_canon, &db->xs_off,
+                      &db->xs_ids, &db->xk_off, &db->xk_keys, &db->xq_canon, &db->xq_ids, &db->xflag, &db->xcnt,
+                      &db->xkoff, &db->xkcnt})
         b->release();
     for (auto &e : db->ev)
         if (e) cudaEventDestroy(e);
@@ -603,7 +615,8 @@ tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32
         if (cfg->row_order > 1) fail(TM_EINVAL, "row_order must be 0 or 1");
         if (cfg->row_order == 1 && cfg->tile_filter == 0)
             fail(TM_EINVAL, "row_order 1 needs tile_filter 1 or 2 (the first/last prefix needs lexicographic order)");
-        if (cfg->reserved[0] | cfg->reserved[1]) fail(TM_EINVAL, "reserved fields must be 0");
+        if (cfg->exact > 1) fail(TM_EINVAL, "exact must be 0 or 1");
+        if (cfg->reserved) fail(TM_EINVAL, "reserved fields must be 0");
     }
     const int dev = check_device(cfg ? cfg->device : -1);
     DeviceGuard g(dev);

@@ -317,7 +317,7 @@ __global__ void k_layout_rows(const uint32_t *__restrict__ row_off, const uint32
                               const uint64_t *__restrict__ u1, const uint64_t *__restrict__ u2,
                               const uint32_t *__restrict__ ustart, const uint64_t *__restrict__ ekscan,
                               uint64_t *__restrict__ w0, uint64_t *__restrict__ w1, uint64_t *__restrict__ w2,
-                              uint32_t *__restrict__ row_u, uint32_t *__restrict__ row_kc) {
+                              uint32_t *__restrict__ row_u, uint32_t *__restrict__ row_kc, int exact) {
     uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (r >= rows) return;
     uint32_t lo = 0, hi = P;
@@ -332,7 +332,8 @@ __global__ void k_layout_rows(const uint32_t *__restrict__ row_off, const uint32
         w1[r] = u1[u];
         w2[r] = u2[u];
         row_u[r] = u;
-        row_kc[r] = (uint32_t)(ekscan[ustart[u + 1]] - ekscan[ustart[u]]);
+        // keys of the row's sets, or (exact mode) the sets themselves
+        row_kc[r] = exact ? ustart[u + 1] - ustart[u] : (uint32_t)(ekscan[ustart[u + 1]] - ekscan[ustart[u]]);
     } else {  // padding row: all ones, no keys
         w0[r] = w1[r] = w2[r] = ~0ULL;
         row_u[r] = kNone;
@@ -344,7 +345,7 @@ __global__ void k_layout_rows(const uint32_t *__restrict__ row_off, const uint32
 __global__ void k_layout_keys(const uint32_t *__restrict__ row_u, const uint32_t *__restrict__ koff_rows,
                               uint64_t rows, const uint32_t *__restrict__ ustart, const uint32_t *__restrict__ idx,
                               const uint64_t *__restrict__ key_off, const uint32_t *__restrict__ keys,
-                              uint32_t *__restrict__ out) {
+                              uint32_t *__restrict__ out, int exact) {
     uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (r >= rows) return;
     const uint32_t u = row_u[r];
@@ -352,6 +353,10 @@ __global__ void k_layout_keys(const uint32_t *__restrict__ row_u, const uint32_t
     uint32_t o = koff_rows[r];
     for (uint32_t e = ustart[u]; e < ustart[u + 1]; ++e) {
         const uint32_t s = idx[e];
+        if (exact) {
+            out[o++] = s;
+            continue;
+        }
         for (uint64_t k = key_off[s]; k < key_off[s + 1]; ++k) out[o++] = keys[k];
     }
 }
@@ -688,7 +693,8 @@ void build_gpu(tm_db *db, uint64_t N, const uint64_t *s0, const uint64_t *s1, co
         k_layout_rows<<<gridn(rows, 256), 256, 0, s>>>(db->part_row.as<uint32_t>(), dlo.as<uint32_t>(),
                                                        db->part_n.as<uint32_t>(), KP, rows, perm.as<uint32_t>(), u0,
                                                        u1, u2, ustart.as<uint32_t>(), ekscan.as<uint64_t>(), w0, w1,
-                                                       w2, rowu.as<uint32_t>(), rowkc.as<uint32_t>());
+                                                       w2, rowu.as<uint32_t>(), rowkc.as<uint32_t>(),
+                                                       (int)db->cfg.exact);
         TMCK(cudaGetLastError());
         TMCK(cudaMemsetAsync(rowkc.as<uint32_t>() + rows, 0, 4, s));
         scan_excl(db, rowkc.as<uint32_t>(), db->key_off.as<uint32_t>(), rows + 1, s);
@@ -696,7 +702,8 @@ void build_gpu(tm_db *db, uint64_t N, const uint64_t *s0, const uint64_t *s1, co
         db->keys.ensure(std::max<uint64_t>(nkeys, 1) * 4);
         k_layout_keys<<<gridn(rows, 256), 256, 0, s>>>(rowu.as<uint32_t>(), db->key_off.as<uint32_t>(), rows,
                                                        ustart.as<uint32_t>(), idx, dkoff.as<uint64_t>(),
-                                                       dkeys.as<uint32_t>(), db->keys.as<uint32_t>());
+                                                       dkeys.as<uint32_t>(), db->keys.as<uint32_t>(),
+                                                       (int)db->cfg.exact);
         TMCK(cudaGetLastError());
         uint64_t *t0 = db->tand.as<uint64_t>(), *t1 = t0 + ntiles, *t2 = t1 + ntiles;
         k_tile_and<<<gridn(ntiles, 256), 256, 0, s>>>(w0, w1, w2, ntiles, t0, t1, t2);

@@ -108,6 +108,10 @@ struct tm_db {
     void *nccl_comm = nullptr;
     int nranks = 1, rank = 0;
     DevBuf xcounts, xall, xrecv, xalt, mq, mk;
+    // exact mode (tm_exact.cu)
+    uint64_t x_nvocab = 0;
+    DevBuf xv_bytes, xv_off, xv_hash, xv_pos, xv_canon, xs_off, xs_ids, xk_off, xk_keys;
+    DevBuf xq_canon, xq_ids, xflag, xcnt, xkoff, xkcnt;
     tm_stats_t st{};
 };
 
@@ -121,6 +125,11 @@ void check_tagsets_device(const tm_tagsets *t);
 int bits_for(uint64_t n);
 std::vector<uint32_t> assign_shards(const std::vector<Partition> &parts, uint32_t n_shards);
 void shard_destroy(tm_db *db);
+// exact subset post-check (tm_exact.cu)
+void exact_build(tm_db *db, const uint8_t *d_bytes, uint64_t n_bytes, const uint64_t *d_voff, uint64_t V,
+                 const uint32_t *d_tidx, const uint64_t *d_soff, uint64_t N, uint64_t n_tags,
+                 const uint64_t *h_key_off, const uint32_t *h_keys);
+uint64_t exact_filter(tm_db *db, const tm_tagsets *q, uint64_t n, cudaStream_t s);
 // consolidate() on the GPU (tm_build.cu): distinct signatures, Alg. 1, row order, table, masks, keys
 void build_gpu(tm_db *db, uint64_t N, const uint64_t *s0, const uint64_t *s1, const uint64_t *s2,
                const uint32_t *idx, const uint64_t *h_key_off, const uint32_t *h_keys,

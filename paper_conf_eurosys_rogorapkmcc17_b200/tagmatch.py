@@ -38,7 +38,7 @@ class tm_tagsets(ctypes.Structure):
 class tm_config(ctypes.Structure):
     _fields_ = [("max_partition", ctypes.c_uint32), ("device", ctypes.c_int32), ("n_shards", ctypes.c_uint32),
                 ("shard", ctypes.c_uint32), ("tile_filter", ctypes.c_uint32), ("row_order", ctypes.c_uint32),
-                ("reserved", ctypes.c_uint32 * 2)]
+                ("exact", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
 
 
 class tm_pairs(ctypes.Structure):
@@ -70,7 +70,8 @@ class tm_stats_t(ctypes.Structure):
                 ("n_queries", "routed", "candidate_pairs", "tile_tests", "pair_checks", "matched_sets",
                  "emitted_pairs", "result_pairs", "work_items", "retries")] + \
                [(n, ctypes.c_double) for n in ("encode_ms", "route_ms", "scan_ms", "merge_ms", "total_ms")] + \
-               [("scan_launches", ctypes.c_uint32), ("kernel_launches", ctypes.c_uint32)]
+               [("scan_launches", ctypes.c_uint32), ("kernel_launches", ctypes.c_uint32),
+                ("exact_checked", ctypes.c_uint64), ("exact_kept", ctypes.c_uint64)]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
@@ -176,7 +177,8 @@ def device_tagsets(vocab_bytes_ptr, vocab_off_ptr, tag_idx_ptr, set_off_ptr, n_b
                       n_bytes, n_vocab, n_tags, n_sets)
 
 
-def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0, row_order=0) -> tm_config:
+def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0, row_order=0,
+                exact=0) -> tm_config:
     c = tm_config()
     c.max_partition = max_partition
     c.device = device
@@ -184,6 +186,7 @@ def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0, 
     c.shard = shard
     c.tile_filter = tile_filter
     c.row_order = row_order
+    c.exact = exact
     return c
 
 
@@ -191,12 +194,12 @@ class Database:
     """A tm_db handle: tm_build on construction, tm_free on close()."""
 
     def __init__(self, sets, key_off=None, keys=None, max_partition=0, device=-1, n_shards=1, shard=0,
-                 tile_filter=0, row_order=0):
+                 tile_filter=0, row_order=0, exact=0):
         L = load()
         self._sets = sets if isinstance(sets, HostTagSets) else HostTagSets.of(sets)
         self._ko = None if key_off is None else np.ascontiguousarray(key_off, dtype=np.uint64)
         self._ks = np.ascontiguousarray(keys if keys is not None else np.zeros(0), dtype=np.uint32)
-        cfg = make_config(max_partition, device, n_shards, shard, tile_filter, row_order)
+        cfg = make_config(max_partition, device, n_shards, shard, tile_filter, row_order, exact)
         h = ctypes.c_void_p()
         _check(L.tm_build(ctypes.byref(self._sets.c), _ptr(self._ko), _ptr(self._ks) if self._ks.size else None,
                           ctypes.byref(cfg), ctypes.byref(h)))

@@ -344,3 +344,67 @@ def test_stream_replay_open_loop(c1):
     assert sorted(got) == list(range(c1.queries.n_sets))
     for j in range(c1.queries.n_sets):
         assert np.array_equal(got[j], want_k[want_q == j])
+
+
+# ------------------------------------------------------------ exact mode --
+def _exact_oracle(db_strings, key_lists, q_strings, unique, db_sig, q_sig):
+    """Exact containment on strings, evaluated on the Bloom candidates only
+    (sound: exact containment implies Bloom containment, pinned in
+    tests/test_oracle_pins.py)."""
+    sets = [frozenset(s) for s in db_strings]
+    out = []
+    for j in range(len(q_strings)):
+        qs = frozenset(q_strings[j])
+        cand = np.nonzero(((db_sig[:, 0] & ~q_sig[j, 0]) | (db_sig[:, 1] & ~q_sig[j, 1]) |
+                           (db_sig[:, 2] & ~q_sig[j, 2])) == 0)[0]
+        ks = [k for i in cand if sets[i] <= qs for k in key_lists[i]]
+        ks = sorted(set(ks)) if unique else sorted(ks)
+        out.extend((j, k) for k in ks)
+    return out
+
+
+@pytest.mark.parametrize("unique", [False, True])
+def test_exact_mode_removes_false_positives(unique):
+    """Dense queries over a 50-tag vocabulary produce many Bloom false
+    positives; exact mode returns exactly the string-level containment."""
+    rnd = random.Random(8)
+    vocab = [f"w{i}".encode() for i in range(50)] + [b"", b"\x00\xff"]
+    sets = [[rnd.choice(vocab) for _ in range(rnd.randint(0, 4))] for _ in range(3000)]
+    sets += [[b"w1", b"w1"], [b"w2", b"w1"]]
+    keys = [[rnd.randrange(1000) for _ in range(rnd.randint(0, 2))] for _ in range(len(sets))]
+    queries = [[rnd.choice(vocab) for _ in range(rnd.randint(10, 40))] for _ in range(200)]
+    queries += [[], [b"zz"], vocab]
+    key_off = np.zeros(len(keys) + 1, np.uint64)
+    key_off[1:] = np.cumsum([len(k) for k in keys])
+    flat = np.array([k for kl in keys for k in kl], np.uint32)
+    want = o1.match_exact(sets, keys, queries, unique)
+    bloom = o1.match([o1.encode(s) for s in sets], keys, [o1.encode(q) for q in queries], unique)
+    assert len(bloom) > len(want)          # the workload does have false positives
+    for max_p in (0xFFFFFFFF, 100, 1):
+        with tmb.Database(tagsets(sets), key_off, flat, max_partition=max_p, exact=1) as db:
+            gq, gk = db.match_batch(tagsets(queries), unique)
+            st = db.stats()
+        assert list(zip(gq.tolist(), gk.tolist())) == want
+        assert st["exact_kept"] <= st["exact_checked"]
+
+
+def test_exact_mode_duplicate_vocabulary_strings():
+    """Vocabulary entries with identical bytes are one tag (canonical ids)."""
+    vb = np.frombuffer(b"aabbaa", np.uint8)
+    vo = np.array([0, 2, 4, 6], np.uint64)            # "aa", "bb", "aa"
+    db_ts = tmgen.TagSets(vb, vo, np.array([0, 1, 2], np.uint32), np.array([0, 2, 3], np.uint64))
+    q_ts = tagsets([[b"aa", b"bb"], [b"aa"], [b"bb"]])
+    with tmb.Database(db_ts, keys=np.array([5, 6], np.uint32), exact=1) as db:
+        q, k = db.match_batch(q_ts, False)
+    assert list(zip(q.tolist(), k.tolist())) == [(0, 5), (0, 6), (1, 6)]
+
+
+@pytest.mark.parametrize("unique", [False, True])
+def test_exact_mode_c1(c1, unique):
+    db_strings = [c1.db.strings(i) for i in range(c1.db.n_sets)]
+    q_strings = [c1.queries.strings(j) for j in range(c1.queries.n_sets)]
+    key_lists = [c1.keys[c1.key_off[i]:c1.key_off[i + 1]].tolist() for i in range(c1.db.n_sets)]
+    want = _exact_oracle(db_strings, key_lists, q_strings, unique, o2.encode(c1.db), o2.encode(c1.queries))
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=500, tile_filter=1, row_order=1, exact=1) as db:
+        gq, gk = db.match_batch(c1.queries, unique)
+    assert list(zip(gq.tolist(), gk.tolist())) == want

@@ -298,3 +298,16 @@ def test_tile_prefix_hand_example_and_soundness():
             tile.sort()
             pre = o1.tile_prefix(tile[0], tile[-1])
             assert all(o1.subset(pre, s) for s in tile)
+
+
+def test_match_exact_definition():
+    """O1.match_exact is plain set containment; on the tiny universe it is the
+    Bloom result minus the false positives (soundness)."""
+    vocab, sets, queries, keys = _tiny_universe(41, n_vocab=30, n_sets=800, n_q=120)
+    ds = [[vocab[t] for t in s] for s in sets]
+    qs = [[vocab[t] for t in q] for q in queries]
+    ex = o1.match_exact(ds, keys, qs, False)
+    bl = o1.match([o1.encode(s) for s in ds], keys, [o1.encode(q) for q in qs], False)
+    want = sorted((j, k) for j, q in enumerate(queries) for i, s in enumerate(sets) if s <= q for k in keys[i])
+    assert ex == want
+    assert set(ex) <= set(bl)
