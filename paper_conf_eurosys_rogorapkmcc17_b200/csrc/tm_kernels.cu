@@ -287,7 +287,12 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // kSubB per pass, block 2 checked on a hit; FULL3 = true: two 16-B entries
 // (blocks 0, 1 | block 2, slot) per survivor, up to kSubB / 2 per pass, all
 // three blocks checked in the main loop.  U = survivors per loop iteration.
-template <int U, bool FULL3>
+// UNION2 (with FULL3 = false): survivors are first tested in pairs against the
+// OR of the pair's blocks 0-1 (a necessary condition: s within a implies s
+// within a|b), and individually only when some lane passes the pair test --
+// about 1 pair in 9 on the Twitter-like workload, so the check loop issues
+// ~40% fewer LOP3.
+template <int U, bool FULL3, bool UNION2 = false>
 __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     ScanSmem &sm = *reinterpret_cast<ScanSmem *>(smem_raw);
@@ -301,7 +306,9 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
     uint4 *sbuf = sm.sbuf[warp];
     uint16_t *sbi = sm.sbi[warp];
     const uint32_t sb_addr = (uint32_t)__cvta_generic_to_shared(sbuf);
-    constexpr uint32_t kPiece = FULL3 ? kSubB / 2 : kSubB;   // level-B survivors per pass
+    // level-B survivors per pass (UNION2: entries [0, 80), pair unions at [80, 120))
+    constexpr uint32_t kPiece = FULL3 ? kSubB / 2 : (UNION2 ? 80 : kSubB);
+    constexpr uint32_t kUnionBase = 80;
 
     for (;;) {
         if (threadIdx.x == 0) {
@@ -490,7 +497,8 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                     st_tests += pe - pb;
                     st_checks += (unsigned long long)nb * nvalid;
                     // pad to a multiple of U with zeros (masked by k < nb below)
-                    if ((uint32_t)lane < ((U - (nb % U)) % U)) {
+                    constexpr uint32_t kPad = UNION2 ? 8 : U;
+                    if ((uint32_t)lane < ((kPad - (nb % kPad)) % kPad)) {
                         if (FULL3) {
                             sbuf[2 * (nb + lane)] = make_uint4(0, 0, 0, 0);
                             sbuf[2 * (nb + lane) + 1] = make_uint4(0, 0, 0, 0);
@@ -500,6 +508,42 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                         }
                     }
                     __syncwarp();
+                    if (UNION2) {
+                        // ---- Alg. 3 with pair unions: 4 pairs (8 survivors) per iteration
+                        const uint32_t npair = (nb + 7) / 8 * 4;
+                        for (uint32_t i = lane; i < npair; i += 32) {
+                            const uint4 x = sbuf[2 * i], y = sbuf[2 * i + 1];
+                            sbuf[kUnionBase + i] = make_uint4(x.x | y.x, x.y | y.y, x.z | y.z, x.w | y.w);
+                        }
+                        __syncwarp();
+                        for (uint32_t k = 0; k < nb; k += 8) {
+                            const uint32_t ua = sb_addr + (kUnionBase + k / 2) * 16;
+                            const uint4 u0 = lds128(ua), u1 = lds128(ua + 16), u2 = lds128(ua + 32),
+                                        u3 = lds128(ua + 48);
+                            bool hu[4];
+                            hu[0] = ((a0l & ~u0.x) | (a0h & ~u0.y) | (a1l & ~u0.z) | (a1h & ~u0.w)) == 0;
+                            hu[1] = ((a0l & ~u1.x) | (a0h & ~u1.y) | (a1l & ~u1.z) | (a1h & ~u1.w)) == 0;
+                            hu[2] = ((a0l & ~u2.x) | (a0h & ~u2.y) | (a1l & ~u2.z) | (a1h & ~u2.w)) == 0;
+                            hu[3] = ((a0l & ~u3.x) | (a0h & ~u3.y) | (a1l & ~u3.z) | (a1h & ~u3.w)) == 0;
+                            if (__any_sync(0xffffffffu, hu[0] | hu[1] | hu[2] | hu[3])) {
+#pragma unroll
+                                for (int j = 0; j < 4; ++j) {
+                                    if (!__any_sync(0xffffffffu, hu[j])) continue;
+#pragma unroll
+                                    for (int t = 0; t < 2; ++t) {
+                                        const uint32_t e = k + 2 * j + t;
+                                        if (e >= nb) continue;
+                                        const uint4 v = lds128(sb_addr + e * 16);
+                                        const bool h = ((a0l & ~v.x) | (a0h & ~v.y) | (a1l & ~v.z) | (a1h & ~v.w)) == 0;
+                                        if (__any_sync(0xffffffffu, h))
+                                            check_block2(h, sbi[e], s2, row, sm, p, lane, st_matched);
+                                    }
+                                }
+                            }
+                        }
+                        __syncwarp();
+                        continue;
+                    }
                     // ---- Alg. 3: U survivors per iteration against the warp's 32 sets
                     for (uint32_t k = 0; k < nb; k += U) {
                         bool h[U];
@@ -640,6 +684,7 @@ ScanFn scan_fn(int variant) {
         case 1: return k_scan<8, false>;
         case 2: return k_scan<4, true>;
         case 3: return k_scan<8, true>;
+        case 4: return k_scan<4, false, true>;
         default: return k_scan<4, false>;
     }
 }
@@ -647,10 +692,11 @@ ScanFn scan_fn(int variant) {
 
 int scan_variant() {
     // scan-kernel variant: 0 = 4 survivors/iteration, blocks 0-1 first (default);
-    // 1 = 8, blocks 0-1; 2 = 4, all three blocks; 3 = 8, all three blocks.  TM_SCAN_VARIANT overrides.
+    // 1 = 8, blocks 0-1; 2 = 4, all three blocks; 3 = 8, all three blocks; 4 = pair unions first.
+    // TM_SCAN_VARIANT overrides.
     const char *e = getenv("TM_SCAN_VARIANT");
     const int v = e ? atoi(e) : 0;
-    return (v >= 0 && v <= 3) ? v : 0;
+    return (v >= 0 && v <= 4) ? v : 0;
 }
 
 int scan_grid(int device) {

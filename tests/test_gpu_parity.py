@@ -408,3 +408,23 @@ def test_exact_mode_c1(c1, unique):
     with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=500, tile_filter=1, row_order=1, exact=1) as db:
         gq, gk = db.match_batch(c1.queries, unique)
     assert list(zip(gq.tolist(), gk.tolist())) == want
+
+
+def test_exact_mode_c2_sample(c2):
+    """Exact mode at C2 size on a 300-query sample: string-level containment."""
+    rng = np.random.default_rng(5)
+    qsel = np.sort(rng.choice(c2.queries.n_sets, 300, replace=False))
+    db_sig, q_sig = o2.encode(c2.db), o2.encode(c2.queries)
+    want = []
+    for j in qsel:
+        qs = frozenset(c2.queries.strings(int(j)))
+        cand = np.nonzero(((db_sig[:, 0] & ~q_sig[j, 0]) | (db_sig[:, 1] & ~q_sig[j, 1]) |
+                           (db_sig[:, 2] & ~q_sig[j, 2])) == 0)[0]
+        ks = sorted(k for i in cand if frozenset(c2.db.strings(int(i))) <= qs
+                    for k in c2.keys[c2.key_off[i]:c2.key_off[i + 1]].tolist())
+        want.extend((int(j), k) for k in ks)
+    with tmb.Database(c2.db, c2.key_off, c2.keys, max_partition=c2.max_partition, tile_filter=1, row_order=1,
+                      exact=1) as db:
+        gq, gk = db.match_batch(c2.queries, False)
+    keep = np.isin(gq, qsel)
+    assert list(zip(gq[keep].tolist(), gk[keep].tolist())) == want
