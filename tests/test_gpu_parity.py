@@ -262,6 +262,43 @@ def test_empty_inputs():
         assert q.size == 0
 
 
+@pytest.mark.parametrize("layout", [(0, 0), (1, 1)])
+def test_degenerate_databases(layout):
+    """Identical sets (one row, Alg. 1 finds no pivot: reading R7), all-empty
+    sets (the zero partition), a single set, and one set per tile boundary."""
+    rnd = random.Random(2)
+    cases = {
+        "identical": [[b"a", b"b"]] * 1000,
+        "all-empty": [[]] * 77,
+        "single": [[b"x"]],
+        "mixed-identical": [[b"a"]] * 500 + [[b"b"]] * 500 + [[]] * 3,
+        "tile-ragged": [[f"t{rnd.randrange(9)}".encode() for _ in range(rnd.randint(1, 3))] for _ in range(33)],
+    }
+    queries = [[b"a", b"b"], [b"a"], [b"b", b"x"], [], [b"t1", b"t2", b"t3", b"a", b"x"]]
+    for name, sets in cases.items():
+        keys = [[i % 7, 1000 + i] for i in range(len(sets))]
+        key_off = np.zeros(len(keys) + 1, np.uint64)
+        key_off[1:] = np.cumsum([len(k) for k in keys])
+        flat = np.array([k for kl in keys for k in kl], np.uint32)
+        for max_p in (0xFFFFFFFF, 200_000, 10, 1):
+            for unique in (False, True):
+                want = o1.match([o1.encode(x) for x in sets], keys, [o1.encode(q) for q in queries], unique)
+                with tmb.Database(tagsets(sets), key_off, flat, max_partition=max_p, tile_filter=layout[0],
+                                  row_order=layout[1]) as db:
+                    gq, gk = db.match_batch(tagsets(queries), unique)
+                assert list(zip(gq.tolist(), gk.tolist())) == want, (name, max_p, unique)
+
+
+def test_range_errors():
+    """Sizes beyond the u32 query / key space are rejected (TM_ERANGE)."""
+    import ctypes
+    from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as tm
+    ts = tm.HostTagSets(np.zeros(0, np.uint8), np.zeros(1, np.uint64), None, np.zeros(2, np.uint64))
+    ts.c.n_sets = 1 << 32
+    h = ctypes.c_void_p()
+    assert tm.load().tm_build(ctypes.byref(ts.c), None, None, None, ctypes.byref(h)) == -5
+
+
 def test_output_overflow_retry():
     """More pairs than the initial capacity: the library re-runs the scan."""
     sets = [[]] * 3 + [[f"t{i}".encode()] for i in range(100)]
