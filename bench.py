@@ -350,12 +350,15 @@ def run_ours(args):
         scan_s = statistics.mean(scan_ms) / 1000.0
         peak_tops = SM_COUNT * ALU_LANES_PER_SM_CLK * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
         achieved = ops / scan_s / 1e12
-        traffic = None
+        traffic, ncu = None, None
         try:
             with open(os.path.join(ROOT, "profiles", "ncu_scan_traffic.json")) as f:
                 tr = json.load(f)
                 if tr.get("config") == args.config:
                     traffic = tr.get("dram_bytes_per_launch")
+                    ncu = {k: tr.get(k) for k in ("alu_pipe_pct", "issue_active_pct", "warps_active_pct",
+                                                  "l2_hit_pct")}
+                    ncu["report"] = tr.get("report")
         except Exception:
             pass
         line = {
@@ -369,6 +372,9 @@ def run_ours(args):
                          "kernel": "k_scan", "kernel_ms": statistics.mean(scan_ms),
                          "kernel_share_of_step": statistics.mean(scan_ms) / statistics.mean(step_ms),
                          "ops_per_launch": ops,
+                         "ops_model": "3 ALU ops per decision (pre-filter test or pair check): the minimum "
+                                      "one 64-bit block test; DESIGN.md sec. 6",
+                         "ncu_same_kernel": ncu,
                          "peak_src": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM_CLK} ALU lanes/clk x "
                                      f"{peaks.get('sm_max_mhz', 1965.0)} MHz ({peak_src} sm_max_mhz)"},
             "e2e": {"value": e2e_value, "unit": "queries/s", "h2d_bytes_per_step": h2d_bytes,

@@ -77,7 +77,11 @@ def main():
         js = {"config": cfg, "report": path, "kernel": m.get("Kernel Name", ""),
               "dram_bytes_per_launch": (rd or 0) * rs + (wr or 0) * ws,
               "duration_ns": num(m.get("gpu__time_duration.sum")),
-              "duration_unit": units.get("gpu__time_duration.sum")}
+              "duration_unit": units.get("gpu__time_duration.sum"),
+              "alu_pipe_pct": num(m.get("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active")),
+              "issue_active_pct": num(m.get("smsp__issue_active.avg.pct_of_peak_sustained_active")),
+              "warps_active_pct": num(m.get("sm__warps_active.avg.pct_of_peak_sustained_active")),
+              "l2_hit_pct": num(m.get("lts__t_sector_hit_rate.pct"))}
         with open(sys.argv[sys.argv.index("--json") + 1], "w") as f:
             json.dump(js, f, indent=1)
 
