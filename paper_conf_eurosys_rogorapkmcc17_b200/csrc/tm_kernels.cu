@@ -182,10 +182,10 @@ constexpr int kSmallBatch = 8;   // batches up to this size take the unfiltered 
 
 struct ScanSmem {
     uint64_t q0[kChunk], q1[kChunk], q2[kChunk];  // the item's query batch (SoA)
-    uint32_t qid[kChunk];                          // batch slot -> query index in the call
     uint16_t sa[kScanWarps][kChunk];               // per-warp level-A survivors (slots)
     uint4 sbuf[kScanWarps][kSubB];                 // per-warp level-B survivors (see SurvivorLayout)
     uint16_t sbi[kScanWarps][kSubB];               // per-warp level-B survivors: slots
+    const uint32_t *qid;                           // batch slot -> query index in the call (global)
     unsigned long long item;
     unsigned int unit_ctr;
 };
@@ -261,7 +261,7 @@ __device__ __forceinline__ void check_block2(bool hit01, uint32_t slot, uint64_t
     const uint32_t b = __ballot_sync(0xffffffffu, m);
     if (b) {
         matched += __popc(b);
-        emit_keys(m, row, sm.qid[slot], p, lane);
+        emit_keys(m, row, __ldg(sm.qid + slot), p, lane);
     }
 }
 
@@ -336,10 +336,10 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
         const uint32_t rlo = prow + range * kRangeRows;
         const uint32_t rhi = min(rlo + (uint32_t)kRangeRows, prow + rows);
 
+        if (threadIdx.x == 0) sm.qid = p.qidx + qbeg;
         // stage the query batch (the batch of queries of partition p)
         for (uint32_t i = threadIdx.x; i < nq; i += blockDim.x) {
             const uint32_t q = __ldg(p.qidx + qbeg + i);
-            sm.qid[i] = q;
             sm.q0[i] = __ldg(p.q0 + q);
             sm.q1[i] = __ldg(p.q1 + q);
             sm.q2[i] = __ldg(p.q2 + q);
@@ -375,12 +375,12 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                         const uint32_t ba = __ballot_sync(0xffffffffu, ha);
                         if (ba) {
                             st_matched += __popc(ba);
-                            emit_keys(ha, ra, sm.qid[j], p, lane);
+                            emit_keys(ha, ra, __ldg(sm.qid + j), p, lane);
                         }
                         const uint32_t bb = __ballot_sync(0xffffffffu, hb);
                         if (bb) {
                             st_matched += __popc(bb);
-                            emit_keys(hb, rb, sm.qid[j], p, lane);
+                            emit_keys(hb, rb, __ldg(sm.qid + j), p, lane);
                         }
                     }
                 }
@@ -574,7 +574,7 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                                         const uint32_t bm = __ballot_sync(0xffffffffu, m);
                                         if (bm) {
                                             st_matched += __popc(bm);
-                                            emit_keys(m, row, sm.qid[slot[j]], p, lane);
+                                            emit_keys(m, row, __ldg(sm.qid + slot[j]), p, lane);
                                         }
                                     } else {
                                         check_block2(h[j], sbi[k + j], s2, row, sm, p, lane, st_matched);
