@@ -369,7 +369,7 @@ def run_ours(args):
             "config": config_block(c, args, wl),
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
                          "frac": achieved / peak_tops, "traffic": traffic,
-                         "kernel": "k_scan", "kernel_ms": statistics.mean(scan_ms),
+                         "kernel": f"k_scan (variant {last['scan_variant']})", "kernel_ms": statistics.mean(scan_ms),
                          "kernel_share_of_step": statistics.mean(scan_ms) / statistics.mean(step_ms),
                          "ops_per_launch": ops,
                          "ops_model": "3 ALU ops per decision (pre-filter test or pair check): the minimum "

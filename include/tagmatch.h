@@ -208,6 +208,8 @@ typedef struct {
     uint32_t kernel_launches;  /* library kernel launches in the last call (CUB excluded) */
     uint64_t exact_checked;    /* exact mode: (query, entry) Bloom matches checked      */
     uint64_t exact_kept;       /* exact mode: ... that are exact subsets                  */
+    uint32_t scan_variant;     /* scan-kernel variant of the last call */
+    uint32_t pad_;
 } tm_stats_t;
 
 tm_status tm_stats(const tm_db *db, tm_stats_t *out);

@@ -83,6 +83,11 @@ struct tm_db {
     cudaEvent_t ev[6] = {};
     tm_config cfg{};
     int scan_grid = 0;
+    // scan-kernel variant: forced by TM_SCAN_VARIANT, else tuned on the first calls by
+    // kernel ns per decision (filter tests + pair checks) between variants 0 and 2
+    int variant = 0, tune_calls = 0;
+    double tune_cost[5] = {0, 0, 0, 0, 0};
+    int grid_of[5] = {0, 0, 0, 0, 0};
     // database (device)
     uint64_t n_sets = 0, n_entries = 0, n_unique = 0, n_rows = 0, n_parts = 0, n_parts_total = 0;
     DevBuf planes;   // 3 x rows u64

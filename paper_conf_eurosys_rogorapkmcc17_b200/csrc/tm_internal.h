@@ -68,8 +68,9 @@ cudaError_t launch_route_scatter(const uint32_t *bm, const unsigned long long *w
 cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const uint32_t *part_row,
                          const uint32_t *part_n, uint32_t n_parts, unsigned long long *qoff,
                          unsigned long long *item_cnt, DevCounters *ctr, cudaStream_t s);
-cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s);
-int scan_grid(int device);
+cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant);
+int scan_grid(int device, int variant);
+int scan_variant_env();  // -1 = auto-tune
 cudaError_t launch_split(const uint64_t *pairs, uint64_t n, uint32_t *q, uint32_t *k, cudaStream_t s);
 cudaError_t launch_gather_planes(const uint64_t *src0, const uint64_t *src1, const uint64_t *src2,
                                  const uint32_t *idx, uint64_t n, uint64_t *d0, uint64_t *d1, uint64_t *d2,

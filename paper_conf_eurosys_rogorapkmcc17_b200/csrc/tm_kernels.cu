@@ -690,19 +690,20 @@ ScanFn scan_fn(int variant) {
 }
 }  // namespace
 
-int scan_variant() {
-    // scan-kernel variant: 0 = 4 survivors/iteration, blocks 0-1 first (default);
-    // 1 = 8, blocks 0-1; 2 = 4, all three blocks; 3 = 8, all three blocks; 4 = pair unions first.
-    // TM_SCAN_VARIANT overrides.
+int scan_variant_env() {
+    // TM_SCAN_VARIANT forces a scan-kernel variant: 0 = 4 survivors per
+    // iteration, blocks 0-1 first; 1 = 8, blocks 0-1; 2 = 4, all three blocks; 3 = 8, all three;
+    // 4 = pair unions first.  Unset (-1): the handle tunes between 0 and 2 on its first calls.
     const char *e = getenv("TM_SCAN_VARIANT");
-    const int v = e ? atoi(e) : 0;
-    return (v >= 0 && v <= 4) ? v : 0;
+    if (!e) return -1;
+    const int v = atoi(e);
+    return (v >= 0 && v <= 4) ? v : -1;
 }
 
-int scan_grid(int device) {
+int scan_grid(int device, int variant) {
     int sms = 0, per = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
-    ScanFn f = scan_fn(scan_variant());
+    ScanFn f = scan_fn(variant);
     cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScanSmem));
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, kScanWarps * 32, sizeof(ScanSmem));
     if (per < 1) per = 1;
@@ -710,8 +711,8 @@ int scan_grid(int device) {
     return sms * per;
 }
 
-cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s) {
-    scan_fn(scan_variant())<<<grid, kScanWarps * 32, sizeof(ScanSmem), s>>>(p);
+cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant) {
+    scan_fn(variant)<<<grid, kScanWarps * 32, sizeof(ScanSmem), s>>>(p);
     return cudaGetLastError();
 }
 
