@@ -146,6 +146,12 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
 
     db->ctr.ensure(sizeof(DevCounters));
     DevCounters *ctr = db->ctr.as<DevCounters>();
+    if (!db->wsel_ok) {  // pre-check word per row (scan variant 5), once per database
+        db->wsel.ensure(std::max<uint64_t>(db->n_rows, 1));
+        TMCK(launch_word_select(db->planes.as<uint64_t>(), db->tand.as<uint64_t>(), db->n_rows,
+                                db->wsel.as<uint8_t>(), s));
+        db->wsel_ok = true;
+    }
     TMCK(cudaEventRecord(db->ev[0], s));
 
     // S1: encode
@@ -215,8 +221,9 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         sp.cap = db->cap_out;
         sp.ctr = ctr;
         sp.filter = db->cfg.tile_filter;
+        sp.wsel = db->wsel.as<uint8_t>();
         int var = scan_variant_env();
-        if (var < 0) var = db->tune_calls < 4 ? ((db->tune_calls & 1) ? 2 : 0) : db->variant;
+        if (var < 0) var = db->tune_calls < 2 * kTuneN ? kTune[db->tune_calls % kTuneN] : db->variant;
         if (!db->grid_of[var]) db->grid_of[var] = scan_grid(db->device, var);
         db->variant = var;
         st.scan_variant = (uint32_t)var;
@@ -305,12 +312,18 @@ void finish_timing(tm_db *db, cudaStream_t s) {
     st.route_ms = ms;
     TMCK(cudaEventElapsedTime(&ms, db->ev[2], db->ev[3]));
     st.scan_ms = ms;
-    // variant tuning: qualifying calls 0-3 alternate variants 0 and 2 (0, 2, 0, 2); calls 2 and 3
-    // (warm: module loaded, buffers grown) are timed as kernel ns per decision; keep the cheaper
+    // variant tuning: qualifying calls 0 .. 2N-1 cycle through the N candidates kTune; the
+    // second round (warm: module loaded, buffers grown) is timed as kernel ns per decision;
+    // the cheapest is kept
     const double dec = (double)(st.tile_tests + st.pair_checks);
-    if (scan_variant_env() < 0 && db->tune_calls < 4 && dec > 1e6 && st.retries == 0) {
-        if (db->tune_calls >= 2) db->tune_cost[db->variant] = ms * 1e6 / dec;
-        if (++db->tune_calls == 4) db->variant = db->tune_cost[2] < db->tune_cost[0] ? 2 : 0;
+    if (scan_variant_env() < 0 && db->tune_calls < 2 * kTuneN && dec > 1e6 && st.retries == 0) {
+        if (db->tune_calls >= kTuneN) db->tune_cost[db->variant] = ms * 1e6 / dec;
+        if (++db->tune_calls == 2 * kTuneN) {
+            int best = kTune[0];
+            for (int i = 1; i < kTuneN; ++i)
+                if (db->tune_cost[kTune[i]] < db->tune_cost[best]) best = kTune[i];
+            db->variant = best;
+        }
     }
     TMCK(cudaEventElapsedTime(&ms, db->ev[3], db->ev[4]));
     st.merge_ms = ms;
@@ -561,7 +574,7 @@ void destroy_db(tm_db *db) {
         shard_destroy(db);
     } catch (...) {
     }
-    for (DevBuf *b : {&db->planes, &db->tand, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
+    for (DevBuf *b : {&db->planes, &db->tand, &db->wsel, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
                       &db->in_voff, &db->in_tidx, &db->in_soff, &db->vsig, &db->qplanes, &db->bm, &db->word_off,
                       &db->qidx, &db->qoff, &db->item_cnt, &db->item_off, &db->out, &db->out_alt, &db->res_q,
                       &db->res_k, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,

@@ -84,14 +84,16 @@ struct tm_db {
     tm_config cfg{};
     int scan_grid = 0;
     // scan-kernel variant: forced by TM_SCAN_VARIANT, else tuned on the first calls by
-    // kernel ns per decision (filter tests + pair checks) between variants 0 and 2
-    int variant = 0, tune_calls = 0;
-    double tune_cost[5] = {0, 0, 0, 0, 0};
-    int grid_of[5] = {0, 0, 0, 0, 0};
+    // kernel ns per decision (filter tests + pair checks) among kTune
+    int variant = kTune[0], tune_calls = 0;
+    double tune_cost[kScanVariants] = {};
+    int grid_of[kScanVariants] = {};
     // database (device)
     uint64_t n_sets = 0, n_entries = 0, n_unique = 0, n_rows = 0, n_parts = 0, n_parts_total = 0;
     DevBuf planes;   // 3 x rows u64
     DevBuf tand;     // 3 x (rows / 32) u64: AND of each tile's real rows
+    DevBuf wsel;     // rows u8: pre-check word per row (scan variant 5), made on first use
+    bool wsel_ok = false;
     DevBuf key_off;  // rows + 1 u32
     DevBuf keys;     // K u32
     DevBuf masks;    // P x 3 u64

@@ -24,6 +24,9 @@ constexpr int kTile = 32;  // rows per warp tile (= one warp, Alg. 4 "thread blo
 constexpr int kScanWarps = 4;      // warps per CTA
 constexpr int kChunk = 512;        // queries per work item (per-partition batch)
 constexpr int kRangeRows = 8192;    // rows per work item (multiple of 256)
+constexpr int kScanVariants = 6;    // k_scan variants (TM_SCAN_VARIANT)
+constexpr int kTune[] = {5, 2, 0};  // variants the handle times on its first calls (first = default)
+constexpr int kTuneN = 3;
 
 struct DevCounters {            // zeroed at the start of every match call
     unsigned long long n_out;   // (q,key) pairs emitted (may exceed capacity)
@@ -53,6 +56,7 @@ struct ScanParams {
     unsigned long long cap;
     DevCounters *ctr;
     uint32_t filter;                  // 0 prefix, 1 AND, 2 none
+    const uint8_t *wsel;              // [rows] pre-check word per row (variant 5)
 };
 
 // ------------------------------------------------------------ launchers --
@@ -71,6 +75,8 @@ cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const 
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant);
 int scan_grid(int device, int variant);
 int scan_variant_env();  // -1 = auto-tune
+cudaError_t launch_word_select(const uint64_t *planes, const uint64_t *tand, uint64_t rows, uint8_t *wsel,
+                               cudaStream_t s);
 cudaError_t launch_split(const uint64_t *pairs, uint64_t n, uint32_t *q, uint32_t *k, cudaStream_t s);
 cudaError_t launch_gather_planes(const uint64_t *src0, const uint64_t *src1, const uint64_t *src2,
                                  const uint32_t *idx, uint64_t n, uint64_t *d0, uint64_t *d1, uint64_t *d2,

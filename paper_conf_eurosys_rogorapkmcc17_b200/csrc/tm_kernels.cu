@@ -180,11 +180,22 @@ constexpr int kSubB = 128;       // level-B survivors buffered per pass
 constexpr int kQSub = 128;       // queries per unit
 constexpr int kSmallBatch = 8;   // batches up to this size take the unfiltered streaming path
 
+// WORD1 survivor planes: word w (= 32-bit half w & 1 of block w >> 1) of level-B
+// survivor k at sw[warp][w][k]; the plane stride (kSubW + 4 words = 400 B, 16 B mod 128)
+// puts the six planes on disjoint bank quads, so the per-lane-plane LDS.128 of the
+// pre-check is conflict-free.
+constexpr int kSubW = 96;                         // level-B survivors per pass (WORD1)
+constexpr int kSubWStride = kSubW + 4;
+
 struct ScanSmem {
     uint64_t q0[kChunk], q1[kChunk], q2[kChunk];  // the item's query batch (SoA)
     uint16_t sa[kScanWarps][kChunk];               // per-warp level-A survivors (slots)
-    uint4 sbuf[kScanWarps][kSubB];                 // per-warp level-B survivors (see SurvivorLayout)
+    union {
+        uint4 sbuf[kScanWarps][kSubB];             // per-warp level-B survivors (see SurvivorLayout)
+        uint32_t sw[kScanWarps][6][kSubWStride];   // WORD1: per-warp level-B survivors, word planes
+    };
     uint16_t sbi[kScanWarps][kSubB];               // per-warp level-B survivors: slots
+    uint64_t tmask[kScanWarps][3][kBlockTiles];    // per-warp: AND masks of the unit's tiles
     const uint32_t *qid;                           // batch slot -> query index in the call (global)
     unsigned long long item;
     unsigned int unit_ctr;
@@ -194,6 +205,40 @@ __device__ __forceinline__ uint4 lds128(uint32_t addr) {
     uint4 v;
     asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
     return v;
+}
+
+// acc |= B << j for each j in 0..3 with (a & ~v_j) == 0: one LOP3 with a predicate result and
+// one predicated OR per survivor (no SEL / add chain)
+// Two-word form: survivor j passes when (a & ~v_j) | (b & ~u_j) == 0.
+// WORD1: survivor k's six words into the per-warp word planes (stride kSubWStride), slot i
+__device__ __forceinline__ void store_survivor(uint32_t *sw, uint16_t *sbi, uint32_t k, uint64_t a0, uint64_t a1,
+                                               uint64_t a2, uint32_t i) {
+    uint32_t *c = sw + k;
+    c[0] = (uint32_t)a0;
+    c[kSubWStride] = (uint32_t)(a0 >> 32);
+    c[2 * kSubWStride] = (uint32_t)a1;
+    c[3 * kSubWStride] = (uint32_t)(a1 >> 32);
+    c[4 * kSubWStride] = (uint32_t)a2;
+    c[5 * kSubWStride] = (uint32_t)(a2 >> 32);
+    sbi[k] = (uint16_t)i;
+}
+
+// Four independent accumulators (one per survivor lane of the uint4) keep the predicated ORs
+// off a single serial dependency chain; the caller ORs them together.
+template <int B>
+__device__ __forceinline__ void precheck4x2(uint32_t &c0, uint32_t &c1, uint32_t &c2, uint32_t &c3, uint32_t a,
+                                            uint4 v, uint32_t b, uint4 u) {
+    asm("{\n\t.reg .pred p0, p1, p2, p3;\n\t.reg .b32 t0, t1, t2, t3, s0, s1, s2, s3;\n\t"
+        "not.b32 t0, %5;\n\tnot.b32 t1, %6;\n\tnot.b32 t2, %7;\n\tnot.b32 t3, %8;\n\t"
+        "and.b32 t0, t0, %4;\n\tand.b32 t1, t1, %4;\n\tand.b32 t2, t2, %4;\n\tand.b32 t3, t3, %4;\n\t"
+        "not.b32 s0, %10;\n\tnot.b32 s1, %11;\n\tnot.b32 s2, %12;\n\tnot.b32 s3, %13;\n\t"
+        "and.b32 s0, s0, %9;\n\tand.b32 s1, s1, %9;\n\tand.b32 s2, s2, %9;\n\tand.b32 s3, s3, %9;\n\t"
+        "or.b32 t0, t0, s0;\n\tor.b32 t1, t1, s1;\n\tor.b32 t2, t2, s2;\n\tor.b32 t3, t3, s3;\n\t"
+        "setp.eq.u32 p0, t0, 0;\n\tsetp.eq.u32 p1, t1, 0;\n\tsetp.eq.u32 p2, t2, 0;\n\tsetp.eq.u32 p3, t3, 0;\n\t"
+        "@p0 or.b32 %0, %0, %14;\n\t@p1 or.b32 %1, %1, %15;\n\t@p2 or.b32 %2, %2, %16;\n\t@p3 or.b32 %3, %3, %17;\n\t}"
+        : "+r"(c0), "+r"(c1), "+r"(c2), "+r"(c3)
+        : "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"(b), "r"(u.x), "r"(u.y), "r"(u.z), "r"(u.w), "n"(B),
+          "n"(B << 1), "n"(B << 2), "n"(B << 3));
 }
 
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
@@ -292,7 +337,14 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // within a|b), and individually only when some lane passes the pair test --
 // about 1 pair in 9 on the Twitter-like workload, so the check loop issues
 // ~40% fewer LOP3.
-template <int U, bool FULL3, bool UNION2 = false>
+// WORD1: per-lane word pre-check.  Every row carries a build-time choice of two of its six
+// 32-bit words (those with the most one-bits outside its tile's AND mask, k_word_select);
+// each lane tests its set's two words against those words of 4 survivors per LDS.128 pair
+// (s_w & ~q_w == 0 is necessary for s within q), collecting a 32-survivor pass mask in a
+// register with no votes; only the (lane, survivor) pairs that pass (about 0.1% on the
+// Twitter-like workload) get the full six-word check, in a divergent loop whose trip count
+// is the largest per-lane pass count.
+template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false>
 __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     ScanSmem &sm = *reinterpret_cast<ScanSmem *>(smem_raw);
@@ -417,9 +469,16 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
             } else if (p.filter == 1) {
                 const uint32_t t = brow0 / kTile + lane;
                 const bool in = (uint32_t)lane < t_end - t_first;
-                f0 = warp_and(in ? __ldg(p.t0 + t) : ~0ULL);
-                f1 = warp_and(in ? __ldg(p.t1 + t) : ~0ULL);
-                f2 = warp_and(in ? __ldg(p.t2 + t) : ~0ULL);
+                const uint64_t m0 = in ? __ldg(p.t0 + t) : ~0ULL, m1 = in ? __ldg(p.t1 + t) : ~0ULL,
+                               m2 = in ? __ldg(p.t2 + t) : ~0ULL;
+                if ((uint32_t)lane < (uint32_t)kBlockTiles) {  // the block's tile masks, for level B
+                    sm.tmask[warp][0][lane] = m0;
+                    sm.tmask[warp][1][lane] = m1;
+                    sm.tmask[warp][2][lane] = m2;
+                }
+                f0 = warp_and(m0);
+                f1 = warp_and(m1);
+                f2 = warp_and(m2);
             }
             uint32_t na = 0;
             if ((f1 | f2) == 0) {
@@ -454,15 +513,109 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                 if (p.filter == 0) {
                     tile_prefix(shfl64(s0, 0), shfl64(s1, 0), shfl64(s2, 0), shfl64(s0, nvalid - 1),
                                 shfl64(s1, nvalid - 1), shfl64(s2, nvalid - 1), g0, g1, g2);
-                } else if (p.filter == 1) {
-                    g0 = __ldg(p.t0 + row0 / kTile);
-                    g1 = __ldg(p.t1 + row0 / kTile);
-                    g2 = __ldg(p.t2 + row0 / kTile);
+                } else if (p.filter == 1) {  // staged at level A (written before the __syncwarp there)
+                    g0 = sm.tmask[warp][0][t - t_first];
+                    g1 = sm.tmask[warp][1][t - t_first];
+                    g2 = sm.tmask[warp][2][t - t_first];
                 }
                 // 32-bit halves of the lane's set (invalid lanes: all ones, never pass)
                 const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
                 const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
                 const uint32_t a2l = valid ? (uint32_t)s2 : ~0u, a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
+                if constexpr (WORD1) {
+                    const uint32_t wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
+                    const uint32_t wl = wsel & 15u, wl2 = wsel >> 4;
+                    const uint32_t aw = wl == 0 ? a0l : wl == 1 ? a0h : wl == 2 ? a1l : wl == 3 ? a1h
+                                                                     : wl == 4 ? a2l : a2h;
+                    const uint32_t aw2 = wl2 == 0 ? a0l : wl2 == 1 ? a0h : wl2 == 2 ? a1l : wl2 == 3 ? a1h
+                                                                        : wl2 == 4 ? a2l : a2h;
+                    st_tests += na;
+                    const uint32_t *swp = sm.sw[warp][0];
+                    const uint32_t sw_base = (uint32_t)__cvta_generic_to_shared(swp);
+                    const uint32_t my_plane = sw_base + wl * (uint32_t)(kSubWStride * 4);
+                    const uint32_t my_plane2 = sw_base + wl2 * (uint32_t)(kSubWStride * 4);
+                    for (uint32_t j = 0; j < na;) {
+                        // ---- level B: level-A survivors that contain the tile's mask -> word planes,
+                        // 32 at a time until the buffer cannot take another 32 (full pre-check groups)
+                        uint32_t nb = 0;
+                        const uint32_t pe = na;
+                        // two independent 32-survivor halves per step (ILP), then one more half
+                        // when it still fits
+                        uint32_t *swk = sm.sw[warp][0];
+                        for (; j < na && nb <= (uint32_t)kSubW - 64; j += 64) {
+                            const uint32_t ja = j + lane, jb = ja + 32;
+                            const uint32_t ia = min((uint32_t)sa[min(ja, (uint32_t)kChunk - 1)], (uint32_t)kChunk - 1);
+                            const uint32_t ib = min((uint32_t)sa[min(jb, (uint32_t)kChunk - 1)], (uint32_t)kChunk - 1);
+                            const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
+                            const uint64_t b0 = sm.q0[ib], b1 = sm.q1[ib], b2 = sm.q2[ib];
+                            const bool oka = ja < pe && ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
+                            const bool okb = jb < pe && ((g0 & ~b0) | (g1 & ~b1) | (g2 & ~b2)) == 0;
+                            const uint32_t ba = __ballot_sync(0xffffffffu, oka);
+                            const uint32_t bb = __ballot_sync(0xffffffffu, okb);
+                            if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
+                            const uint32_t nba = nb + __popc(ba);
+                            if (okb) store_survivor(swk, sbi, nba + __popc(bb & lt_mask), b0, b1, b2, ib);
+                            nb = nba + __popc(bb);
+                        }
+                        if (j < na && nb <= (uint32_t)kSubW - 32) {
+                            const uint32_t ja = j + lane;
+                            const uint32_t ia = min((uint32_t)sa[min(ja, (uint32_t)kChunk - 1)], (uint32_t)kChunk - 1);
+                            const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
+                            const bool oka = ja < pe && ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
+                            const uint32_t ba = __ballot_sync(0xffffffffu, oka);
+                            if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
+                            nb += __popc(ba);
+                            j += 32;
+                        }
+                        st_checks += (unsigned long long)nb * nvalid;
+                        __syncwarp();
+                        for (uint32_t k0 = 0; k0 < nb; k0 += 32) {
+                            const uint32_t cnt = min(32u, nb - k0);
+                            // ---- pre-check: the lane's word against 32 survivors, pass bits in acc
+                            uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0;
+                            const uint32_t pa = my_plane + k0 * 4, pa2 = my_plane2 + k0 * 4;
+#define TM_PRE(B, o) precheck4x2<B>(c0, c1, c2, c3, aw, lds128(pa + (o)), aw2, lds128(pa2 + (o)))
+                            TM_PRE(1u << 0, 0);
+                            TM_PRE(1u << 4, 16);
+                            if (cnt > 8) {
+                                TM_PRE(1u << 8, 32);
+                                TM_PRE(1u << 12, 48);
+                            }
+                            if (cnt > 16) {
+                                TM_PRE(1u << 16, 64);
+                                TM_PRE(1u << 20, 80);
+                            }
+                            if (cnt > 24) {
+                                TM_PRE(1u << 24, 96);
+                                TM_PRE(1u << 28, 112);
+                            }
+#undef TM_PRE
+                            uint32_t acc = (c0 | c1) | (c2 | c3);
+                            if (cnt < 32) acc &= (1u << cnt) - 1u;
+                            if (!valid) acc = 0;
+                            // ---- Alg. 3 on the pairs that passed: all six words, then emit
+                            while (__any_sync(0xffffffffu, acc != 0)) {
+                                bool m = false;
+                                uint32_t e = 0;
+                                if (acc) {
+                                    e = k0 + (uint32_t)(__ffs(acc) - 1);
+                                    acc &= acc - 1;
+                                    const uint32_t *c = swp + e;
+                                    m = ((a0l & ~c[0]) | (a0h & ~c[kSubWStride]) | (a1l & ~c[2 * kSubWStride]) |
+                                         (a1h & ~c[3 * kSubWStride]) | (a2l & ~c[4 * kSubWStride]) |
+                                         (a2h & ~c[5 * kSubWStride])) == 0;
+                                }
+                                const uint32_t bm = __ballot_sync(0xffffffffu, m);
+                                if (bm) {
+                                    st_matched += __popc(bm);
+                                    emit_keys(m, row, m ? __ldg(sm.qid + sbi[e]) : 0u, p, lane);
+                                }
+                            }
+                        }
+                        __syncwarp();
+                    }
+                    continue;
+                }
                 for (uint32_t pb = 0; pb < na; pb += kPiece) {
                     const uint32_t pe = min(na, pb + kPiece);
                     // ---- level B: level-A survivors that contain the tile's mask
@@ -629,6 +782,35 @@ __global__ void k_iota(uint32_t *v, uint64_t n) {
     if (i < n) v[i] = (uint32_t)i;
 }
 
+// Per row: which two of its six 32-bit words (w = 2 * block + half, half 1 = the high 32
+// bits) have the most one-bits outside its tile's AND mask -- the words the WORD1 pre-check
+// tests (low nibble: the best, high nibble: the second; ties: lowest w).  Any choice is
+// lossless; this one makes the pre-check most selective.
+__global__ void k_word_select(const uint64_t *__restrict__ w0, const uint64_t *__restrict__ w1,
+                              const uint64_t *__restrict__ w2, const uint64_t *__restrict__ t0,
+                              const uint64_t *__restrict__ t1, const uint64_t *__restrict__ t2, uint64_t rows,
+                              uint8_t *__restrict__ wsel) {
+    uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (r >= rows) return;
+    const uint64_t t = r / kTile;
+    const uint64_t x[3] = {w0[r] & ~t0[t], w1[r] & ~t1[t], w2[r] & ~t2[t]};
+    int best = 0, bc = -1, second = 1, sc = -1;
+#pragma unroll
+    for (int w = 0; w < 6; ++w) {
+        const int c = __popc((uint32_t)(x[w >> 1] >> (32 * (w & 1))));
+        if (c > bc) {
+            second = best;
+            sc = bc;
+            bc = c;
+            best = w;
+        } else if (c > sc) {
+            sc = c;
+            second = w;
+        }
+    }
+    wsel[r] = (uint8_t)(best | (second << 4));
+}
+
 struct PopcAt {
     const uint32_t *bm;
     uint64_t n;
@@ -685,6 +867,7 @@ ScanFn scan_fn(int variant) {
         case 2: return k_scan<4, true>;
         case 3: return k_scan<8, true>;
         case 4: return k_scan<4, false, true>;
+        case 5: return k_scan<4, false, false, true>;
         default: return k_scan<4, false>;
     }
 }
@@ -693,11 +876,12 @@ ScanFn scan_fn(int variant) {
 int scan_variant_env() {
     // TM_SCAN_VARIANT forces a scan-kernel variant: 0 = 4 survivors per
     // iteration, blocks 0-1 first; 1 = 8, blocks 0-1; 2 = 4, all three blocks; 3 = 8, all three;
-    // 4 = pair unions first.  Unset (-1): the handle tunes between 0 and 2 on its first calls.
+    // 4 = pair unions first; 5 = per-lane word pre-check (WORD1).  Unset (-1): the handle tunes
+    // on its first calls.
     const char *e = getenv("TM_SCAN_VARIANT");
     if (!e) return -1;
     const int v = atoi(e);
-    return (v >= 0 && v <= 4) ? v : -1;
+    return (v >= 0 && v < kScanVariants) ? v : -1;
 }
 
 int scan_grid(int device, int variant) {
@@ -713,6 +897,15 @@ int scan_grid(int device, int variant) {
 
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant) {
     scan_fn(variant)<<<grid, kScanWarps * 32, sizeof(ScanSmem), s>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_word_select(const uint64_t *planes, const uint64_t *tand, uint64_t rows, uint8_t *wsel,
+                               cudaStream_t s) {
+    if (!rows) return cudaSuccess;
+    const uint64_t nt = rows / kTile;
+    k_word_select<<<grid_for(rows, 256), 256, 0, s>>>(planes, planes + rows, planes + 2 * rows, tand, tand + nt,
+                                                      tand + 2 * nt, rows, wsel);
     return cudaGetLastError();
 }
 

@@ -17,4 +17,6 @@ for v in "${VARS[@]}"; do
   timeout 600 python bench.py --steps 10 --warmup 3 --no-cpu-baseline $v > gpurun_out/${TAG}_var$i.json 2>&1
   echo "variant $v:"; python -c "import json,sys; d=json.loads(open('gpurun_out/${TAG}_var$i.json').read().strip().splitlines()[-1]); print(d['value'], d['stages_ms'], d['path_stats'])"
 done
-bash scripts/gpu_profile.sh ${TAG} > gpurun_out/${TAG}_profile.log 2>&1
+# profile the variant the bench's handle tuned to (under ncu the tuner's timings are not meaningful)
+VAR=$(python -c "import json,re; d=json.loads(open('gpurun_out/${TAG}_bench.json').read().strip().splitlines()[-1]); print(re.findall(r'variant (\d+)', d['roofline']['kernel'])[0])" 2>/dev/null)
+TM_SCAN_VARIANT=${VAR:-5} bash scripts/gpu_profile.sh ${TAG} > gpurun_out/${TAG}_profile.log 2>&1

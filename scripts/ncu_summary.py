@@ -58,10 +58,12 @@ def main():
                 lines.append(f"  {k:66s} {m[k]:>18s} {units.get(k, '')}")
         st = []
         for k, v in m.items():
-            if k.startswith("smsp__average_warp_latency_issue_stalled_") and k.endswith(".ratio"):
-                x = num(v)
-                if x:
-                    st.append((x, k.replace("smsp__average_warp_latency_issue_stalled_", "").replace(".ratio", "")))
+            for pre, suf in (("smsp__average_warp_latency_issue_stalled_", ".ratio"),
+                             ("smsp__average_warps_issue_stalled_", "_per_issue_active.ratio")):
+                if k.startswith(pre) and k.endswith(suf):
+                    x = num(v)
+                    if x:
+                        st.append((x, k[len(pre):-len(suf)]))
         lines.append("  top stall reasons (avg cycles per issued instruction):")
         for x, k in sorted(st, reverse=True)[:10]:
             lines.append(f"    {k:40s} {x:8.2f}")

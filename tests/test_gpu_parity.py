@@ -204,6 +204,20 @@ def test_c2_full_parity(c2, c2_oracle, layout):
     assert np.unique(got[0]).size == wl.queries.n_sets
 
 
+@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5"])
+def test_c2_every_scan_variant(c2, c2_oracle, variant, monkeypatch):
+    """Every scan-kernel variant (TM_SCAN_VARIANT) gives the oracle's
+    pairs at C2, in the layout bench.py times (balanced splits + AND masks)."""
+    monkeypatch.setenv("TM_SCAN_VARIANT", variant)
+    wl = c2
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=1,
+                      row_order=1) as db:
+        for unique in (False, True):
+            got = db.match_batch(wl.queries, unique)
+            assert_pairs_equal(got, c2_oracle[unique], f"C2 variant={variant} unique={unique}")
+            assert db.stats()["scan_variant"] == int(variant)
+
+
 def test_c2_sampled_against_brute_force(c2):
     """The partitioned oracle is itself pinned to brute force on a query sample."""
     wl = c2
