@@ -210,6 +210,13 @@ __device__ __forceinline__ uint4 lds128(uint32_t addr) {
 // acc |= B << j for each j in 0..3 with (a & ~v_j) == 0: one LOP3 with a predicate result and
 // one predicated OR per survivor (no SEL / add chain)
 // Two-word form: survivor j passes when (a & ~v_j) | (b & ~u_j) == 0.
+__device__ __forceinline__ uint32_t pick_word(uint64_t s0, uint64_t s1, uint64_t s2, uint32_t w, bool valid) {
+    const uint64_t lo = (w & 2u) ? s1 : s0;
+    const uint64_t b = (w & 4u) ? s2 : lo;
+    const uint32_t x = (w & 1u) ? (uint32_t)(b >> 32) : (uint32_t)b;
+    return valid ? x : ~0u;
+}
+
 // WORD1: survivor k's six words into the per-warp word planes (stride kSubWStride), slot i
 __device__ __forceinline__ void store_survivor(uint32_t *sw, uint16_t *sbi, uint32_t k, uint64_t a0, uint64_t a1,
                                                uint64_t a2, uint32_t i) {
@@ -525,10 +532,9 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                 if constexpr (WORD1) {
                     const uint32_t wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
                     const uint32_t wl = wsel & 15u, wl2 = wsel >> 4;
-                    const uint32_t aw = wl == 0 ? a0l : wl == 1 ? a0h : wl == 2 ? a1l : wl == 3 ? a1h
-                                                                     : wl == 4 ? a2l : a2h;
-                    const uint32_t aw2 = wl2 == 0 ? a0l : wl2 == 1 ? a0h : wl2 == 2 ? a1l : wl2 == 3 ? a1h
-                                                                        : wl2 == 4 ? a2l : a2h;
+                    // branch-free word select: block wl >> 1, half wl & 1 (invalid lanes: all ones)
+                    const uint32_t aw = pick_word(s0, s1, s2, wl, valid);
+                    const uint32_t aw2 = pick_word(s0, s1, s2, wl2, valid);
                     st_tests += na;
                     const uint32_t *swp = sm.sw[warp][0];
                     const uint32_t sw_base = (uint32_t)__cvta_generic_to_shared(swp);
