@@ -86,6 +86,8 @@ struct tm_db {
     // scan-kernel variant: forced by TM_SCAN_VARIANT, else tuned on the first calls by
     // kernel ns per decision (filter tests + pair checks) among kTune
     int variant = kTune[0], tune_calls = 0;
+    int call_variant = kTune[0];  // the variant the last call launched
+    bool call_tunes = false;      // the last call is a tuning sample
     double tune_cost[kScanVariants] = {};
     int grid_of[kScanVariants] = {};
     // database (device)

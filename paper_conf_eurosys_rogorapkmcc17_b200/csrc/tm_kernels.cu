@@ -412,12 +412,75 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
             // three blocks -- the HBM-bound regime of the scan.
             const uint32_t vend = min(real_end, rhi);
             const uint32_t nunit = (rhi - rlo + 63) / 64;
+            // WORD1 with 3..8 queries: pre-check; one or two queries: the direct check below is cheaper
+            const bool pre = WORD1 && nq > 2;
+            if (pre) {
+                // the batch as six 32-bit word planes (warp 0's survivor planes; read-only here)
+                if (threadIdx.x < 6 * kSmallBatch) {
+                    const uint32_t w = threadIdx.x / kSmallBatch, j = threadIdx.x % kSmallBatch;
+                    const uint64_t b = j < nq ? (w < 2 ? sm.q0[j] : w < 4 ? sm.q1[j] : sm.q2[j]) : 0ULL;
+                    sm.sw[0][w][j] = (w & 1) ? (uint32_t)(b >> 32) : (uint32_t)b;
+                }
+                __syncthreads();
+            }
             for (;;) {
                 uint32_t u = 0;
                 if (lane == 0) u = atomicAdd(&sm.unit_ctr, 1u);
                 u = __shfl_sync(0xffffffffu, u, 0);
                 if (u >= nunit) break;
                 const uint32_t ra = rlo + u * 64 + lane, rb = ra + 32;
+                if (pre) {
+                    // two-word pre-check of both rows against the batch (4 queries per LDS.128 pair),
+                    // full check only on the (row, query) pairs that pass
+                    const uint64_t a0 = __ldg(p.w0 + ra), a1 = __ldg(p.w1 + ra), a2 = __ldg(p.w2 + ra);
+                    const bool va = ra < vend, vb = rb < vend;
+                    uint64_t b0 = ~0ULL, b1 = ~0ULL, b2 = ~0ULL;
+                    uint32_t wb = 0x10u;
+                    if (rb < rhi) {
+                        b0 = __ldg(p.w0 + rb);
+                        b1 = __ldg(p.w1 + rb);
+                        b2 = __ldg(p.w2 + rb);
+                        wb = __ldg(p.wsel + rb);
+                    }
+                    const uint32_t wa = __ldg(p.wsel + ra);
+                    const uint32_t base = (uint32_t)__cvta_generic_to_shared(sm.sw[0][0]);
+                    constexpr uint32_t kPl = kSubWStride * 4;
+                    const uint32_t xa = pick_word(a0, a1, a2, wa & 15u, va), ya = pick_word(a0, a1, a2, wa >> 4, va);
+                    const uint32_t xb = pick_word(b0, b1, b2, wb & 15u, vb), yb = pick_word(b0, b1, b2, wb >> 4, vb);
+                    const uint32_t pxa = base + (wa & 15u) * kPl, pya = base + (wa >> 4) * kPl;
+                    const uint32_t pxb = base + (wb & 15u) * kPl, pyb = base + (wb >> 4) * kPl;
+                    uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0, d0 = 0, d1 = 0, d2 = 0, d3 = 0;
+                    precheck4x2<1u>(c0, c1, c2, c3, xa, lds128(pxa), ya, lds128(pya));
+                    precheck4x2<1u>(d0, d1, d2, d3, xb, lds128(pxb), yb, lds128(pyb));
+                    if (nq > 4) {
+                        precheck4x2<16u>(c0, c1, c2, c3, xa, lds128(pxa + 16), ya, lds128(pya + 16));
+                        precheck4x2<16u>(d0, d1, d2, d3, xb, lds128(pxb + 16), yb, lds128(pyb + 16));
+                    }
+                    const uint32_t qmask = (1u << nq) - 1u;
+                    uint32_t acc = va ? ((c0 | c1) | (c2 | c3)) & qmask : 0u;
+                    acc |= vb ? (((d0 | d1) | (d2 | d3)) & qmask) << 16 : 0u;  // row b: bits 16..
+                    while (__any_sync(0xffffffffu, acc != 0)) {
+                        bool m = false;
+                        uint32_t j = 0, row = ra;
+                        if (acc) {
+                            const uint32_t bit = (uint32_t)(__ffs(acc) - 1);
+                            acc &= acc - 1;
+                            const bool isb = bit >= 16;
+                            j = bit & 15u;
+                            row = isb ? rb : ra;
+                            const uint64_t s0 = isb ? b0 : a0, s1 = isb ? b1 : a1, s2 = isb ? b2 : a2;
+                            m = ((s0 & ~sm.q0[j]) | (s1 & ~sm.q1[j]) | (s2 & ~sm.q2[j])) == 0;
+                        }
+                        const uint32_t bm = __ballot_sync(0xffffffffu, m);
+                        if (bm) {
+                            st_matched += __popc(bm);
+                            emit_keys(m, row, m ? __ldg(sm.qid + j) : 0u, p, lane);
+                        }
+                    }
+                    const uint32_t u0 = rlo + u * 64;
+                    st_checks += (unsigned long long)nq * (vend > u0 ? min(64u, vend - u0) : 0u);
+                    continue;
+                }
                 uint64_t a0 = __ldg(p.w0 + ra), a1 = __ldg(p.w1 + ra), a2 = __ldg(p.w2 + ra);
                 uint64_t b0 = ~0ULL, b1 = ~0ULL, b2 = ~0ULL;
                 if (rb < rhi) {
