@@ -186,9 +186,10 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         TMCK(launch_route_scatter(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words,
                                   (uint32_t)QW, db->qidx.as<uint32_t>(), db->cap_qidx, s));
         // S3: per-partition batches -> work items
+        const uint32_t range_rows = range_rows_env(db->n_rows);
         TMCK(launch_items(db->word_off.as<unsigned long long>(), (uint32_t)QW, db->part_row.as<uint32_t>(),
                           db->part_n.as<uint32_t>(), P, db->qoff.as<unsigned long long>(),
-                          db->item_cnt.as<unsigned long long>(), ctr, s));
+                          db->item_cnt.as<unsigned long long>(), ctr, range_rows, s));
         launches += 2;
         tb = 0;
         TMCK(cub_exclusive_scan_u64(db->item_cnt.as<unsigned long long>(), db->item_off.as<unsigned long long>(),
@@ -222,6 +223,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         sp.ctr = ctr;
         sp.filter = db->cfg.tile_filter;
         sp.wsel = db->wsel.as<uint8_t>();
+        sp.range_rows = range_rows;
         int var = scan_variant_env();
         if (var < 0) var = db->tune_calls < 2 * kTuneN ? kTune[db->tune_calls % kTuneN] : db->variant;
         // a call of one or two queries only takes the direct streaming path, which runs faster in

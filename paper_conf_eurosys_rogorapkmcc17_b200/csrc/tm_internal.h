@@ -23,7 +23,7 @@ constexpr int kTile = 32;  // rows per warp tile (= one warp, Alg. 4 "thread blo
 // Scan-kernel geometry.
 constexpr int kScanWarps = 4;      // warps per CTA
 constexpr int kChunk = 512;        // queries per work item (per-partition batch)
-constexpr int kRangeRows = 8192;    // rows per work item (multiple of 256)
+constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
 constexpr int kScanVariants = 6;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {5, 2, 0};  // variants the handle times on its first calls (first = default)
 constexpr int kTuneN = 3;
@@ -57,6 +57,7 @@ struct ScanParams {
     DevCounters *ctr;
     uint32_t filter;                  // 0 prefix, 1 AND, 2 none
     const uint8_t *wsel;              // [rows] pre-check word per row (variant 5)
+    uint32_t range_rows;              // rows per work item (multiple of 256)
 };
 
 // ------------------------------------------------------------ launchers --
@@ -71,7 +72,8 @@ cudaError_t launch_route_scatter(const uint32_t *bm, const unsigned long long *w
                                  uint32_t qw, uint32_t *qidx, unsigned long long cap, cudaStream_t s);
 cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const uint32_t *part_row,
                          const uint32_t *part_n, uint32_t n_parts, unsigned long long *qoff,
-                         unsigned long long *item_cnt, DevCounters *ctr, cudaStream_t s);
+                         unsigned long long *item_cnt, DevCounters *ctr, uint32_t range_rows, cudaStream_t s);
+uint32_t range_rows_env(uint64_t n_rows);  // TM_RANGE_ROWS (multiple of 256), else by table size
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant);
 int scan_grid(int device, int variant);
 int scan_variant_env();  // -1 = auto-tune
