@@ -224,14 +224,24 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         sp.filter = db->cfg.tile_filter;
         sp.wsel = db->wsel.as<uint8_t>();
         sp.range_rows = range_rows;
-        int var = scan_variant_env();
-        if (var < 0) var = db->tune_calls < 2 * kTuneN ? kTune[db->tune_calls % kTuneN] : db->variant;
-        // a call of one or two queries only takes the direct streaming path, which runs faster in
-        // the leaner variant-0 kernel (fewer registers live: 0.49 vs 0.60 ms per 2.4 GB at B = 1)
-        db->call_tunes = scan_variant_env() < 0 && db->tune_calls < 2 * kTuneN;
-        if (var == 5 && Q <= 2 && scan_variant_env() < 0) {
-            var = 0;
-            db->call_tunes = false;  // not a tuning sample
+        // variant: TM_SCAN_VARIANT if set; else a call whose partition batches are all small
+        // (Q <= kSmallBatch) takes the streaming path only -- up to four queries checked directly
+        // in the leaner variant-0 kernel (fewer live registers), 5-8 through variant 5's two-word
+        // pre-check (scripts/hbm_sweep.py) -- and is not a
+        // tuning sample (the candidates differ only in the filtered path); other calls cycle
+        // through the candidates on the handle's first qualifying calls, then keep the cheapest
+        const int forced = scan_variant_env();
+        int var = forced;
+        db->call_tunes = false;
+        if (var < 0) {
+            if (Q <= (uint64_t)kSmallBatch) {
+                var = Q <= 4 ? 0 : 5;
+            } else if (db->tune_calls < 2 * kTuneN) {
+                var = kTune[db->tune_calls % kTuneN];
+                db->call_tunes = true;
+            } else {
+                var = db->variant;
+            }
         }
         if (!db->grid_of[var]) db->grid_of[var] = scan_grid(db->device, var);
         db->call_variant = var;

@@ -147,6 +147,14 @@ __global__ void k_route_scatter(const uint32_t *__restrict__ bm, const unsigned 
 }
 
 // ------------------------------------------------------------------ S3 ---
+constexpr uint32_t kSmallRange = 4096;  // rows per work item of a partition routed to <= kSmallBatch queries
+
+// Rows per work item of a partition with nq routed queries: a streaming (HBM-bound) partition is
+// cut into short ranges so that the persistent grid's last wave is a small fraction of the scan.
+__device__ __forceinline__ uint32_t part_range_rows(unsigned long long nq, uint32_t range_rows) {
+    return nq <= (unsigned long long)kSmallBatch ? min(range_rows, kSmallRange) : range_rows;
+}
+
 // Per partition: routed query count -> (chunks of kChunk queries) x (ranges of
 // range_rows rows) work items.
 __global__ void k_items(const unsigned long long *__restrict__ word_off, uint32_t qw_total,
@@ -165,7 +173,8 @@ __global__ void k_items(const unsigned long long *__restrict__ word_off, uint32_
     const unsigned long long nq = word_off[(uint64_t)(p + 1) * qw_total] - o;
     const uint32_t rows = part_row[p + 1] - part_row[p];
     const unsigned long long nchunk = (nq + kChunk - 1) / kChunk;
-    const unsigned long long nrange = (rows + range_rows - 1) / range_rows;
+    const uint32_t rr = part_range_rows(nq, range_rows);
+    const unsigned long long nrange = (rows + rr - 1) / rr;
     item_cnt[p] = nchunk * nrange;
     if (nq) atomicAdd(&ctr->candidates, nq * (unsigned long long)part_n[p]);
 }
@@ -178,7 +187,6 @@ __global__ void k_items(const unsigned long long *__restrict__ word_off, uint32_
 constexpr int kBlockTiles = 8;   // tiles per level-A block (256 rows)
 constexpr int kSubB = 128;       // level-B survivors buffered per pass
 constexpr int kQSub = 128;       // queries per unit
-constexpr int kSmallBatch = 8;   // batches up to this size take the unfiltered streaming path
 
 // WORD1 survivor planes: word w (= 32-bit half w & 1 of block w >> 1) of level-B
 // survivor k at sw[warp][w][k]; the plane stride (kSubW + 4 words = 400 B, 16 B mod 128)
@@ -246,6 +254,13 @@ __device__ __forceinline__ void precheck4x2(uint32_t &c0, uint32_t &c1, uint32_t
         : "+r"(c0), "+r"(c1), "+r"(c2), "+r"(c3)
         : "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"(b), "r"(u.x), "r"(u.y), "r"(u.z), "r"(u.w), "n"(B),
           "n"(B << 1), "n"(B << 2), "n"(B << 3));
+}
+
+// 16-B streaming load of two consecutive rows of a plane (read-only path, no L1 allocation)
+__device__ __forceinline__ ulonglong2 ldg_stream2(const uint64_t *ptr) {
+    ulonglong2 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v2.u64 {%0, %1}, [%2];" : "=l"(v.x), "=l"(v.y) : "l"(ptr));
+    return v;
 }
 
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
@@ -387,13 +402,15 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
         const uint32_t prow = __ldg(p.part_row + part);
         const uint32_t rows = __ldg(p.part_row + part + 1) - prow;
         const uint32_t real_end = prow + __ldg(p.part_n + part);
-        const uint32_t nrange = (rows + p.range_rows - 1) / p.range_rows;
+        const unsigned long long pq0 = __ldg(p.qoff + part), pq1 = __ldg(p.qoff + part + 1);
+        const uint32_t rr = part_range_rows(pq1 - pq0, p.range_rows);
+        const uint32_t nrange = (rows + rr - 1) / rr;
         const unsigned long long local = item - __ldg(p.item_off + part);
         const uint32_t chunk = (uint32_t)(local / nrange), range = (uint32_t)(local % nrange);
-        const unsigned long long qbeg = __ldg(p.qoff + part) + (unsigned long long)chunk * kChunk;
-        const uint32_t nq = (uint32_t)min((unsigned long long)kChunk, __ldg(p.qoff + part + 1) - qbeg);
-        const uint32_t rlo = prow + range * p.range_rows;
-        const uint32_t rhi = min(rlo + p.range_rows, prow + rows);
+        const unsigned long long qbeg = pq0 + (unsigned long long)chunk * kChunk;
+        const uint32_t nq = (uint32_t)min((unsigned long long)kChunk, pq1 - qbeg);
+        const uint32_t rlo = prow + range * rr;
+        const uint32_t rhi = min(rlo + rr, prow + rows);
 
         if (threadIdx.x == 0) sm.qid = p.qidx + qbeg;
         // stage the query batch (the batch of queries of partition p)
@@ -411,9 +428,12 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
             // lane, all loads issued up front) and checks every row against every query on all
             // three blocks -- the HBM-bound regime of the scan.
             const uint32_t vend = min(real_end, rhi);
-            const uint32_t nunit = (rhi - rlo + 63) / 64;
             // WORD1 with 3..8 queries: pre-check; one or two queries: the direct check below is cheaper
-            const bool pre = WORD1 && nq > 2;
+            const bool pre = WORD1 && nq > 4;
+            // units: 64 rows (pre-check: two rows per lane) or 128 rows (direct: four rows per lane as
+            // two 16-B loads per plane, 96 B in flight per lane)
+            const uint32_t ush = pre ? 6u : 7u;
+            const uint32_t nunit = (rhi - rlo + (1u << ush) - 1) >> ush;
             if (pre) {
                 // the batch as six 32-bit word planes (warp 0's survivor planes; read-only here)
                 if (threadIdx.x < 6 * kSmallBatch) {
@@ -428,21 +448,22 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                 if (lane == 0) u = atomicAdd(&sm.unit_ctr, 1u);
                 u = __shfl_sync(0xffffffffu, u, 0);
                 if (u >= nunit) break;
-                const uint32_t ra = rlo + u * 64 + lane, rb = ra + 32;
                 if (pre) {
                     // two-word pre-check of both rows against the batch (4 queries per LDS.128 pair),
-                    // full check only on the (row, query) pairs that pass
-                    const uint64_t a0 = __ldg(p.w0 + ra), a1 = __ldg(p.w1 + ra), a2 = __ldg(p.w2 + ra);
-                    const bool va = ra < vend, vb = rb < vend;
-                    uint64_t b0 = ~0ULL, b1 = ~0ULL, b2 = ~0ULL;
-                    uint32_t wb = 0x10u;
-                    if (rb < rhi) {
-                        b0 = __ldg(p.w0 + rb);
-                        b1 = __ldg(p.w1 + rb);
-                        b2 = __ldg(p.w2 + rb);
-                        wb = __ldg(p.wsel + rb);
+                    // full check only on the (row, query) pairs that pass; rows (ra, ra + 1) per lane
+                    // as one 16-B load per plane (a tile never straddles rhi)
+                    const uint32_t ra = rlo + u * 64 + 2 * (uint32_t)lane, rb = ra + 1;
+                    ulonglong2 v0 = make_ulonglong2(~0ULL, ~0ULL), v1 = v0, v2 = v0;
+                    uint32_t wab = 0x1010u;
+                    if (ra < rhi) {
+                        v0 = ldg_stream2(p.w0 + ra);
+                        v1 = ldg_stream2(p.w1 + ra);
+                        v2 = ldg_stream2(p.w2 + ra);
+                        wab = __ldg(reinterpret_cast<const unsigned short *>(p.wsel + ra));
                     }
-                    const uint32_t wa = __ldg(p.wsel + ra);
+                    const uint64_t a0 = v0.x, a1 = v1.x, a2 = v2.x, b0 = v0.y, b1 = v1.y, b2 = v2.y;
+                    const bool va = ra < vend, vb = rb < vend;
+                    const uint32_t wa = wab & 0xffu, wb = wab >> 8;
                     const uint32_t base = (uint32_t)__cvta_generic_to_shared(sm.sw[0][0]);
                     constexpr uint32_t kPl = kSubWStride * 4;
                     const uint32_t xa = pick_word(a0, a1, a2, wa & 15u, va), ya = pick_word(a0, a1, a2, wa >> 4, va);
@@ -481,33 +502,43 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                     st_checks += (unsigned long long)nq * (vend > u0 ? min(64u, vend - u0) : 0u);
                     continue;
                 }
-                uint64_t a0 = __ldg(p.w0 + ra), a1 = __ldg(p.w1 + ra), a2 = __ldg(p.w2 + ra);
-                uint64_t b0 = ~0ULL, b1 = ~0ULL, b2 = ~0ULL;
-                if (rb < rhi) {
-                    b0 = __ldg(p.w0 + rb);
-                    b1 = __ldg(p.w1 + rb);
-                    b2 = __ldg(p.w2 + rb);
+                // direct check: rows (r, r+1) and (r+64, r+65) per lane, r = base + 2 lane; a tile
+                // is either wholly inside the range or wholly outside, so a pair never straddles rhi
+                const uint32_t u0 = rlo + (u << 7);
+                const uint32_t r0 = u0 + 2 * (uint32_t)lane, r1 = r0 + 64;
+                ulonglong2 a0 = make_ulonglong2(~0ULL, ~0ULL), a1 = a0, a2 = a0, b0 = a0, b1 = a0, b2 = a0;
+                if (r0 < rhi) {
+                    a0 = ldg_stream2(p.w0 + r0);
+                    a1 = ldg_stream2(p.w1 + r0);
+                    a2 = ldg_stream2(p.w2 + r0);
                 }
-                const bool va = ra < vend, vb = rb < vend;
+                if (r1 < rhi) {
+                    b0 = ldg_stream2(p.w0 + r1);
+                    b1 = ldg_stream2(p.w1 + r1);
+                    b2 = ldg_stream2(p.w2 + r1);
+                }
+                const bool v0 = r0 < vend, v1 = r0 + 1 < vend, v2 = r1 < vend, v3 = r1 + 1 < vend;
                 for (uint32_t j = 0; j < nq; ++j) {
                     const uint64_t q0 = sm.q0[j], q1 = sm.q1[j], q2 = sm.q2[j];
-                    const bool ha = va && ((a0 & ~q0) | (a1 & ~q1) | (a2 & ~q2)) == 0;
-                    const bool hb = vb && ((b0 & ~q0) | (b1 & ~q1) | (b2 & ~q2)) == 0;
-                    if (__any_sync(0xffffffffu, ha || hb)) {
-                        const uint32_t ba = __ballot_sync(0xffffffffu, ha);
-                        if (ba) {
-                            st_matched += __popc(ba);
-                            emit_keys(ha, ra, __ldg(sm.qid + j), p, lane);
-                        }
-                        const uint32_t bb = __ballot_sync(0xffffffffu, hb);
-                        if (bb) {
-                            st_matched += __popc(bb);
-                            emit_keys(hb, rb, __ldg(sm.qid + j), p, lane);
+                    const bool h0 = v0 && ((a0.x & ~q0) | (a1.x & ~q1) | (a2.x & ~q2)) == 0;
+                    const bool h1 = v1 && ((a0.y & ~q0) | (a1.y & ~q1) | (a2.y & ~q2)) == 0;
+                    const bool h2 = v2 && ((b0.x & ~q0) | (b1.x & ~q1) | (b2.x & ~q2)) == 0;
+                    const bool h3 = v3 && ((b0.y & ~q0) | (b1.y & ~q1) | (b2.y & ~q2)) == 0;
+                    if (__any_sync(0xffffffffu, (h0 || h1) || (h2 || h3))) {
+                        const uint32_t qg = __ldg(sm.qid + j);
+                        const bool hh[4] = {h0, h1, h2, h3};
+                        const uint32_t rr4[4] = {r0, r0 + 1, r1, r1 + 1};
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            const uint32_t bq = __ballot_sync(0xffffffffu, hh[e]);
+                            if (bq) {
+                                st_matched += __popc(bq);
+                                emit_keys(hh[e], rr4[e], qg, p, lane);
+                            }
                         }
                     }
                 }
-                const uint32_t u0 = rlo + u * 64;
-                st_checks += (unsigned long long)nq * (vend > u0 ? min(64u, vend - u0) : 0u);
+                st_checks += (unsigned long long)nq * (vend > u0 ? min(128u, vend - u0) : 0u);
             }
             __syncthreads();
             continue;

@@ -68,6 +68,7 @@ def main():
                               "table_gbs": gbs, "frac_of_measured_hbm": gbs / hbm,
                               "pair_checks": st["pair_checks"], "tile_tests": st["tile_tests"],
                               "checks_per_s": st["pair_checks"] / (ms / 1e3), "parity": ok,
+                              "variant": st["scan_variant"], "work_items": st["work_items"],
                               "gen_s": gen_s, "build_s": build_s}), flush=True)
         db.close()
 
