@@ -236,11 +236,15 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         if (var < 0) {
             if (Q <= (uint64_t)kSmallBatch) {
                 var = Q <= 4 ? 0 : 5;
-            } else if (db->tune_calls < 2 * kTuneN) {
-                var = kTune[db->tune_calls % kTuneN];
-                db->call_tunes = true;
             } else {
-                var = db->variant;
+                const int c = 63 - __builtin_clzll(Q);
+                db->call_class = c;
+                if (db->tune_calls[c] < 2 * kTuneN) {
+                    var = kTune[db->tune_calls[c] % kTuneN];
+                    db->call_tunes = true;
+                } else {
+                    var = db->variant[c];
+                }
             }
         }
         if (!db->grid_of[var]) db->grid_of[var] = scan_grid(db->device, var);
@@ -336,12 +340,13 @@ void finish_timing(tm_db *db, cudaStream_t s) {
     // the cheapest is kept
     const double dec = (double)(st.tile_tests + st.pair_checks);
     if (db->call_tunes && dec > 1e6 && st.retries == 0) {
-        if (db->tune_calls >= kTuneN) db->tune_cost[db->call_variant] = ms * 1e6 / dec;
-        if (++db->tune_calls == 2 * kTuneN) {
+        const int c = db->call_class;
+        if (db->tune_calls[c] >= kTuneN) db->tune_cost[c][db->call_variant] = ms * 1e6 / dec;
+        if (++db->tune_calls[c] == 2 * kTuneN) {
             int best = kTune[0];
             for (int i = 1; i < kTuneN; ++i)
-                if (db->tune_cost[kTune[i]] < db->tune_cost[best]) best = kTune[i];
-            db->variant = best;
+                if (db->tune_cost[c][kTune[i]] < db->tune_cost[c][best]) best = kTune[i];
+            db->variant[c] = best;
         }
     }
     TMCK(cudaEventElapsedTime(&ms, db->ev[3], db->ev[4]));

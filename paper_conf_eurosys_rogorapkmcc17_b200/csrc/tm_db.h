@@ -83,12 +83,18 @@ struct tm_db {
     cudaEvent_t ev[6] = {};
     tm_config cfg{};
     int scan_grid = 0;
-    // scan-kernel variant: forced by TM_SCAN_VARIANT, else tuned on the first calls by
-    // kernel ns per decision (filter tests + pair checks) among kTune
-    int variant = kTune[0], tune_calls = 0;
+    // scan-kernel variant: forced by TM_SCAN_VARIANT, else tuned per batch-size class
+    // (floor(log2 Q): the best variant depends on how many queries share a partition) on the
+    // first calls of that class, by kernel ns per decision (filter tests + pair checks) among kTune
+    static constexpr int kClasses = 33;
+    int variant[kClasses], tune_calls[kClasses] = {};
+    double tune_cost[kClasses][kScanVariants] = {};
     int call_variant = kTune[0];  // the variant the last call launched
+    int call_class = 0;           // the batch-size class of the last call
     bool call_tunes = false;      // the last call is a tuning sample
-    double tune_cost[kScanVariants] = {};
+    tm_db() {
+        for (int &v : variant) v = kTune[0];
+    }
     int grid_of[kScanVariants] = {};
     // database (device)
     uint64_t n_sets = 0, n_entries = 0, n_unique = 0, n_rows = 0, n_parts = 0, n_parts_total = 0;

@@ -150,9 +150,13 @@ __global__ void k_route_scatter(const uint32_t *__restrict__ bm, const unsigned 
 constexpr uint32_t kSmallRange = 4096;  // rows per work item of a partition routed to <= kSmallBatch queries
 
 // Rows per work item of a partition with nq routed queries: a streaming (HBM-bound) partition is
-// cut into short ranges so that the persistent grid's last wave is a small fraction of the scan.
+// cut into short ranges, and a partition of at most three query chunks into quarter ranges, so that
+// a large partition that few queries reach still yields many items and the persistent grid's last
+// wave stays a small fraction of the scan (the item's query staging is cheap for few queries).
 __device__ __forceinline__ uint32_t part_range_rows(unsigned long long nq, uint32_t range_rows) {
-    return nq <= (unsigned long long)kSmallBatch ? min(range_rows, kSmallRange) : range_rows;
+    if (nq <= (unsigned long long)kSmallBatch) return min(range_rows, kSmallRange);
+    if (nq <= 3ULL * kChunk) return max((range_rows / 4) & ~255u, 256u);
+    return range_rows;
 }
 
 // Per partition: routed query count -> (chunks of kChunk queries) x (ranges of
