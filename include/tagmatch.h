@@ -82,8 +82,12 @@ typedef enum {
  * signature).  Sizes are given explicitly so the same struct can describe
  * device-resident arrays (tm_match_batch_device):
  *   n_bytes = vocab_off[n_vocab], n_tags = set_off[n_sets], set_off[0] = 0,
- * offsets non-decreasing, tag_idx[t] < n_vocab.  Host calls validate all of
- * this (TM_EINVAL); device calls validate only what is checkable on the host.
+ * offsets non-decreasing, tag_idx[t] < n_vocab.  tm_build and tm_encode
+ * validate all of this on the host (TM_EINVAL).  The match calls check pointers,
+ * sizes and the end points on the host and leave the O(n) checks (monotone
+ * offsets, indices in range) to the query encoder kernels, which never read
+ * out of bounds: a malformed batch fails with TM_EINVAL and no result, on both
+ * tm_match_batch and tm_match_batch_device, and the handle stays usable.
  */
 typedef struct {
     const uint8_t *vocab_bytes; /* n_bytes bytes (may be NULL if n_bytes == 0)  */

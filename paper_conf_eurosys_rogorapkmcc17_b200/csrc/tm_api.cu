@@ -99,6 +99,27 @@ void check_tagsets_host(const tm_tagsets *t, const char *what) {
             if (t->tag_idx[i] >= t->n_vocab) fail(TM_EINVAL, w + ": tag_idx out of range");
 }
 
+// O(1) checks of host query arrays (pointers, sizes, end points); the O(n) monotonicity and range
+// checks run inside the encoder kernels (match_core)
+void check_tagsets_shape(const tm_tagsets *t, const char *what) {
+    const std::string w(what);
+    if (!t) fail(TM_EINVAL, w + ": NULL tagsets");
+    if (t->n_sets > 0xFFFFFFFFull) fail(TM_ERANGE, w + ": more than 2^32-1 sets");
+    if (!t->set_off) fail(TM_EINVAL, w + ": set_off is NULL");
+    if (t->n_vocab > 0 && !t->vocab_off) fail(TM_EINVAL, w + ": vocab_off is NULL");
+    if (t->n_bytes > 0 && !t->vocab_bytes) fail(TM_EINVAL, w + ": vocab_bytes is NULL");
+    if (t->n_tags > 0 && t->tag_idx == nullptr && t->n_tags != t->n_vocab)
+        fail(TM_EINVAL, w + ": tag_idx NULL requires n_tags == n_vocab");
+    if (t->n_vocab > 0xFFFFFFFFull) fail(TM_ERANGE, w + ": more than 2^32-1 vocabulary strings");
+    if (t->set_off[0] != 0 || t->set_off[t->n_sets] != t->n_tags) fail(TM_EINVAL, w + ": set_off[0] != 0 or set_off[n_sets] != n_tags");
+    if (t->n_vocab > 0) {
+        if (t->vocab_off[0] != 0 || t->vocab_off[t->n_vocab] != t->n_bytes)
+            fail(TM_EINVAL, w + ": vocab_off[0] != 0 or vocab_off[n_vocab] != n_bytes");
+    } else if (t->n_tags > 0) {
+        fail(TM_EINVAL, w + ": tags without a vocabulary");
+    }
+}
+
 void check_tagsets_device(const tm_tagsets *t) {
     if (!t) fail(TM_EINVAL, "queries: NULL tagsets");
     if (t->n_sets > 0xFFFFFFFFull) fail(TM_ERANGE, "queries: more than 2^32-1 sets");
@@ -158,8 +179,13 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
     db->vsig.ensure(std::max<uint64_t>(q->n_vocab, 1) * 24);
     db->qplanes.ensure(Q * 24);
     uint64_t *q0 = db->qplanes.as<uint64_t>(), *q1 = q0 + Q, *q2 = q1 + Q;
-    TMCK(launch_hash_vocab(q->vocab_bytes, q->vocab_off, q->n_vocab, db->vsig.as<uint64_t>(), s));
-    TMCK(launch_encode_sets(db->vsig.as<uint64_t>(), q->tag_idx, q->set_off, Q, q0, q1, q2, s));
+    // the query CSR is validated by the encoder kernels themselves (input_err, checked below with
+    // the scan counters): no O(n) host pass over the batch on the call's critical path
+    TMCK(cudaMemsetAsync(&ctr->input_err, 0, sizeof(ctr->input_err), s));
+    TMCK(launch_hash_vocab(q->vocab_bytes, q->vocab_off, q->n_vocab, q->n_bytes, db->vsig.as<uint64_t>(),
+                           &ctr->input_err, s));
+    TMCK(launch_encode_sets(db->vsig.as<uint64_t>(), q->tag_idx, q->set_off, Q, q->n_tags, q->n_vocab, q0, q1, q2,
+                            &ctr->input_err, s));
     launches += 2;
     TMCK(cudaEventRecord(db->ev[1], s));
 
@@ -182,7 +208,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
     for (int attempt = 0;; ++attempt) {
         db->qidx.ensure(db->cap_qidx * 4);
         db->out.ensure(db->cap_out * 8);
-        TMCK(cudaMemsetAsync(ctr, 0, sizeof(DevCounters), s));
+        TMCK(cudaMemsetAsync(ctr, 0, offsetof(DevCounters, input_err), s));
         TMCK(launch_route_scatter(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words,
                                   (uint32_t)QW, db->qidx.as<uint32_t>(), db->cap_qidx, s));
         // S3: per-partition batches -> work items
@@ -257,6 +283,10 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         TMCK(cudaMemcpyAsync(db->h_ctr, ctr, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
         TMCK(cudaStreamSynchronize(s));
         const DevCounters c = *db->h_ctr;
+        if (c.input_err)
+            fail(TM_EINVAL, std::string("queries: malformed CSR found by the encoder (") +
+                                ((c.input_err & 1u) ? "vocab_off " : "") + ((c.input_err & 2u) ? "set_off " : "") +
+                                ((c.input_err & 4u) ? "tag_idx out of range" : "") + ")");
         bool retry = false;
         if (c.routed > db->cap_qidx) {
             db->cap_qidx = c.routed + c.routed / 4;
@@ -443,9 +473,10 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
         d_vsig.ensure(std::max<uint64_t>(sets->n_vocab, 1) * 24);
         d_planes.ensure(N * 24);
         uint64_t *w0 = d_planes.as<uint64_t>(), *w1 = w0 + N, *w2 = w1 + N;
-        TMCK(launch_hash_vocab(d_bytes.as<uint8_t>(), d_voff.as<uint64_t>(), sets->n_vocab, d_vsig.as<uint64_t>(), s));
+        TMCK(launch_hash_vocab(d_bytes.as<uint8_t>(), d_voff.as<uint64_t>(), sets->n_vocab, sets->n_bytes,
+                               d_vsig.as<uint64_t>(), nullptr, s));
         TMCK(launch_encode_sets(d_vsig.as<uint64_t>(), (sets->tag_idx && sets->n_tags) ? d_tidx.as<uint32_t>() : nullptr,
-                                d_soff.as<uint64_t>(), N, w0, w1, w2, s));
+                                d_soff.as<uint64_t>(), N, sets->n_tags, sets->n_vocab, w0, w1, w2, nullptr, s));
         // S0b: lexicographic sort of the signatures (LSD: word 2, then 1, then 0; stable)
         d_idx.ensure(N * 4);
         d_idx2.ensure(N * 4);
@@ -708,7 +739,7 @@ tm_status tm_match_batch(tm_db *db, const tm_tagsets *q, int unique, tm_pairs *o
     TM_API_BEGIN
     if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
     if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
-    check_tagsets_host(q, "queries");
+    check_tagsets_shape(q, "queries");
     DeviceGuard g(db->device);
     cudaStream_t s = db->stream;
     // one H2D copy of the query batch
@@ -824,8 +855,10 @@ tm_status tm_encode(const tm_tagsets *sets, uint64_t *sig_out, int device) {
         dti = ti.as<uint32_t>();
     }
     uint64_t *w0 = pl.as<uint64_t>(), *w1 = w0 + N, *w2 = w1 + N;
-    TMCK(launch_hash_vocab(b.as<uint8_t>(), vo.as<uint64_t>(), sets->n_vocab, vs.as<uint64_t>(), s));
-    TMCK(launch_encode_sets(vs.as<uint64_t>(), dti, so.as<uint64_t>(), N, w0, w1, w2, s));
+    TMCK(launch_hash_vocab(b.as<uint8_t>(), vo.as<uint64_t>(), sets->n_vocab, sets->n_bytes, vs.as<uint64_t>(),
+                           nullptr, s));
+    TMCK(launch_encode_sets(vs.as<uint64_t>(), dti, so.as<uint64_t>(), N, sets->n_tags, sets->n_vocab, w0, w1, w2,
+                            nullptr, s));
     std::vector<uint64_t> h(3 * N);
     TMCK(cudaMemcpyAsync(h.data(), pl.p, N * 24, cudaMemcpyDeviceToHost, s));
     TMCK(cudaStreamSynchronize(s));

@@ -38,6 +38,8 @@ struct DevCounters {            // zeroed at the start of every match call
     unsigned long long matched_sets;
     unsigned long long routed;      // R = routed (q, p) pairs
     unsigned long long candidates;  // sum |P| over routed pairs
+    unsigned int input_err;         // malformed query CSR seen by the encoder (zeroed before it)
+    unsigned int pad_;
 };
 
 struct ScanParams {
@@ -63,10 +65,11 @@ struct ScanParams {
 
 // ------------------------------------------------------------ launchers --
 // All launchers are asynchronous on `s` and return the launch error.
-cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_t n_vocab, uint64_t *vsig,
-                              cudaStream_t s);
+cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_t n_vocab, uint64_t n_bytes,
+                              uint64_t *vsig, unsigned int *err, cudaStream_t s);
 cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, const uint64_t *set_off,
-                               uint64_t n_sets, uint64_t *w0, uint64_t *w1, uint64_t *w2, cudaStream_t s);
+                               uint64_t n_sets, uint64_t n_tags, uint64_t n_vocab, uint64_t *w0, uint64_t *w1,
+                               uint64_t *w2, unsigned int *err, cudaStream_t s);
 cudaError_t launch_route_bitmap(const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
                                 const uint64_t *q2, uint64_t n_q, uint32_t *bm, cudaStream_t s);
 cudaError_t launch_route_scatter(const uint32_t *bm, const unsigned long long *word_off, uint64_t n_words,

@@ -39,11 +39,17 @@ inline unsigned grid_for(uint64_t n, unsigned bs) {
 // ------------------------------------------------------------------ S1 ---
 // One thread per vocabulary string: FNV-1a-64 of the bytes, then positions
 // floor(z*192/2^64) of the first 7 SplitMix64 outputs seeded with it.
+// The CSR is validated on the device (non-decreasing offsets inside [0, n_bytes], end points):
+// a malformed string sets *err and is hashed as empty, so nothing is read out of bounds.
 __global__ void k_hash_vocab(const uint8_t *__restrict__ bytes, const uint64_t *__restrict__ off, uint64_t n,
-                             uint64_t *__restrict__ vsig) {
+                             uint64_t n_bytes, uint64_t *__restrict__ vsig, unsigned int *err) {
     uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (v >= n) return;
     uint64_t b = off[v], e = off[v + 1];
+    if (e < b || e > n_bytes || (v == 0 && b != 0) || (v == n - 1 && e != n_bytes)) {
+        if (err) atomicOr(err, 1u);
+        e = b = 0;
+    }
     uint64_t h = kFnvOffset;
     for (uint64_t i = b; i < e; ++i) {
         h ^= (uint64_t)__ldg(bytes + i);
@@ -67,15 +73,26 @@ __global__ void k_hash_vocab(const uint8_t *__restrict__ bytes, const uint64_t *
 }
 
 // One thread per set; writes the three signature planes.
+// Validated like k_hash_vocab: offsets non-decreasing inside [0, n_tags] with set_off[0] = 0 and
+// set_off[n] = n_tags, tag indices < n_vocab; violations set *err and are skipped.
 __global__ void k_encode_sets(const uint64_t *__restrict__ vsig, const uint32_t *__restrict__ tag_idx,
-                              const uint64_t *__restrict__ set_off, uint64_t n, uint64_t *__restrict__ w0,
-                              uint64_t *__restrict__ w1, uint64_t *__restrict__ w2) {
+                              const uint64_t *__restrict__ set_off, uint64_t n, uint64_t n_tags, uint64_t n_vocab,
+                              uint64_t *__restrict__ w0, uint64_t *__restrict__ w1, uint64_t *__restrict__ w2,
+                              unsigned int *err) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i >= n) return;
     uint64_t b = set_off[i], e = set_off[i + 1];
+    if (e < b || e > n_tags || (i == 0 && b != 0) || (i == n - 1 && e != n_tags)) {
+        if (err) atomicOr(err, 2u);
+        e = b = 0;
+    }
     uint64_t a0 = 0, a1 = 0, a2 = 0;
     for (uint64_t t = b; t < e; ++t) {
         const uint64_t v = tag_idx ? (uint64_t)__ldg(tag_idx + t) : t;
+        if (v >= n_vocab) {
+            if (err) atomicOr(err, 4u);
+            continue;
+        }
         a0 |= __ldg(vsig + 3 * v + 0);
         a1 |= __ldg(vsig + 3 * v + 1);
         a2 |= __ldg(vsig + 3 * v + 2);
@@ -926,17 +943,19 @@ struct PopcAt {
 }  // namespace
 
 // ------------------------------------------------------------ launchers ---
-cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_t n_vocab, uint64_t *vsig,
-                              cudaStream_t s) {
+cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_t n_vocab, uint64_t n_bytes,
+                              uint64_t *vsig, unsigned int *err, cudaStream_t s) {
     if (!n_vocab) return cudaSuccess;
-    k_hash_vocab<<<grid_for(n_vocab, 256), 256, 0, s>>>(bytes, off, n_vocab, vsig);
+    k_hash_vocab<<<grid_for(n_vocab, 256), 256, 0, s>>>(bytes, off, n_vocab, n_bytes, vsig, err);
     return cudaGetLastError();
 }
 
 cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, const uint64_t *set_off,
-                               uint64_t n_sets, uint64_t *w0, uint64_t *w1, uint64_t *w2, cudaStream_t s) {
+                               uint64_t n_sets, uint64_t n_tags, uint64_t n_vocab, uint64_t *w0, uint64_t *w1,
+                               uint64_t *w2, unsigned int *err, cudaStream_t s) {
     if (!n_sets) return cudaSuccess;
-    k_encode_sets<<<grid_for(n_sets, 256), 256, 0, s>>>(vsig, tag_idx, set_off, n_sets, w0, w1, w2);
+    k_encode_sets<<<grid_for(n_sets, 256), 256, 0, s>>>(vsig, tag_idx, set_off, n_sets, n_tags, n_vocab, w0, w1, w2,
+                                                         err);
     return cudaGetLastError();
 }
 

@@ -335,6 +335,43 @@ class _CAI:
         self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3}
 
 
+def _malformed_batches(c1):
+    """(what, TagSets) query batches whose CSR breaks include/tagmatch.h's rules in the middle
+    (the O(1) end-point checks pass; only the encoder kernels' device validation sees it)."""
+    q = c1.queries
+    vo, ti, so = q.vocab_off.copy(), q.tag_idx.copy(), q.set_off.copy()
+    bad_so = so.copy()
+    bad_so[5], bad_so[6] = so[6], so[5]                      # non-decreasing broken
+    bad_ti = ti.copy()
+    bad_ti[17] = q.vocab_off.size + 1000                     # index past the vocabulary
+    bad_vo = vo.copy()
+    bad_vo[3] = vo[-1] + 7                                   # string past n_bytes
+    return [("set_off", tmgen.TagSets(q.vocab_bytes, vo, ti, bad_so)),
+            ("tag_idx", tmgen.TagSets(q.vocab_bytes, vo, bad_ti, so)),
+            ("vocab_off", tmgen.TagSets(q.vocab_bytes, bad_vo, ti, so))]
+
+
+def test_malformed_query_batch_is_rejected(c1):
+    """A malformed query CSR fails with TM_EINVAL on both entry points (validated on the device by
+    the encoder, no out-of-bounds read), and the handle keeps working afterwards."""
+    torch = pytest.importorskip("torch")
+    want = oracle_pairs(c1, False)
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=2000, tile_filter=1, row_order=1) as db:
+        for what, bad in _malformed_batches(c1):
+            with pytest.raises(tmb.TagMatchError) as e:
+                db.match_batch(bad, False)
+            assert e.value.status == -1, what
+            t = [torch.from_numpy(np.ascontiguousarray(a)).cuda() for a in
+                 (bad.vocab_bytes, bad.vocab_off.view(np.int64), bad.tag_idx.view(np.int32),
+                  bad.set_off.view(np.int64))]
+            dq = tmb.device_tagsets(t[0].data_ptr(), t[1].data_ptr(), t[2].data_ptr(), t[3].data_ptr(),
+                                    bad.vocab_bytes.size, bad.vocab_off.size - 1, bad.tag_idx.size, bad.n_sets)
+            with pytest.raises(tmb.TagMatchError) as e:
+                db.match_batch_device(dq, False, torch.cuda.current_stream().cuda_stream)
+            assert e.value.status == -1, what
+            assert_pairs_equal(db.match_batch(c1.queries, False), want, f"after malformed {what}")
+
+
 def test_device_entry_point_matches_host(c1):
     torch = pytest.importorskip("torch")
     with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=200_000) as db:
