@@ -44,6 +44,8 @@ SM_COUNT = 148
 # block test = and-not of both 32-bit halves + zero test = 3 ALU ops.
 OPS_PER_TILE_TEST = 3
 OPS_PER_PAIR_CHECK = 3
+SURVEY_OPS_PER_TILE_TEST = 4    # SURVEY.md 8(d) per-unit figures (plain Alg. 4 / Alg. 3)
+SURVEY_OPS_PER_PAIR_CHECK = 7
 
 
 class _CAI:
@@ -374,6 +376,11 @@ def run_ours(args):
                          "ops_per_launch": ops,
                          "ops_model": "3 ALU ops per decision (pre-filter test or pair check): the minimum "
                                       "one 64-bit block test; DESIGN.md sec. 6",
+                         "frac_survey_model": (SURVEY_OPS_PER_TILE_TEST * last["tile_tests"] +
+                                               SURVEY_OPS_PER_PAIR_CHECK * last["pair_checks"]) / scan_s / 1e12
+                                              / peak_tops,
+                         "survey_model": "SURVEY.md 8(d): 4 ops per tile test + 7 per pair check (the full "
+                                         "three-block check); informational, frac above is the primary",
                          "ncu_same_kernel": ncu,
                          "peak_src": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM_CLK} ALU lanes/clk x "
                                      f"{peaks.get('sm_max_mhz', 1965.0)} MHz ({peak_src} sm_max_mhz)"},

@@ -603,10 +603,13 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                 f2 = warp_and(m2);
             }
             uint32_t na = 0;
-            if ((f1 | f2) == 0) {
+            if ((f0 != 0) + (f1 != 0) + (f2 != 0) <= 1) {
+                // the block mask lives in one word (or none): test that word only (warp-uniform)
+                const uint64_t *qw = f1 ? sm.q1 : (f2 ? sm.q2 : sm.q0);
+                const uint64_t fm = f0 | f1 | f2;
                 for (uint32_t qb = qs; qb < qe; qb += 32) {
                     const uint32_t i = qb + lane;
-                    const bool ok = i < qe && (f0 & ~sm.q0[i]) == 0;
+                    const bool ok = i < qe && (fm & ~qw[i]) == 0;
                     const uint32_t b = __ballot_sync(0xffffffffu, ok);
                     if (ok) sa[na + __popc(b & lt_mask)] = (uint16_t)i;
                     na += __popc(b);
