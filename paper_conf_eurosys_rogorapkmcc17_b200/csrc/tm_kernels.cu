@@ -344,7 +344,7 @@ __device__ __forceinline__ void emit_keys(bool m, uint32_t row, uint32_t qg, con
 // Block 2 of one survivor whose blocks 0-1 passed in some lane, then emit.
 __device__ __forceinline__ void check_block2(bool hit01, uint32_t slot, uint64_t s2, uint32_t row,
                                              const ScanSmem &sm, const ScanParams &p, int lane,
-                                             unsigned long long &matched) {
+                                             uint32_t &matched) {
     const bool m = hit01 && (s2 & ~sm.q2[slot]) == 0;
     const uint32_t b = __ballot_sync(0xffffffffu, m);
     if (b) {
@@ -387,13 +387,17 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // register with no votes; only the (lane, survivor) pairs that pass (about 0.1% on the
 // Twitter-like workload) get the full six-word check, in a divergent loop whose trip count
 // is the largest per-lane pass count.
-template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false>
-__global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
+// MINB: resident CTAs per SM the register allocator must allow (__launch_bounds__); shared memory
+// caps residency at 8 CTAs, which ptxas cannot see (the scan's shared memory is dynamic).
+template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8>
+__global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     ScanSmem &sm = *reinterpret_cast<ScanSmem *>(smem_raw);
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
-    unsigned long long st_tests = 0, st_checks = 0, st_matched = 0;
+    // per-warp statistics, 32-bit (one item decides at most kChunk x range_rows pairs) and flushed to
+    // the 64-bit global counters at every item boundary
+    uint32_t st_tests = 0, st_checks = 0, st_matched = 0;
     const unsigned long long n_items = p.item_off[p.n_parts];
     if (blockIdx.x == 0 && threadIdx.x == 0) p.ctr->n_items = n_items;
     if (p.ctr->routed > p.qcap) return;  // query lists truncated: the host grows qidx and re-runs
@@ -406,6 +410,12 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
     constexpr uint32_t kUnionBase = 80;
 
     for (;;) {
+        if (lane == 0 && (st_tests | st_checks | st_matched)) {
+            atomicAdd(&p.ctr->tile_tests, (unsigned long long)st_tests);
+            atomicAdd(&p.ctr->pair_checks, (unsigned long long)st_checks);
+            atomicAdd(&p.ctr->matched_sets, (unsigned long long)st_matched);
+        }
+        st_tests = st_checks = st_matched = 0;
         if (threadIdx.x == 0) {
             sm.item = atomicAdd(&p.ctr->item_ctr, 1ULL);
             sm.unit_ctr = 0;
@@ -520,7 +530,7 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                         }
                     }
                     const uint32_t u0 = rlo + u * 64;
-                    st_checks += (unsigned long long)nq * (vend > u0 ? min(64u, vend - u0) : 0u);
+                    st_checks += nq * (vend > u0 ? min(64u, vend - u0) : 0u);
                     continue;
                 }
                 // direct check: rows (r, r+1) and (r+64, r+65) per lane, r = base + 2 lane; a tile
@@ -559,7 +569,7 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                         }
                     }
                 }
-                st_checks += (unsigned long long)nq * (vend > u0 ? min(128u, vend - u0) : 0u);
+                st_checks += nq * (vend > u0 ? min(128u, vend - u0) : 0u);
             }
             __syncthreads();
             continue;
@@ -668,8 +678,9 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                         uint32_t *swk = sm.sw[warp][0];
                         for (; j < na && nb <= (uint32_t)kSubW - 64; j += 64) {
                             const uint32_t ja = j + lane, jb = ja + 32;
-                            const uint32_t ia = min((uint32_t)sa[min(ja, (uint32_t)kChunk - 1)], (uint32_t)kChunk - 1);
-                            const uint32_t ib = min((uint32_t)sa[min(jb, (uint32_t)kChunk - 1)], (uint32_t)kChunk - 1);
+                            // sa[0, pe) holds valid slots (< kChunk); lanes past pe read slot 0
+                            const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
+                            const uint32_t ib = jb < pe ? (uint32_t)sa[jb] : 0u;
                             const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
                             const uint64_t b0 = sm.q0[ib], b1 = sm.q1[ib], b2 = sm.q2[ib];
                             const bool oka = ja < pe && ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
@@ -683,7 +694,7 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                         }
                         if (j < na && nb <= (uint32_t)kSubW - 32) {
                             const uint32_t ja = j + lane;
-                            const uint32_t ia = min((uint32_t)sa[min(ja, (uint32_t)kChunk - 1)], (uint32_t)kChunk - 1);
+                            const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
                             const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
                             const bool oka = ja < pe && ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
                             const uint32_t ba = __ballot_sync(0xffffffffu, oka);
@@ -691,7 +702,7 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                             nb += __popc(ba);
                             j += 32;
                         }
-                        st_checks += (unsigned long long)nb * nvalid;
+                        st_checks += nb * nvalid;
                         __syncwarp();
                         for (uint32_t k0 = 0; k0 < nb; k0 += 32) {
                             const uint32_t cnt = min(32u, nb - k0);
@@ -772,7 +783,7 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
                         nb += __popc(b);
                     }
                     st_tests += pe - pb;
-                    st_checks += (unsigned long long)nb * nvalid;
+                    st_checks += nb * nvalid;
                     // pad to a multiple of U with zeros (masked by k < nb below)
                     constexpr uint32_t kPad = UNION2 ? 8 : U;
                     if ((uint32_t)lane < ((kPad - (nb % kPad)) % kPad)) {
@@ -867,9 +878,9 @@ __global__ void __launch_bounds__(kScanWarps * 32) k_scan(const ScanParams p) {
         __syncthreads();
     }
     if (lane == 0) {
-        atomicAdd(&p.ctr->tile_tests, st_tests);
-        atomicAdd(&p.ctr->pair_checks, st_checks);
-        atomicAdd(&p.ctr->matched_sets, st_matched);
+        atomicAdd(&p.ctr->tile_tests, (unsigned long long)st_tests);
+        atomicAdd(&p.ctr->pair_checks, (unsigned long long)st_checks);
+        atomicAdd(&p.ctr->matched_sets, (unsigned long long)st_matched);
     }
 }
 
@@ -993,7 +1004,9 @@ ScanFn scan_fn(int variant) {
         case 2: return k_scan<4, true>;
         case 3: return k_scan<8, true>;
         case 4: return k_scan<4, false, true>;
-        case 5: return k_scan<4, false, false, true>;
+        // 72 registers and 7 CTAs/SM, no spills: 2.00 ms at C2 vs 2.10 ms with 64 registers and
+        // 8 CTAs (spills) and 2.05 ms with 76 registers and 6 CTAs (profiles/r1v29_minb.txt)
+        case 5: return k_scan<4, false, false, true, 7>;
         default: return k_scan<4, false>;
     }
 }
