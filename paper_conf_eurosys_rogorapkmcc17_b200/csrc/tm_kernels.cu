@@ -1030,7 +1030,8 @@ uint32_t range_rows_env(uint64_t n_rows) {
     const char *e = getenv("TM_RANGE_ROWS");
     if (!e) return def;
     const long v = atol(e);
-    return (v >= 256 && v <= (1L << 30) && v % 256 == 0) ? (uint32_t)v : def;
+    // at most 2^20 rows: one item then decides < 2^32 pairs (the kernel's 32-bit per-item statistics)
+    return (v >= 256 && v <= (1L << 20) && v % 256 == 0) ? (uint32_t)v : def;
 }
 
 int scan_grid(int device, int variant) {

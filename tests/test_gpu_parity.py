@@ -111,14 +111,17 @@ def test_row_order_needs_and_masks(c1):
         tmb.Database(c1.db, c1.key_off, c1.keys, tile_filter=0, row_order=1)
 
 
-@pytest.mark.parametrize("nq", [1, 3, 8, 9, 40])
+@pytest.mark.parametrize("nq", [1, 2, 3, 4, 5, 8, 9, 40])
 @pytest.mark.parametrize("max_p", [0xFFFFFFFF, 500])
-def test_small_batches(c1, nq, max_p):
-    """Batches of <= 8 routed queries take the unfiltered streaming path; 9 and
-    40 straddle it (per partition)."""
+@pytest.mark.parametrize("layout", [(0, 0), (1, 1)])
+def test_small_batches(c1, nq, max_p, layout):
+    """Batches of <= 8 routed queries take the unfiltered streaming path (<= 4: direct check
+    over 128-row units, 5-8: the two-word pre-check); 9 and 40 straddle it (per partition).
+    MAX_P 500 makes partitions whose padded row counts are not multiples of the unit."""
     qsel = np.arange(0, c1.queries.n_sets, c1.queries.n_sets // nq)[:nq]
     q = c1.queries.subset(qsel)
-    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=max_p) as db:
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=max_p, tile_filter=layout[0],
+                      row_order=layout[1]) as db:
         for unique in (False, True):
             got = db.match_batch(q, unique)
             want = o2.match_brute(o2.encode(c1.db), c1.key_off, c1.keys, o2.encode(q), unique)
