@@ -53,6 +53,7 @@ def _compile(src: str, verbose_ptxas: bool) -> str:
     obj = os.path.join(BUILD, os.path.basename(src) + ".o")
     cmd = [NVCC, "-c", src, "-o", obj, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(),
            "-Xcompiler", "-fPIC,-O3,-Wall", "--expt-relaxed-constexpr", "-DNDEBUG"]
+    cmd += os.environ.get("TM_NVCC_FLAGS", "").split()  # experiments only (e.g. -DTM_BLOCK_TILES=4)
     if verbose_ptxas and src.endswith(".cu"):
         cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)

@@ -251,17 +251,19 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         sp.wsel = db->wsel.as<uint8_t>();
         sp.range_rows = range_rows;
         // variant: TM_SCAN_VARIANT if set; else a call whose partition batches are all small
-        // (Q <= kSmallBatch) takes the streaming path only -- up to four queries checked directly
-        // in the leaner variant-0 kernel (fewer live registers), 5-8 through variant 5's two-word
-        // pre-check (scripts/hbm_sweep.py) -- and is not a
+        // (Q <= kSmallBatch) takes the streaming path only, in the streaming-only kernels (small
+        // shared memory: 8 CTAs/SM) -- up to four queries checked directly (variant 6), 5-8
+        // through the two-word pre-check (variant 7; scripts/hbm_sweep.py) -- and is not a
         // tuning sample (the candidates differ only in the filtered path); other calls cycle
         // through the candidates on the handle's first qualifying calls, then keep the cheapest
         const int forced = scan_variant_env();
         int var = forced;
+        // the streaming-only kernels cannot take a filtered batch: a forced 6 / 7 maps to 0 / 5 then
+        if (var >= 6 && Q > (uint64_t)kSmallBatch) var = var == 6 ? 0 : 5;
         db->call_tunes = false;
         if (var < 0) {
             if (Q <= (uint64_t)kSmallBatch) {
-                var = Q <= 4 ? 0 : 5;
+                var = Q <= 4 ? 6 : 7;
             } else {
                 const int c = 63 - __builtin_clzll(Q);
                 db->call_class = c;

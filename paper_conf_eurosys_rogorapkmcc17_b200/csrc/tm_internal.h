@@ -22,10 +22,13 @@ constexpr int kTile = 32;  // rows per warp tile (= one warp, Alg. 4 "thread blo
 
 // Scan-kernel geometry.
 constexpr int kScanWarps = 4;      // warps per CTA
-constexpr int kChunk = 512;        // queries per work item (per-partition batch)
+#ifndef TM_CHUNK
+#define TM_CHUNK 640
+#endif
+constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch); 640 fits 7 CTAs/SM of shared memory and measured 1.3% faster than 512 (profiles/r1v34_ab.txt)
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
-constexpr int kScanVariants = 6;    // k_scan variants (TM_SCAN_VARIANT)
+constexpr int kScanVariants = 8;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {5, 2, 0};  // variants the handle times on its first calls (first = default)
 constexpr int kTuneN = 3;
 

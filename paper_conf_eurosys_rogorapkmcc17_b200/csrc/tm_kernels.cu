@@ -14,6 +14,7 @@
 // plus CUB scans / radix sorts / unique (S2, S8) and small gather kernels used
 // by tm_build.
 #include <cub/cub.cuh>
+#include <type_traits>
 
 #include "tm_internal.h"
 
@@ -205,7 +206,10 @@ __global__ void k_items(const unsigned long long *__restrict__ word_off, uint32_
 // the common mask of a 256-row block (8 tiles), level B tests the level-A
 // survivors against the mask of each 32-row tile; only level-B survivors are
 // checked against the tile's 32 sets (Alg. 3).
-constexpr int kBlockTiles = 8;   // tiles per level-A block (256 rows)
+#ifndef TM_BLOCK_TILES
+#define TM_BLOCK_TILES 8
+#endif
+constexpr int kBlockTiles = TM_BLOCK_TILES;  // tiles per level-A block (8: 256 rows)
 constexpr int kSubB = 128;       // level-B survivors buffered per pass
 constexpr int kQSub = 128;       // queries per unit
 
@@ -213,7 +217,10 @@ constexpr int kQSub = 128;       // queries per unit
 // survivor k at sw[warp][w][k]; the plane stride (kSubW + 4 words = 400 B, 16 B mod 128)
 // puts the six planes on disjoint bank quads, so the per-lane-plane LDS.128 of the
 // pre-check is conflict-free.
-constexpr int kSubW = 96;                         // level-B survivors per pass (WORD1)
+#ifndef TM_SUBW
+#define TM_SUBW 96
+#endif
+constexpr int kSubW = TM_SUBW;                         // level-B survivors per pass (WORD1)
 constexpr int kSubWStride = kSubW + 4;
 
 struct ScanSmem {
@@ -228,6 +235,24 @@ struct ScanSmem {
     const uint32_t *qid;                           // batch slot -> query index in the call (global)
     unsigned long long item;
     unsigned int unit_ctr;
+    unsigned long long cnt[3];                     // CTA totals: tile tests, pair checks, matched sets
+};
+
+// Shared memory of the streaming-only kernels (calls of <= kSmallBatch queries: every partition batch
+// is small): the same members as ScanSmem, sized for the streaming path, so that residency is
+// bounded by registers (8 CTAs/SM) instead of ScanSmem's 32 KB (7 CTAs/SM).
+struct StreamSmem {
+    uint64_t q0[kSmallBatch], q1[kSmallBatch], q2[kSmallBatch];
+    uint16_t sa[kScanWarps][1];
+    union {
+        uint4 sbuf[kScanWarps][1];
+        uint32_t sw[1][6][kSubWStride];   // warp 0's planes hold the batch (pre-check)
+    };
+    uint16_t sbi[kScanWarps][1];
+    const uint32_t *qid;
+    unsigned long long item;
+    unsigned int unit_ctr;
+    unsigned long long cnt[3];
 };
 
 __device__ __forceinline__ uint4 lds128(uint32_t addr) {
@@ -402,10 +427,12 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // is the largest per-lane pass count.
 // MINB: resident CTAs per SM the register allocator must allow (__launch_bounds__); shared memory
 // caps residency at 8 CTAs, which ptxas cannot see (the scan's shared memory is dynamic).
-template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8>
+// STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
+template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8, bool STREAM = false>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    ScanSmem &sm = *reinterpret_cast<ScanSmem *>(smem_raw);
+    using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
+    Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint32_t lt_mask = (1u << lane) - 1u;
     // per-warp statistics, 32-bit (one item decides at most kChunk x range_rows pairs) and flushed to
@@ -414,6 +441,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
     const unsigned long long n_items = p.item_off[p.n_parts];
     if (blockIdx.x == 0 && threadIdx.x == 0) p.ctr->n_items = n_items;
     if (p.ctr->routed > p.qcap) return;  // query lists truncated: the host grows qidx and re-runs
+    if (threadIdx.x < 3) sm.cnt[threadIdx.x] = 0;  // ordered before any flush by the item loop's barrier
     uint16_t *sa = sm.sa[warp];
     uint4 *sbuf = sm.sbuf[warp];
     uint16_t *sbi = sm.sbi[warp];
@@ -423,10 +451,10 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
     constexpr uint32_t kUnionBase = 80;
 
     for (;;) {
-        if (lane == 0 && (st_tests | st_checks | st_matched)) {
-            atomicAdd(&p.ctr->tile_tests, (unsigned long long)st_tests);
-            atomicAdd(&p.ctr->pair_checks, (unsigned long long)st_checks);
-            atomicAdd(&p.ctr->matched_sets, (unsigned long long)st_matched);
+        if (lane == 0 && (st_tests | st_checks | st_matched)) {  // shared atomics: no global contention
+            atomicAdd(&sm.cnt[0], (unsigned long long)st_tests);
+            atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
+            atomicAdd(&sm.cnt[2], (unsigned long long)st_matched);
         }
         st_tests = st_checks = st_matched = 0;
         if (threadIdx.x == 0) {
@@ -456,6 +484,9 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
         const uint32_t rlo = prow + range * rr;
         const uint32_t rhi = min(rlo + rr, prow + rows);
 
+        if constexpr (STREAM) {
+            if (nq > (uint32_t)kSmallBatch) __trap();  // the host launches STREAM kernels for Q <= kSmallBatch only
+        }
         if (threadIdx.x == 0) sm.qid = p.qidx + qbeg;
         // stage the query batch (the batch of queries of partition p)
         for (uint32_t i = threadIdx.x; i < nq; i += blockDim.x) {
@@ -588,6 +619,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
             continue;
         }
 
+        if constexpr (!STREAM) {
         const uint32_t ntile = (rhi - rlo) / kTile;
         const uint32_t nblock = (ntile + kBlockTiles - 1) / kBlockTiles;
         // unit = (256-row block, query sub-range), taken dynamically through unit_ctr;
@@ -888,12 +920,20 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                 }
             }
         }
+        }  // !STREAM
         __syncthreads();
     }
-    if (lane == 0) {
-        atomicAdd(&p.ctr->tile_tests, (unsigned long long)st_tests);
-        atomicAdd(&p.ctr->pair_checks, (unsigned long long)st_checks);
-        atomicAdd(&p.ctr->matched_sets, (unsigned long long)st_matched);
+    // the loop ends for all warps together (after the barrier that read the last item)
+    if (lane == 0 && (st_tests | st_checks | st_matched)) {
+        atomicAdd(&sm.cnt[0], (unsigned long long)st_tests);
+        atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
+        atomicAdd(&sm.cnt[2], (unsigned long long)st_matched);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (sm.cnt[0]) atomicAdd(&p.ctr->tile_tests, sm.cnt[0]);
+        if (sm.cnt[1]) atomicAdd(&p.ctr->pair_checks, sm.cnt[1]);
+        if (sm.cnt[2]) atomicAdd(&p.ctr->matched_sets, sm.cnt[2]);
     }
 }
 
@@ -1020,16 +1060,23 @@ ScanFn scan_fn(int variant) {
         // 72 registers and 7 CTAs/SM, no spills: 2.00 ms at C2 vs 2.10 ms with 64 registers and
         // 8 CTAs (spills) and 2.05 ms with 76 registers and 6 CTAs (profiles/r1v29_minb.txt)
         case 5: return k_scan<4, false, false, true, 7>;
+        case 6: return k_scan<4, false, false, false, 8, true>;  // streaming only, direct check
+        case 7: return k_scan<4, false, false, true, 8, true>;   // streaming only, word pre-check
         default: return k_scan<4, false>;
     }
 }
 }  // namespace
 
+size_t scan_smem(int variant) {
+    return variant >= 6 ? sizeof(StreamSmem) : sizeof(ScanSmem);
+}
+
 int scan_variant_env() {
     // TM_SCAN_VARIANT forces a scan-kernel variant: 0 = 4 survivors per
     // iteration, blocks 0-1 first; 1 = 8, blocks 0-1; 2 = 4, all three blocks; 3 = 8, all three;
-    // 4 = pair unions first; 5 = per-lane word pre-check (WORD1).  Unset (-1): the handle tunes
-    // on its first calls.
+    // 4 = pair unions first; 5 = per-lane word pre-check (WORD1); 6 / 7 = streaming-only kernels
+    // (direct check / word pre-check; calls of <= kSmallBatch queries, else mapped to 0 / 5 by the
+    // caller).  Unset (-1): the handle tunes on its first calls.
     const char *e = getenv("TM_SCAN_VARIANT");
     if (!e) return -1;
     const int v = atoi(e);
@@ -1051,15 +1098,15 @@ int scan_grid(int device, int variant) {
     int sms = 0, per = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
     ScanFn f = scan_fn(variant);
-    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(ScanSmem));
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, kScanWarps * 32, sizeof(ScanSmem));
+    cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem(variant));
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, kScanWarps * 32, scan_smem(variant));
     if (per < 1) per = 1;
     if (sms < 1) sms = 1;
     return sms * per;
 }
 
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant) {
-    scan_fn(variant)<<<grid, kScanWarps * 32, sizeof(ScanSmem), s>>>(p);
+    scan_fn(variant)<<<grid, kScanWarps * 32, scan_smem(variant), s>>>(p);
     return cudaGetLastError();
 }
 

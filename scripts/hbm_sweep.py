@@ -39,7 +39,7 @@ def main():
         db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=tmb.TM_NO_PARTITIONING, tile_filter=filt)
         build_s = time.time() - t0
         rows = db.stats()["n_rows"]
-        for B in (1, 2, 4, 8, 16, 32, 64, 128, 256):
+        for B in [int(x) for x in os.environ.get("HBM_B", "1,2,4,8,16,32,64,128,256").split(",")]:
             q = wl.queries.subset(np.arange(B))
             arrs = [np.ascontiguousarray(a) for a in (q.vocab_bytes, q.vocab_off.view(np.int64),
                                                       q.tag_idx.view(np.int32), q.set_off.view(np.int64))]

@@ -116,8 +116,9 @@ def test_row_order_needs_and_masks(c1):
 @pytest.mark.parametrize("layout", [(0, 0), (1, 1)])
 def test_small_batches(c1, nq, max_p, layout):
     """Batches of <= 8 routed queries take the unfiltered streaming path (<= 4: direct check
-    over 128-row units, 5-8: the two-word pre-check); 9 and 40 straddle it (per partition).
-    MAX_P 500 makes partitions whose padded row counts are not multiples of the unit."""
+    over 128-row units, 5-8: the two-word pre-check), in the streaming-only kernels when the
+    whole call has <= 8 queries; 9 and 40 straddle it (per partition).  MAX_P 500 makes
+    partitions whose padded row counts are not multiples of the unit."""
     qsel = np.arange(0, c1.queries.n_sets, c1.queries.n_sets // nq)[:nq]
     q = c1.queries.subset(qsel)
     with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=max_p, tile_filter=layout[0],
@@ -126,6 +127,8 @@ def test_small_batches(c1, nq, max_p, layout):
             got = db.match_batch(q, unique)
             want = o2.match_brute(o2.encode(c1.db), c1.key_off, c1.keys, o2.encode(q), unique)
             assert_pairs_equal(got, want, f"nq={nq}")
+            if nq <= 8:
+                assert db.stats()["scan_variant"] == (6 if nq <= 4 else 7)
 
 
 @pytest.mark.parametrize("max_p", [200_000, 1000, 64, 1])
@@ -207,7 +210,7 @@ def test_c2_full_parity(c2, c2_oracle, layout):
     assert np.unique(got[0]).size == wl.queries.n_sets
 
 
-@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5"])
+@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7"])
 def test_c2_every_scan_variant(c2, c2_oracle, variant, monkeypatch):
     """Every scan-kernel variant (TM_SCAN_VARIANT) gives the oracle's
     pairs at C2, in the layout bench.py times (balanced splits + AND masks)."""
@@ -218,7 +221,8 @@ def test_c2_every_scan_variant(c2, c2_oracle, variant, monkeypatch):
         for unique in (False, True):
             got = db.match_batch(wl.queries, unique)
             assert_pairs_equal(got, c2_oracle[unique], f"C2 variant={variant} unique={unique}")
-            assert db.stats()["scan_variant"] == int(variant)
+            # the streaming-only kernels (6, 7) cannot take a filtered call: they map to 0 / 5
+            assert db.stats()["scan_variant"] == {"6": 0, "7": 5}.get(variant, int(variant))
 
 
 def test_c2_sampled_against_brute_force(c2):
