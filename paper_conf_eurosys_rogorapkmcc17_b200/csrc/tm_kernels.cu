@@ -213,6 +213,11 @@ constexpr int kBlockTiles = TM_BLOCK_TILES;  // tiles per level-A block (8: 256 
 constexpr int kSubB = 128;       // level-B survivors buffered per pass
 constexpr int kQSub = 128;       // queries per unit
 
+// Matches are staged per warp (kPend entries in shared memory) and emitted in batches: one
+// global atomic per batch instead of one per matching warp step (the output counter is a single
+// address every SM hits).
+constexpr uint32_t kPend = 8;
+
 // WORD1 survivor planes: word w (= 32-bit half w & 1 of block w >> 1) of level-B
 // survivor k at sw[warp][w][k]; the plane stride (kSubW + 4 words = 400 B, 16 B mod 128)
 // puts the six planes on disjoint bank quads, so the per-lane-plane LDS.128 of the
@@ -236,6 +241,7 @@ struct ScanSmem {
     unsigned long long item;
     unsigned int unit_ctr;
     unsigned long long cnt[3];                     // CTA totals: tile tests, pair checks, matched sets
+    uint2 pend[kScanWarps][kPend];                 // per-warp matches (row, query) awaiting emission
 };
 
 // Shared memory of the streaming-only kernels (calls of <= kSmallBatch queries: every partition batch
@@ -253,6 +259,7 @@ struct StreamSmem {
     unsigned long long item;
     unsigned int unit_ctr;
     unsigned long long cnt[3];
+    uint2 pend[kScanWarps][kPend];
 };
 
 __device__ __forceinline__ uint4 lds128(uint32_t addr) {
@@ -340,24 +347,10 @@ __device__ __forceinline__ void tile_prefix(uint64_t f0, uint64_t f1, uint64_t f
     p2 = f2 & k2;
 }
 
-// Emit the (query, key) pairs of the lanes whose set matched (warp-uniform
-// call).  One atomic per warp reserves the output range (warp-aggregated
-// compaction replacing the per-pair atomic of PAPER.md:158); each matching
-// lane then writes its set's keys (key lookup).
-// bm = the warp's ballot of m (warp-uniform).  One matching lane -- the common case, matches are
-// ~0.03% of the pair checks -- reserves its own range: no warp prefix sum.
-__device__ __forceinline__ void emit_keys(bool m, uint32_t bm, uint32_t row, uint32_t qg, const ScanParams &p,
-                                          int lane) {
-    if ((bm & (bm - 1)) == 0) {
-        if (m) {
-            const uint32_t kb = __ldg(p.key_off + row), nk = __ldg(p.key_off + row + 1) - kb;
-            unsigned long long o = nk ? atomicAdd(&p.ctr->n_out, (unsigned long long)nk) : 0ULL;
-            const uint64_t hi = (uint64_t)qg << 32;
-            for (uint32_t j = 0; j < nk; ++j, ++o)
-                if (o < p.cap) p.out[o] = hi | (uint64_t)__ldg(p.keys + kb + j);
-        }
-        return;
-    }
+// Emit the (query, key) pairs of the lanes whose set matched: the key lookup and a
+// warp-aggregated output reservation (replacing the per-pair atomic of PAPER.md:158).  bm = the
+// warp's ballot of m (warp-uniform call); m lanes write their set's keys.
+__device__ __forceinline__ void emit_direct(bool m, uint32_t row, uint32_t qg, const ScanParams &p, int lane) {
     uint32_t kb = 0, nk = 0;
     if (m) {
         kb = __ldg(p.key_off + row);
@@ -379,15 +372,59 @@ __device__ __forceinline__ void emit_keys(bool m, uint32_t bm, uint32_t row, uin
         if (o < p.cap) p.out[o] = hi | (uint64_t)__ldg(p.keys + kb + j);
 }
 
+// Emit the warp's staged matches (lanes 0..npend-1 take one each); warp-uniform call.
+__device__ __forceinline__ void flush_pend(uint2 *pend, uint32_t &npend, const ScanParams &p, int lane) {
+    if (!npend) return;
+    __syncwarp();
+    const bool m = (uint32_t)lane < npend;
+    uint2 e = make_uint2(0u, 0u);
+    if (m) e = pend[lane];
+    uint32_t kb = 0, nk = 0;
+    if (m) {
+        kb = __ldg(p.key_off + e.x);
+        nk = __ldg(p.key_off + e.x + 1) - kb;
+    }
+    uint32_t incl = nk;
+#pragma unroll
+    for (int o = 1; o < (int)kPend; o <<= 1) {
+        const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += t;
+    }
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, kPend - 1);
+    unsigned long long base = 0;
+    if (lane == (int)kPend - 1 && total) base = atomicAdd(&p.ctr->n_out, (unsigned long long)total);
+    base = __shfl_sync(0xffffffffu, base, kPend - 1);
+    unsigned long long o = base + (incl - nk);
+    const uint64_t hi = (uint64_t)e.y << 32;
+    for (uint32_t j = 0; j < nk; ++j, ++o)
+        if (o < p.cap) p.out[o] = hi | (uint64_t)__ldg(p.keys + kb + j);
+    npend = 0;
+    __syncwarp();
+}
+
+// Stage the matches of one warp step (bm = ballot of m, nonzero, warp-uniform); a step with more
+// matches than the stage holds is emitted directly.
+__device__ __forceinline__ void emit_keys(bool m, uint32_t bm, uint32_t row, uint32_t qg, const ScanParams &p,
+                                          int lane, uint2 *pend, uint32_t &npend) {
+    const uint32_t c = __popc(bm);
+    if (npend + c > kPend) flush_pend(pend, npend, p, lane);
+    if (c > kPend) {
+        emit_direct(m, row, qg, p, lane);
+        return;
+    }
+    if (m) pend[npend + __popc(bm & ((1u << lane) - 1u))] = make_uint2(row, qg);
+    npend += c;
+}
+
 // Block 2 of one survivor whose blocks 0-1 passed in some lane, then emit.
 __device__ __forceinline__ void check_block2(bool hit01, uint32_t slot, uint64_t s2, uint32_t row,
-                                             const ScanSmem &sm, const ScanParams &p, int lane,
-                                             uint32_t &matched) {
+                                             ScanSmem &sm, const ScanParams &p, int lane,
+                                             uint32_t &matched, uint32_t &npend) {
     const bool m = hit01 && (s2 & ~sm.q2[slot]) == 0;
     const uint32_t b = __ballot_sync(0xffffffffu, m);
     if (b) {
         matched += __popc(b);
-        emit_keys(m, b, row, __ldg(sm.qid + slot), p, lane);
+        emit_keys(m, b, row, __ldg(sm.qid + slot), p, lane, sm.pend[threadIdx.x >> 5], npend);
     }
 }
 
@@ -438,6 +475,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
     // per-warp statistics, 32-bit (one item decides at most kChunk x range_rows pairs) and flushed to
     // the 64-bit global counters at every item boundary
     uint32_t st_tests = 0, st_checks = 0, st_matched = 0;
+    uint32_t npend = 0;  // the warp's staged matches (sm.pend[warp])
     const unsigned long long n_items = p.item_off[p.n_parts];
     if (blockIdx.x == 0 && threadIdx.x == 0) p.ctr->n_items = n_items;
     if (p.ctr->routed > p.qcap) return;  // query lists truncated: the host grows qidx and re-runs
@@ -570,7 +608,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                         const uint32_t bm = __ballot_sync(0xffffffffu, m);
                         if (bm) {
                             st_matched += __popc(bm);
-                            emit_keys(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane);
+                            emit_keys(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane, sm.pend[warp], npend);
                         }
                     }
                     const uint32_t u0 = rlo + u * 64;
@@ -608,7 +646,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                             const uint32_t bq = __ballot_sync(0xffffffffu, hh[e]);
                             if (bq) {
                                 st_matched += __popc(bq);
-                                emit_keys(hh[e], bq, rr4[e], qg, p, lane);
+                                emit_keys(hh[e], bq, rr4[e], qg, p, lane, sm.pend[warp], npend);
                             }
                         }
                     }
@@ -788,7 +826,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                                 const uint32_t bm = __ballot_sync(0xffffffffu, m);
                                 if (bm) {
                                     st_matched += __popc(bm);
-                                    emit_keys(m, bm, row, m ? __ldg(sm.qid + sbi[e]) : 0u, p, lane);
+                                    emit_keys(m, bm, row, m ? __ldg(sm.qid + sbi[e]) : 0u, p, lane, sm.pend[warp], npend);
                                 }
                             }
                         }
@@ -869,7 +907,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                                         const uint4 v = lds128(sb_addr + e * 16);
                                         const bool h = ((a0l & ~v.x) | (a0h & ~v.y) | (a1l & ~v.z) | (a1h & ~v.w)) == 0;
                                         if (__any_sync(0xffffffffu, h))
-                                            check_block2(h, sbi[e], s2, row, sm, p, lane, st_matched);
+                                            check_block2(h, sbi[e], s2, row, sm, p, lane, st_matched, npend);
                                     }
                                 }
                             }
@@ -907,10 +945,10 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                                         const uint32_t bm = __ballot_sync(0xffffffffu, m);
                                         if (bm) {
                                             st_matched += __popc(bm);
-                                            emit_keys(m, bm, row, __ldg(sm.qid + slot[j]), p, lane);
+                                            emit_keys(m, bm, row, __ldg(sm.qid + slot[j]), p, lane, sm.pend[warp], npend);
                                         }
                                     } else {
-                                        check_block2(h[j], sbi[k + j], s2, row, sm, p, lane, st_matched);
+                                        check_block2(h[j], sbi[k + j], s2, row, sm, p, lane, st_matched, npend);
                                     }
                                 }
                             }
@@ -924,6 +962,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
         __syncthreads();
     }
     // the loop ends for all warps together (after the barrier that read the last item)
+    flush_pend(sm.pend[warp], npend, p, lane);
     if (lane == 0 && (st_tests | st_checks | st_matched)) {
         atomicAdd(&sm.cnt[0], (unsigned long long)st_tests);
         atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
