@@ -293,6 +293,19 @@ def run_ours(args):
             host[out.n:].copy_(kt)
         return out.n * 8
 
+    # the handle times its scan-kernel variants on its first calls of a batch size (DESIGN.md
+    # sec. 6): finish that before the W warm-up steps, so that no timed step runs a candidate
+    tune_calls = 0
+    for _ in range(16):
+        step_device()
+        tune_calls += 1
+        done = 0 if db.stats()["tuning"] else 1
+        if world > 1:   # the ranks agree (the sharded step has collectives inside)
+            t = torch.tensor([done], device=f"cuda:{dev}" if pg == "nccl" else "cpu", dtype=torch.int32)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN)
+            done = int(t.item())
+        if done:
+            break
     for _ in range(args.warmup):
         step_device()
         step_e2e()
@@ -394,6 +407,7 @@ def run_ours(args):
                                                 "pair_checks", "matched_sets", "emitted_pairs", "result_pairs",
                                                 "work_items", "exact_checked", "exact_kept")},
             "build_s": build_s,
+            "tuning_calls": tune_calls,   # untimed calls that finished the variant tuning before the W warm-ups
         }
         if not args.no_cpu_baseline and world == 1:
             from oracle import o2

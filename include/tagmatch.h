@@ -213,7 +213,8 @@ typedef struct {
     uint64_t exact_checked;    /* exact mode: (query, entry) Bloom matches checked      */
     uint64_t exact_kept;       /* exact mode: ... that are exact subsets                  */
     uint32_t scan_variant;     /* scan-kernel variant of the last call */
-    uint32_t pad_;
+    uint32_t tuning;           /* 1: the handle is still timing variants for batches of this size
+                                  (ceil log2 class), so later calls may run other variants */
 } tm_stats_t;
 
 tm_status tm_stats(const tm_db *db, tm_stats_t *out);

@@ -381,6 +381,7 @@ void finish_timing(tm_db *db, cudaStream_t s) {
             db->variant[c] = best;
         }
     }
+    if (db->call_tunes) st.tuning = db->tune_calls[db->call_class] < 2 * kTuneN ? 1u : 0u;
     TMCK(cudaEventElapsedTime(&ms, db->ev[3], db->ev[4]));
     st.merge_ms = ms;
     TMCK(cudaEventElapsedTime(&ms, db->ev[0], db->ev[4]));

@@ -72,7 +72,7 @@ class tm_stats_t(ctypes.Structure):
                [(n, ctypes.c_double) for n in ("encode_ms", "route_ms", "scan_ms", "merge_ms", "total_ms")] + \
                [("scan_launches", ctypes.c_uint32), ("kernel_launches", ctypes.c_uint32),
                 ("exact_checked", ctypes.c_uint64), ("exact_kept", ctypes.c_uint64),
-                ("scan_variant", ctypes.c_uint32), ("pad_", ctypes.c_uint32)]
+                ("scan_variant", ctypes.c_uint32), ("tuning", ctypes.c_uint32)]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}

@@ -44,7 +44,11 @@ def main():
         dq = tmb.device_tagsets(dt[0].data_ptr(), dt[1].data_ptr(), dt[2].data_ptr(), dt[3].data_ptr(),
                                 arrs[0].size, arrs[1].size - 1, arrs[2].size, q.n_sets)
         for unique in (True, False):
-            for _ in range(3):
+            for _ in range(16):   # warm-up, then until the handle has tuned this batch size
+                db.match_batch_device(dq, unique, stream.cuda_stream)
+                if not db.stats()["tuning"]:
+                    break
+            for _ in range(2):
                 db.match_batch_device(dq, unique, stream.cuda_stream)
             ms = []
             for _ in range(steps):
