@@ -10,8 +10,9 @@ sets, 100k-query stream, MAX_P = 200K), `match` (Table 1).
 
 value  : queries/s over all ranks, inputs resident in HBM (tm_match_batch_device),
          per-step CUDA events on the launching stream, L2 flushed between steps.
-e2e    : queries/s through tm_match_batch with pinned host queries (H2D inside
-         the timed region) and the sorted pairs copied back to host (D2H).
+e2e    : queries/s through tm_match_batch_csr with pinned host queries (H2D inside
+         the timed region) and the result -- every query's sorted keys -- copied
+         back to host (D2H: 4 B per pair + 8 B per query offset).
 N > 1  : one process per GPU (torchrun); every rank holds a replica of the
          database and matches its own query batch (replicated mode, PAPER.md:110,
          228: no data-path collective) -> "scaling": "weak"; time = max over ranks.
@@ -277,11 +278,11 @@ def run_ours(args):
 
     def step_e2e():
         """Public API end to end: host queries in, host pairs out; returns D2H bytes."""
-        if not sharded:
-            p = db.match_batch_raw(hq, unique)
+        if not sharded:   # per-query key lists: 4 B per pair + 8 B per query come back
+            p = db.match_batch_csr_raw(hq, unique)
             n = p.n
-            db.free_pairs(p)
-            return n * 8
+            db.free_csr(p)
+            return n * 4 + (Q + 1) * 8
         for d, h in zip(dt_, pinned):          # H2D of the batch (every rank receives it)
             d.copy_(h, non_blocking=True)
         out = db.match_batch_sharded_device(dq, unique, stream.cuda_stream)

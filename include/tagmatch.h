@@ -47,7 +47,7 @@
 extern "C" {
 #endif
 
-#define TM_ABI_VERSION 2u
+#define TM_ABI_VERSION 3u
 /* Bloom filter width and number of hash functions. */
 #define TM_SIG_BITS 192u
 #define TM_SIG_WORDS 3u
@@ -133,6 +133,19 @@ typedef struct {
     void *priv_; /* library bookkeeping; do not touch */
 } tm_pairs;
 
+/* Result as per-query key lists in host memory (match / match-unique
+ * return, for each query, its keys), allocated by the library (pinned), released
+ * by tm_csr_free().  Query j's keys are key[q_off[j] .. q_off[j+1]), ascending;
+ * q_off[0] = 0 and q_off[n_queries] = n.  The same pairs as tm_pairs, in the
+ * same order, with 4 B per pair + 8 B per query instead of 8 B per pair. */
+typedef struct {
+    uint64_t n_queries;
+    uint64_t n;
+    uint64_t *q_off; /* n_queries + 1 */
+    uint32_t *key;   /* n */
+    void *priv_;     /* library bookkeeping; do not touch */
+} tm_csr;
+
 /* Result pairs in device memory owned by the tm_db; valid until the next call
  * on the same handle or tm_free. */
 typedef struct {
@@ -164,6 +177,12 @@ tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32
  * Errors: TM_EINVAL, TM_ERANGE, TM_ECUDA, TM_ENOMEM. */
 tm_status tm_match_batch(tm_db *db, const tm_tagsets *queries, int unique, tm_pairs *out);
 
+/* tm_match_batch with the result as per-query key lists (tm_csr): the query
+ * offsets are found on the GPU (one binary search per query over the sorted
+ * pairs) and only the keys and the offsets are copied back.
+ * Errors: as tm_match_batch. */
+tm_status tm_match_batch_csr(tm_db *db, const tm_tagsets *queries, int unique, tm_csr *out);
+
 /* Same as tm_match_batch with the query arrays already resident in device
  * memory of the handle's device (pointers in *queries are device pointers;
  * the struct itself is host memory) and the result left in device memory.
@@ -173,6 +192,7 @@ tm_status tm_match_batch_device(tm_db *db, const tm_tagsets *queries, int unique
                                 void *stream);
 
 void tm_pairs_free(tm_pairs *p); /* NULL-safe; resets *p */
+void tm_csr_free(tm_csr *c);     /* NULL-safe; resets *c */
 void tm_free(tm_db *db);         /* NULL-safe */
 const char *tm_strerror(tm_status s);
 const char *tm_last_error(void); /* thread-local detail of the last failure ("" if none) */

@@ -738,14 +738,9 @@ tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32
     }
 }
 
-tm_status tm_match_batch(tm_db *db, const tm_tagsets *q, int unique, tm_pairs *out) {
-    TM_API_BEGIN
-    if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
-    if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
-    check_tagsets_shape(q, "queries");
-    DeviceGuard g(db->device);
-    cudaStream_t s = db->stream;
-    // one H2D copy of the query batch
+namespace tmb {
+// H2D of a host query batch into the handle's input buffers; returns the device-side tagsets.
+tm_tagsets upload_queries(tm_db *db, const tm_tagsets *q, cudaStream_t s) {
     tm_tagsets dq = *q;
     dq.vocab_bytes = nullptr;
     dq.vocab_off = nullptr;
@@ -769,6 +764,18 @@ tm_status tm_match_batch(tm_db *db, const tm_tagsets *q, int unique, tm_pairs *o
     } else {
         dq.tag_idx = nullptr;
     }
+    return dq;
+}
+}  // namespace tmb
+
+tm_status tm_match_batch(tm_db *db, const tm_tagsets *q, int unique, tm_pairs *out) {
+    TM_API_BEGIN
+    if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
+    if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
+    check_tagsets_shape(q, "queries");
+    DeviceGuard g(db->device);
+    cudaStream_t s = db->stream;
+    const tm_tagsets dq = upload_queries(db, q, s);  // one H2D copy of the query batch
     const uint64_t n = match_core(db, &dq, unique, s);
     PinnedBlock *blk = pinned_get(std::max<uint64_t>(n, 1) * 8);
     uint32_t *hq = static_cast<uint32_t *>(blk->p), *hk = hq + n;
@@ -794,6 +801,43 @@ tm_status tm_match_batch(tm_db *db, const tm_tagsets *q, int unique, tm_pairs *o
     TM_API_END
 }
 
+tm_status tm_match_batch_csr(tm_db *db, const tm_tagsets *q, int unique, tm_csr *out) {
+    TM_API_BEGIN
+    if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
+    if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
+    check_tagsets_shape(q, "queries");
+    DeviceGuard g(db->device);
+    cudaStream_t s = db->stream;
+    const tm_tagsets dq = upload_queries(db, q, s);
+    const uint64_t n = match_core(db, &dq, unique, s);
+    const uint64_t Q = q->n_sets;
+    db->res_off.ensure((Q + 1) * 8);
+    const uint64_t *sorted = n ? db->last_sorted : nullptr;
+    TMCK(launch_query_offsets(sorted, n, Q, db->res_off.as<uint64_t>(), s));
+    PinnedBlock *blk = pinned_get((Q + 1) * 8 + std::max<uint64_t>(n, 1) * 4);
+    uint64_t *hoff = static_cast<uint64_t *>(blk->p);
+    uint32_t *hk = reinterpret_cast<uint32_t *>(hoff + Q + 1);
+    cudaError_t e1 = cudaMemcpyAsync(hoff, db->res_off.p, (Q + 1) * 8, cudaMemcpyDeviceToHost, s);
+    cudaError_t e2 = n ? cudaMemcpyAsync(hk, db->res_k.p, n * 4, cudaMemcpyDeviceToHost, s) : cudaSuccess;
+    if (e1 != cudaSuccess || e2 != cudaSuccess) {
+        pinned_put(blk);
+        throw CudaFail{e1 != cudaSuccess ? e1 : e2, "cudaMemcpyAsync(D2H results)", __LINE__};
+    }
+    try {
+        finish_timing(db, s);
+    } catch (...) {
+        pinned_put(blk);
+        throw;
+    }
+    out->n_queries = Q;
+    out->n = n;
+    out->q_off = hoff;
+    out->key = hk;
+    out->priv_ = blk;
+    return TM_OK;
+    TM_API_END
+}
+
 tm_status tm_match_batch_device(tm_db *db, const tm_tagsets *q, int unique, tm_dev_pairs *out, void *stream) {
     TM_API_BEGIN
     if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
@@ -810,6 +854,16 @@ tm_status tm_match_batch_device(tm_db *db, const tm_tagsets *q, int unique, tm_d
     out->key = db->res_k.as<uint32_t>();
     return TM_OK;
     TM_API_END
+}
+
+void tm_csr_free(tm_csr *c) {
+    if (!c) return;
+    if (c->priv_) tmb::pinned_put(static_cast<tmb::PinnedBlock *>(c->priv_));
+    c->n_queries = 0;
+    c->n = 0;
+    c->q_off = nullptr;
+    c->key = nullptr;
+    c->priv_ = nullptr;
 }
 
 void tm_pairs_free(tm_pairs *p) {

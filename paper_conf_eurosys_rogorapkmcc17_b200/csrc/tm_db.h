@@ -112,7 +112,7 @@ struct tm_db {
     double build_ms = 0;
     // per-call workspace
     DevBuf in_bytes, in_voff, in_tidx, in_soff;  // host-API staging of the queries
-    DevBuf vsig, qplanes, bm, word_off, qidx, qoff, item_cnt, item_off, out, out_alt, res_q, res_k, tmp, ctr;
+    DevBuf vsig, qplanes, bm, word_off, qidx, qoff, item_cnt, item_off, out, out_alt, res_q, res_k, res_off, tmp, ctr;
     DevCounters *h_ctr = nullptr;  // pinned
     unsigned long long *h_nuniq = nullptr;
     unsigned long long cap_qidx = 0, cap_out = 0;

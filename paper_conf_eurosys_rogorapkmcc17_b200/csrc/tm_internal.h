@@ -87,6 +87,7 @@ int scan_variant_env();  // -1 = auto-tune
 cudaError_t launch_word_select(const uint64_t *planes, const uint64_t *tand, uint64_t rows, uint8_t *wsel,
                                cudaStream_t s);
 cudaError_t launch_split(const uint64_t *pairs, uint64_t n, uint32_t *q, uint32_t *k, cudaStream_t s);
+cudaError_t launch_query_offsets(const uint64_t *pairs, uint64_t n, uint64_t Q, uint64_t *q_off, cudaStream_t s);
 cudaError_t launch_gather_planes(const uint64_t *src0, const uint64_t *src1, const uint64_t *src2,
                                  const uint32_t *idx, uint64_t n, uint64_t *d0, uint64_t *d1, uint64_t *d2,
                                  cudaStream_t s);

@@ -986,6 +986,25 @@ __global__ void k_split(const uint64_t *__restrict__ pairs, uint64_t n, uint32_t
     k[i] = (uint32_t)v;
 }
 
+// q_off[j] = first index of query j in the sorted (q<<32 | key) pairs (lower bound), one thread
+// per query; q_off[Q] = n.
+__global__ void k_query_offsets(const uint64_t *__restrict__ pairs, uint64_t n, uint64_t Q,
+                                uint64_t *__restrict__ q_off) {
+    const uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (j > Q) return;
+    if (j == Q) {
+        q_off[Q] = n;
+        return;
+    }
+    const uint64_t key = j << 32;
+    uint64_t lo = 0, hi = n;
+    while (lo < hi) {
+        const uint64_t mid = (lo + hi) >> 1;
+        if (__ldg(pairs + mid) < key) lo = mid + 1; else hi = mid;
+    }
+    q_off[j] = lo;
+}
+
 // ---------------------------------------------------------------- build ---
 __global__ void k_gather_planes(const uint64_t *__restrict__ s0, const uint64_t *__restrict__ s1,
                                 const uint64_t *__restrict__ s2, const uint32_t *__restrict__ idx, uint64_t n,
@@ -1155,6 +1174,11 @@ cudaError_t launch_word_select(const uint64_t *planes, const uint64_t *tand, uin
     const uint64_t nt = rows / kTile;
     k_word_select<<<grid_for(rows, 256), 256, 0, s>>>(planes, planes + rows, planes + 2 * rows, tand, tand + nt,
                                                       tand + 2 * nt, rows, wsel);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_query_offsets(const uint64_t *pairs, uint64_t n, uint64_t Q, uint64_t *q_off, cudaStream_t s) {
+    k_query_offsets<<<grid_for(Q + 1, 256), 256, 0, s>>>(pairs, n, Q, q_off);
     return cudaGetLastError();
 }
 

@@ -46,6 +46,11 @@ class tm_pairs(ctypes.Structure):
                 ("key", ctypes.POINTER(ctypes.c_uint32)), ("priv_", ctypes.c_void_p)]
 
 
+class tm_csr(ctypes.Structure):
+    _fields_ = [("n_queries", ctypes.c_uint64), ("n", ctypes.c_uint64), ("q_off", ctypes.POINTER(ctypes.c_uint64)),
+                ("key", ctypes.POINTER(ctypes.c_uint32)), ("priv_", ctypes.c_void_p)]
+
+
 class tm_dev_pairs(ctypes.Structure):
     _fields_ = [("n", ctypes.c_uint64), ("query", ctypes.c_void_p), ("key", ctypes.c_void_p)]
 
@@ -78,7 +83,8 @@ class tm_stats_t(ctypes.Structure):
         return {n: getattr(self, n) for n, _ in self._fields_}
 
 
-EXPORTS = ["tm_build", "tm_match_batch", "tm_match_batch_device", "tm_pairs_free", "tm_free", "tm_strerror",
+EXPORTS = ["tm_build", "tm_match_batch", "tm_match_batch_csr", "tm_match_batch_device", "tm_pairs_free",
+           "tm_csr_free", "tm_free", "tm_strerror",
            "tm_last_error", "tm_abi_version", "tm_encode", "tm_stats", "tm_partitions", "tm_partition_sigs",
            "tm_owner_range", "tm_shard_plan", "tm_partition_host", "tm_last_result", "tm_shard_counts",
            "tm_shard_merge", "tm_nccl_unique_id", "tm_comm_init", "tm_match_batch_sharded_device",
@@ -105,6 +111,9 @@ def load(path: str = LIB_PATH):
     L.tm_match_batch_device.restype = ctypes.c_int
     L.tm_match_batch_device.argtypes = [vp, P(tm_tagsets), ctypes.c_int, P(tm_dev_pairs), vp]
     L.tm_pairs_free.argtypes = [P(tm_pairs)]
+    L.tm_match_batch_csr.restype = ctypes.c_int
+    L.tm_match_batch_csr.argtypes = [vp, P(tm_tagsets), ctypes.c_int, P(tm_csr)]
+    L.tm_csr_free.argtypes = [P(tm_csr)]
     L.tm_free.argtypes = [vp]
     L.tm_strerror.restype = ctypes.c_char_p
     L.tm_strerror.argtypes = [ctypes.c_int]
@@ -224,6 +233,29 @@ class Database:
         finally:
             L.tm_pairs_free(ctypes.byref(out))
         return qa, ka
+
+    def match_batch_csr(self, queries, unique: bool) -> tuple[np.ndarray, np.ndarray]:
+        """tm_match_batch_csr: host queries -> (q_off [Q+1] uint64, key [n] uint32) per-query key lists."""
+        L = load()
+        q = queries if isinstance(queries, HostTagSets) else HostTagSets.of(queries)
+        out = tm_csr()
+        _check(L.tm_match_batch_csr(self.h, ctypes.byref(q.c), int(bool(unique)), ctypes.byref(out)))
+        try:
+            off = np.ctypeslib.as_array(out.q_off, shape=(out.n_queries + 1,)).copy()
+            key = np.ctypeslib.as_array(out.key, shape=(out.n,)).copy() if out.n else np.zeros(0, np.uint32)
+        finally:
+            L.tm_csr_free(ctypes.byref(out))
+        return off, key
+
+    def match_batch_csr_raw(self, queries: HostTagSets, unique: bool) -> tm_csr:
+        """tm_match_batch_csr returning the library-owned pinned tm_csr (caller must free_csr)."""
+        out = tm_csr()
+        _check(load().tm_match_batch_csr(self.h, ctypes.byref(queries.c), int(bool(unique)), ctypes.byref(out)))
+        return out
+
+    @staticmethod
+    def free_csr(c: tm_csr):
+        load().tm_csr_free(ctypes.byref(c))
 
     def match_batch_raw(self, queries: HostTagSets, unique: bool) -> tm_pairs:
         """tm_match_batch returning the library-owned pinned tm_pairs (caller must free_pairs)."""

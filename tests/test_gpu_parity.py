@@ -379,6 +379,22 @@ def test_malformed_query_batch_is_rejected(c1):
             assert_pairs_equal(db.match_batch(c1.queries, False), want, f"after malformed {what}")
 
 
+@pytest.mark.parametrize("unique", [False, True])
+def test_csr_result_equals_pairs(c1, unique):
+    """tm_match_batch_csr returns the pairs of tm_match_batch as per-query key lists, also for
+    queries without matches and for an empty batch."""
+    extra = tagsets([[b"zz-none-1"], [], [b"zz-none-2", b"zz-none-3"]])
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=2000, tile_filter=1, row_order=1) as db:
+        for qs in (c1.queries, extra, c1.queries.subset(np.arange(0))):
+            q, k = db.match_batch(qs, unique)
+            off, key = db.match_batch_csr(qs, unique)
+            Q = qs.n_sets
+            assert off.size == Q + 1 and off[0] == 0 and off[-1] == key.size
+            assert np.all(np.diff(off.astype(np.int64)) >= 0)
+            assert np.array_equal(np.repeat(np.arange(Q, dtype=np.uint32), np.diff(off).astype(np.int64)), q)
+            assert np.array_equal(key, k)
+
+
 def test_device_entry_point_matches_host(c1):
     torch = pytest.importorskip("torch")
     with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=200_000) as db:
