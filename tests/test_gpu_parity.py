@@ -379,6 +379,31 @@ def test_malformed_query_batch_is_rejected(c1):
             assert_pairs_equal(db.match_batch(c1.queries, False), want, f"after malformed {what}")
 
 
+def test_variant_tuning_flag(c1, c2, c2_oracle, monkeypatch):
+    """tm_stats.tuning: 1 while the handle still times variants for this batch size (it then
+    cycles through them), 0 once it has settled; never set for forced variants or streaming calls."""
+    monkeypatch.delenv("TM_SCAN_VARIANT", raising=False)
+    want = c2_oracle[False]
+    with tmb.Database(c2.db, c2.key_off, c2.keys, max_partition=c2.max_partition, tile_filter=1,
+                      row_order=1) as db:
+        flags, variants = [], []
+        for _ in range(10):
+            assert_pairs_equal(db.match_batch(c2.queries, False), want, "during tuning")
+            st = db.stats()
+            flags.append(st["tuning"])
+            variants.append(st["scan_variant"])
+        assert flags[0] == 1 and 0 in flags, flags
+        settled = flags.index(0)
+        assert all(f == 0 for f in flags[settled:]) and len(set(variants[settled + 1:])) == 1, (flags, variants)
+        assert {5, 2, 0} <= set(variants[:settled + 1]), variants
+        db.match_batch(c2.queries.subset(np.arange(3)), False)    # streaming-only call
+        assert db.stats()["tuning"] == 0
+    monkeypatch.setenv("TM_SCAN_VARIANT", "5")
+    with tmb.Database(c1.db, c1.key_off, c1.keys, max_partition=2000, tile_filter=1, row_order=1) as db:
+        db.match_batch(c1.queries, False)
+        assert db.stats()["tuning"] == 0
+
+
 @pytest.mark.parametrize("unique", [False, True])
 def test_csr_result_equals_pairs(c1, unique):
     """tm_match_batch_csr returns the pairs of tm_match_batch as per-query key lists, also for
