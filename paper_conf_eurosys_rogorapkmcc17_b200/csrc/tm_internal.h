@@ -29,8 +29,8 @@ constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
 constexpr int kScanVariants = 8;    // k_scan variants (TM_SCAN_VARIANT)
-constexpr int kTune[] = {5, 2, 0};  // variants the handle times on its first calls (first = default)
-constexpr int kTuneN = 3;
+constexpr int kTune[] = {5, 0};  // variants the handle times on its first calls (first = default); 2 never won
+constexpr int kTuneN = 2;
 
 struct DevCounters {            // zeroed at the start of every match call
     unsigned long long n_out;   // (q,key) pairs emitted (may exceed capacity)
