@@ -368,7 +368,9 @@ def run_ours(args):
         achieved = ops / scan_s / 1e12
         traffic, ncu = None, None
         try:
-            with open(os.path.join(ROOT, "profiles", "ncu_scan_traffic.json")) as f:
+            per_cfg = os.path.join(ROOT, "profiles", f"ncu_scan_traffic_{args.config}.json")
+            with open(per_cfg if os.path.exists(per_cfg) else
+                      os.path.join(ROOT, "profiles", "ncu_scan_traffic.json")) as f:
                 tr = json.load(f)
                 if tr.get("config") == args.config:
                     traffic = tr.get("dram_bytes_per_launch")
