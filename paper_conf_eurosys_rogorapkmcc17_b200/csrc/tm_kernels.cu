@@ -707,6 +707,17 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     if (ok) sa[na + __popc(b & lt_mask)] = (uint16_t)i;
                     na += __popc(b);
                 }
+            } else if (f0 == 0 || f1 == 0 || f2 == 0) {
+                // two nonzero words: test those two only
+                const uint64_t *qa = f0 ? sm.q0 : sm.q1, *qb2 = f2 ? sm.q2 : sm.q1;
+                const uint64_t fa = f0 ? f0 : f1, fb = f2 ? f2 : f1;
+                for (uint32_t qb = qs; qb < qe; qb += 32) {
+                    const uint32_t i = qb + lane;
+                    const bool ok = i < qe && ((fa & ~qa[i]) | (fb & ~qb2[i])) == 0;
+                    const uint32_t b = __ballot_sync(0xffffffffu, ok);
+                    if (ok) sa[na + __popc(b & lt_mask)] = (uint16_t)i;
+                    na += __popc(b);
+                }
             } else {
                 for (uint32_t qb = qs; qb < qe; qb += 32) {
                     const uint32_t i = qb + lane;
