@@ -267,7 +267,9 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
             } else {
                 const int c = 63 - __builtin_clzll(Q);
                 db->call_class = c;
-                if (db->tune_calls[c] < 2 * kTuneN) {
+                // batches below kTuneMinQ queries keep the default variant: a tuning round there
+                // would put slow candidates into a latency-bound stream for little gain
+                if (Q >= (uint64_t)kTuneMinQ && db->tune_calls[c] < 2 * kTuneN) {
                     var = kTune[db->tune_calls[c] % kTuneN];
                     db->call_tunes = true;
                 } else {
@@ -711,6 +713,9 @@ tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32
     TMCK(cudaMallocHost((void **)&db->h_nuniq, 8));
     db->scan_grid = 0;
     build_impl(db, sets, key_off, keys);
+    // load every scan-kernel variant now (lazy module loading would otherwise put ~10-30 ms into
+    // the first call that picks a variant: a latency spike inside a stream, profiles/r1v46_stream_*)
+    for (int v = 0; v < kScanVariants; ++v) db->grid_of[v] = scan_grid(db->device, v);
     db->st.n_sets = db->n_sets;
     *out = db;
     db = nullptr;

@@ -31,6 +31,7 @@ constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 2
 constexpr int kScanVariants = 8;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {5, 0};  // variants the handle times on its first calls (first = default); 2 never won
 constexpr int kTuneN = 2;
+constexpr int kTuneMinQ = 4096;     // smaller calls are not tuned (default variant kTune[0])
 
 struct DevCounters {            // zeroed at the start of every match call
     unsigned long long n_out;   // (q,key) pairs emitted (may exceed capacity)

@@ -32,6 +32,8 @@ def main():
     q = wl.queries.subset(np.arange(nq))
     db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], tile_filter=1, row_order=1)
     db.match_batch(q, True)          # warm-up: grow every device / pinned buffer once
+    for b in (1, 8, 100, 1000, 3000, 10000):   # and load the kernels small batches use (CUB
+        db.match_batch(q.subset(np.arange(min(b, nq))), True)  # single-tile sorts; lazy loading)
     rng = np.random.default_rng(7)
     arrivals = np.cumsum(rng.exponential(1e9 / rate, nq)).astype(np.uint64)
     for to in timeouts:
