@@ -119,6 +119,11 @@ class ClockSampler:
 def load_workload(name: str, rank: int = 0):
     """BASELINE config `name`; rank r > 0 matches its own query batch (query seed + 7919 r)."""
     import tmgen
+    if name in tmgen.CRAFTED:  # sec. 4.4 crafted workloads (PAPER.md:391-399)
+        c = dict(tmgen.CRAFTED[name], max_partition=getattr(load_workload, "max_partition", 0) or 200_000, total_tags=0)
+        wl = tmgen.config(name, max_partition=c["max_partition"],
+                          query_seed=c["seed"] + (1 << 32) + 7919 * rank)
+        return wl, c
     c = dict(tmgen.CONFIGS[name])
     if getattr(load_workload, "max_partition", 0):
         c["max_partition"] = load_workload.max_partition
@@ -192,7 +197,9 @@ def run_reference(args):
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * tot / len(times),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
-            "data": "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)",
+            "data": ("synthetic (seeded sec. 4.4 crafted workload, tmgen.generate_crafted, PAPER.md:391-399)"
+                     if args.config.startswith(("C6", "C7")) else
+                     "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)"),
             "config": config_block(c, args, wl),
             "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
                              "sample": f"{size} of {q_sig.shape[0]} queries per step ("
@@ -205,7 +212,9 @@ def run_reference(args):
 
 def config_block(c, args, wl):
     return {"workload": args.config, "n_sets": c["n_sets"], "n_queries": c["n_queries"],
-            "query_tags": "base set + 2..4 extra" if not c["total_tags"] else f"total {c['total_tags']}",
+            "query_tags": (f"{c['set_tags']}-tag DB sets, {c['query_tags']}-tag queries (PAPER.md:391-399)"
+                           if "set_tags" in c else
+                           "base set + 2..4 extra" if not c["total_tags"] else f"total {c['total_tags']}"),
             "max_partition": c["max_partition"], "mode": "match-unique" if args.unique else "match",
             "tile_filter": ["alg4-prefix", "tile-and", "none"][args.tile_filter],
             "row_order": ["lexicographic", "balanced-splits"][args.row_order],
@@ -383,7 +392,9 @@ def run_ours(args):
             "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": statistics.mean(step_ms), "higher_is_better": True,
             "scaling": "strong" if sharded else "weak", "vs_baseline": None, "dtype": "u64",
-            "data": "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)",
+            "data": ("synthetic (seeded sec. 4.4 crafted workload, tmgen.generate_crafted, PAPER.md:391-399)"
+                     if args.config.startswith(("C6", "C7")) else
+                     "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)"),
             "config": config_block(c, args, wl),
             "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
                          "frac": achieved / peak_tops, "traffic": traffic,

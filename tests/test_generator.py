@@ -68,3 +68,23 @@ def test_c1_oracles_agree(c1):
         for mp in (0xFFFFFFFF, 200_000, 1000):
             qb, kb, _ = o2.Index(db, mp).match(c1.key_off, c1.keys, qs, unique)
             assert np.array_equal(qa, qb) and np.array_equal(ka, kb)
+
+
+def test_crafted_workload_shape():
+    """Sec. 4.4 crafted workload: sets of exactly s distinct tags, distinct
+    sets, queries of exactly t distinct tags that contain their base set; deterministic."""
+    for s, t in ((2, 10), (3, 6)):
+        w = tmgen.generate_crafted(20000, s, t, 500, seed=11)
+        assert np.all(np.diff(w.db.set_off) == s) and np.all(np.diff(w.queries.set_off) == t)
+        vb = w.db.vocab_bytes.tobytes()
+        dstr = [vb[w.db.vocab_off[i]:w.db.vocab_off[i + 1]] for i in range(w.db.vocab_off.size - 1)]
+        qb = w.queries.vocab_bytes.tobytes()
+        qstr = [qb[w.queries.vocab_off[i]:w.queries.vocab_off[i + 1]] for i in range(w.queries.vocab_off.size - 1)]
+        rows = [frozenset(dstr[x] for x in w.db.tag_idx[i * s:(i + 1) * s]) for i in range(w.db.n_sets)]
+        assert all(len(r) == s for r in rows) and len(set(rows)) == w.db.n_sets
+        for j in range(w.queries.n_sets):
+            q = frozenset(qstr[x] for x in w.queries.tag_idx[j * t:(j + 1) * t])
+            assert len(q) == t and rows[int(w.query_base[j])] <= q
+        assert np.array_equal(w.keys, np.arange(w.db.n_sets, dtype=np.uint32))
+        w2 = tmgen.generate_crafted(20000, s, t, 500, seed=11)
+        assert np.array_equal(w.db.tag_idx, w2.db.tag_idx) and np.array_equal(w.queries.tag_idx, w2.queries.tag_idx)

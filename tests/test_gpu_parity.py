@@ -564,3 +564,39 @@ def test_exact_mode_c2_sample(c2):
         gq, gk = db.match_batch(c2.queries, False)
     keep = np.isin(gq, qsel)
     assert list(zip(gq[keep].tolist(), gk[keep].tolist())) == want
+
+
+# ------------------------------------------ sec. 4.4 crafted workload (C6/C7 shapes) --
+@pytest.mark.parametrize("s,t", [(2, 10), (3, 6)])
+@pytest.mark.parametrize("unique", [False, True])
+def test_crafted_workload_parity(s, t, unique):
+    """The sec. 4.4 workload at a size the brute-force oracle finishes in
+    seconds: 300K sets of s tags, 4,000 queries of t tags; bit-exact vs O2 brute force; every
+    query returns its base set's key (keys = set index)."""
+    wl = tmgen.generate_crafted(300_000, s, t, 4000, seed=40 + s, max_partition=20_000)
+    want = oracle_pairs(wl, unique)
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition) as db:
+        got = db.match_batch(wl.queries, unique)
+    assert_pairs_equal(got, want, f"crafted s={s} t={t}")
+    pairs = set(zip(got[0].tolist(), got[1].tolist()))
+    assert all((j, int(b)) in pairs for j, b in enumerate(wl.query_base))
+
+
+@pytest.mark.parametrize("s,t", [(2, 10), (3, 6)])
+def test_crafted_workload_exact_mode(s, t):
+    """Exact mode on the crafted workload: string-level containment, checked on a 300-query
+    sample against the definition (the Bloom candidates of O2, then exact set containment)."""
+    wl = tmgen.generate_crafted(300_000, s, t, 2000, seed=50 + s)
+    rng = np.random.default_rng(6)
+    qsel = np.sort(rng.choice(wl.queries.n_sets, 300, replace=False))
+    db_sig, q_sig = o2.encode(wl.db), o2.encode(wl.queries)
+    want = []
+    for j in qsel:
+        qs = frozenset(wl.queries.strings(int(j)))
+        cand = np.nonzero(((db_sig[:, 0] & ~q_sig[j, 0]) | (db_sig[:, 1] & ~q_sig[j, 1]) |
+                           (db_sig[:, 2] & ~q_sig[j, 2])) == 0)[0]
+        want.extend((int(j), int(i)) for i in cand if frozenset(wl.db.strings(int(i))) <= qs)
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, exact=1) as db:
+        gq, gk = db.match_batch(wl.queries, False)
+    keep = np.isin(gq, qsel)
+    assert list(zip(gq[keep].tolist(), gk[keep].tolist())) == want

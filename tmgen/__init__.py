@@ -187,7 +187,72 @@ def generate(n_sets: int, n_queries: int, seed: int, extra: tuple[int, int] = (2
     return wl
 
 
+def _zipf_draw(rng: np.random.Generator, cdf: np.ndarray, shape) -> np.ndarray:
+    return np.searchsorted(cdf, rng.random(shape), side="right").astype(np.uint32)
+
+
+def generate_crafted(n_sets: int, set_tags: int, query_tags: int, n_queries: int, seed: int,
+                     vocab: int = 1 << 20, max_partition: int = 200_000, name: str = "crafted",
+                     query_seed: int | None = None) -> Workload:
+    """The scaled-down second workload of sec. 4.4: every DB set has exactly
+    `set_tags` distinct tags (2 or 3), every query has exactly `query_tags` tags (6-10) = one DB
+    set (its base) plus query_tags - set_tags extra tags.  Tags are drawn from
+    a Zipf(1) vocabulary of `vocab` ids (the popularity law of the Twitter workload,
+    PAPER.md:264); DB sets are distinct; one key per set (key = set index).  numpy PCG64, seeded."""
+    assert 1 <= set_tags <= query_tags and vocab <= (1 << 20)
+    rng = np.random.Generator(np.random.PCG64(seed))
+    w = 1.0 / np.arange(1, vocab + 1, dtype=np.float64)
+    cdf = np.cumsum(w) / w.sum()
+    cdf[-1] = 1.0
+    assert set_tags <= 3, "sets are deduplicated as one packed u64 (3 x 20-bit ids)"
+    packed = np.zeros(0, np.uint64)
+    while packed.size < n_sets:
+        d = np.sort(_zipf_draw(rng, cdf, (int((n_sets - packed.size) * 1.3) + 64, set_tags)), axis=1)
+        d = d[np.all(d[:, 1:] != d[:, :-1], axis=1)].astype(np.uint64)
+        p = np.zeros(d.shape[0], np.uint64)
+        for c in range(set_tags):
+            p = (p << np.uint64(20)) | d[:, c]
+        packed = np.sort(np.concatenate([packed, p]))
+        packed = packed[np.concatenate(([True], packed[1:] != packed[:-1]))]
+    packed = packed[rng.permutation(packed.size)[:n_sets]]
+    rows = np.zeros((n_sets, set_tags), np.uint32)
+    for c in range(set_tags - 1, -1, -1):
+        rows[:, c] = (packed & np.uint64(0xFFFFF)).astype(np.uint32)
+        packed = packed >> np.uint64(20)
+    set_off = np.arange(n_sets + 1, dtype=np.uint64) * np.uint64(set_tags)
+    key_off = np.arange(n_sets + 1, dtype=np.uint64)
+    keys = np.arange(n_sets, dtype=np.uint32)
+    rng = np.random.Generator(np.random.PCG64(seed + (1 << 32) if query_seed is None else query_seed))
+    base = rng.integers(0, n_sets, n_queries).astype(np.uint64)
+    e = query_tags - set_tags
+    q = np.zeros((n_queries, query_tags), np.uint32)
+    q[:, :set_tags] = rows[base]
+    todo = np.arange(n_queries)
+    while todo.size and e:
+        q[todo, set_tags:] = _zipf_draw(rng, cdf, (todo.size, e))
+        s = np.sort(q[todo], axis=1)
+        todo = todo[np.any(s[:, 1:] == s[:, :-1], axis=1)]
+    q_off = np.arange(n_queries + 1, dtype=np.uint64) * np.uint64(query_tags)
+    return Workload(name, intern(set_off, rows.reshape(-1)), key_off, keys, intern(q_off, q.reshape(-1)),
+                    base, max_partition)
+
+
+# sec. 4.4 crafted workloads (PAPER.md:391-399): C6 = the paper's hardest case, 2-tag sets and
+# 10-tag queries over the largest DB of Fig. 10 (5M sets; "more than 32,000 queries per second",
+# PAPER.md:395); C7 = the Fig. 11 workload, 3M sets of 3 tags, 6-tag queries (PAPER.md:399).
+CRAFTED = {
+    "C6": dict(n_sets=5_000_000, set_tags=2, query_tags=10, n_queries=100_000, seed=6),
+    "C7": dict(n_sets=3_000_000, set_tags=3, query_tags=6, n_queries=100_000, seed=7),
+}
+
+
 def config(name: str, **overrides) -> Workload:
+    if name in CRAFTED:
+        c = dict(CRAFTED[name])
+        c.update(overrides)
+        return generate_crafted(c["n_sets"], c["set_tags"], c["query_tags"], c["n_queries"], c["seed"],
+                                max_partition=c.get("max_partition", 200_000), name=name,
+                                query_seed=c.get("query_seed"))
     c = dict(CONFIGS[name])
     c.update(overrides)
     return generate(c["n_sets"], c["n_queries"], c["seed"], total_tags=c["total_tags"],
