@@ -61,3 +61,28 @@ def test_full_size_sampled_parity(full, unique):
     print(f"oracle sample: {time.time() - t:.1f} s")
     keep = np.isin(gq, qsel)
     assert np.array_equal(gq[keep], wq) and np.array_equal(gk[keep], wk)
+
+
+@pytest.mark.parametrize("name", ["C6", "C7"])
+def test_crafted_full_size_sampled_parity(name):
+    """The sec. 4.4 crafted workloads at full size (C6: 5M 2-tag sets x 100k 10-tag queries;
+    C7: 3M x 3 tags x 100k 6-tag queries) in the layout bench.py times:
+    whole-output properties, then bit-exact parity on a 192-query sample against O2 brute force
+    over the whole database, for match and match-unique."""
+    wl = tmgen.config(name)
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=1,
+                      row_order=1) as db:
+        db_sig = o2.encode(wl.db)
+        for unique in (False, True):
+            gq, gk = db.match_batch(wl.queries, unique)
+            key = (gq.astype(np.uint64) << np.uint64(32)) | gk.astype(np.uint64)
+            assert np.all(key[1:] > key[:-1]) if unique else np.all(key[1:] >= key[:-1])
+            # every query returns its base set's key (key = set index)
+            base_key = (np.arange(wl.queries.n_sets, dtype=np.uint64) << np.uint64(32)) | wl.query_base
+            assert np.all(np.isin(base_key, key))
+            rng = np.random.default_rng(77 + unique)
+            qsel = np.sort(rng.choice(wl.queries.n_sets, 192, replace=False))
+            qs = o2.encode(wl.queries.subset(qsel))
+            wq, wk = o2.match_brute(db_sig, wl.key_off, wl.keys, qs, unique, qid=qsel.astype(np.uint32))
+            keep = np.isin(gq, qsel)
+            assert np.array_equal(gq[keep], wq) and np.array_equal(gk[keep], wk)
