@@ -224,6 +224,22 @@ def config_block(c, args, wl):
             "l2": "flushed between timed steps (512 MiB write)", "bloom": "192 bits, k=7 (PAPER.md:106)"}
 
 
+def memory_block(db, mem0, mem1, dev):
+    """Fig. 9 analogue: device memory the library holds, from
+    cudaMemGetInfo deltas minus torch's own reservations (the library allocates with
+    cudaMallocAsync, so pool memory it keeps counts): after tm_build (the database: tagset
+    table, masks, key CSR) and after the timed calls (plus the per-call work buffers)."""
+    import torch
+    torch.cuda.synchronize(dev)
+    free2, res2 = torch.cuda.mem_get_info(dev)[0], torch.cuda.memory_reserved(dev)
+    st = db.stats()
+    lib_db = (mem0[0] - mem1[0]) - (mem1[1] - mem0[1])
+    lib_all = (mem0[0] - free2) - (res2 - mem0[1])
+    return {"device_db_bytes": int(lib_db), "device_after_calls_bytes": int(lib_all),
+            "tagset_table_bytes": int(st["n_rows"]) * 24, "key_table_bytes": int(st["n_entries"]) * 4,
+            "note": "the key table lives on the GPU (the paper keeps it on the host, P:387)"}
+
+
 # --------------------------------------------------------------------- ours --
 def run_ours(args):
     import torch
@@ -256,11 +272,15 @@ def run_ours(args):
     wl, c = load_workload(args.config, 0 if sharded else rank)
     unique = bool(args.unique)
     Q = wl.queries.n_sets
+    torch.cuda.synchronize(dev)
+    mem0 = (torch.cuda.mem_get_info(dev)[0], torch.cuda.memory_reserved(dev))
     t0 = time.perf_counter()
     db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], device=dev,
                       tile_filter=args.tile_filter, row_order=args.row_order, exact=int(args.exact),
                       n_shards=world if sharded else 1, shard=rank if sharded else 0)
     build_s = time.perf_counter() - t0
+    torch.cuda.synchronize(dev)
+    mem1 = (torch.cuda.mem_get_info(dev)[0], torch.cuda.memory_reserved(dev))
     if sharded:
         from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as tmx
         uid = [tmx.nccl_unique_id() if rank == 0 else None]
@@ -421,6 +441,7 @@ def run_ours(args):
                                                 "pair_checks", "matched_sets", "emitted_pairs", "result_pairs",
                                                 "work_items", "exact_checked", "exact_kept")},
             "build_s": build_s,
+            "memory": memory_block(db, mem0, mem1, dev),
             "tuning_calls": tune_calls,   # untimed calls that finished the variant tuning before the W warm-ups
         }
         if not args.no_cpu_baseline and world == 1:
