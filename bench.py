@@ -3,22 +3,28 @@
 
 A step = one tm_match_batch over one batch of queries = the whole hot path
 (encode, route, batch, pre-filter, subset scan, compaction,
-key expansion, sort/merge).  Default workload: BASELINE config C2 (1M tag
-sets, 100k-query stream, MAX_P = 200K), `match` (Table 1).
+key expansion, sort/merge).  Default workload: N = 1 -> BASELINE config C3
+(100M tag sets, 1M-query stream, MAX_P = 200K: the largest single-GPU config);
+N > 1 -> C4 (300M tag sets) partition-sharded over the N ranks; `match`
+(Table 1).
 
-  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C2] [--unique]
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--config C3] [--unique]
 
 value  : queries/s over all ranks, inputs resident in HBM (tm_match_batch_device),
          per-step CUDA events on the launching stream, L2 flushed between steps.
 e2e    : queries/s through tm_match_batch_csr with pinned host queries (H2D inside
          the timed region) and the result -- every query's sorted keys -- copied
          back to host (D2H: 4 B per pair + 8 B per query offset).
-N > 1  : one process per GPU (torchrun); every rank holds a replica of the
-         database and matches its own query batch (replicated mode, PAPER.md:110,
-         228: no data-path collective) -> "scaling": "weak"; time = max over ranks.
-         --shard: the database is partition-sharded over the ranks, every
-         rank matches the same batch against its partitions and the pairs go to
-         query owners over NCCL (tm_match_batch_sharded_device) -> "strong".
+hbm    : (N = 1) the subset scan of the whole table as ONE partition, pre-filter off,
+         B = 1 / 4 / 16 queries: table bytes / scan-kernel time vs the measured HBM
+         copy bandwidth (the BASELINE metric's "subset-scan HBM GB/s vs roofline").
+roofline: the dominant kernel (k_scan) against the INT/logic-pipe peak measured on
+         this box by build/int_peak (scripts/int_peak.cu), SURVEY 8(d) ops model.
+N > 1  : one process per GPU (torchrun).  Default: the database is partition-sharded
+         over the ranks: every rank matches the same batch against
+         its partitions and the pairs go to query owners over NCCL
+         (tm_match_batch_sharded_device) -> "scaling": "strong".  --replicated: every
+         rank holds the whole database and matches its own batch -> "weak".
 --impl reference : the oracle (oracle/o2.c, the paper's CPU method) on the
          host cores, on a bounded sample of the same workload per step.
 """
@@ -38,15 +44,14 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "queries/sec vs DB size at 1/2/4/8 B200; subset-scan HBM GB/s vs roofline"
-ALU_LANES_PER_SM_CLK = 64     # LOP3/IADD3 ALU pipe: 16 lanes/clk/SMSP x 4 SMSP (B300_MICROARCH.md)
+ALU_LANES_PER_SM_CLK = 64     # fallback only: LOP3 ALU pipe 16 lanes/clk/SMSP x 4 (B300_MICROARCH.md)
 SM_COUNT = 148
-# algorithmic INT ops per decision: every pre-filter test
-# (mask vs query) and every pair check (set vs query) needs at least one 64-bit
-# block test = and-not of both 32-bit halves + zero test = 3 ALU ops.
-OPS_PER_TILE_TEST = 3
-OPS_PER_PAIR_CHECK = 3
-SURVEY_OPS_PER_TILE_TEST = 4    # SURVEY.md 8(d) per-unit figures (plain Alg. 4 / Alg. 3)
+# SURVEY.md 8(d) per-unit figures (the primary roofline model): a pre-filter test (mask vs
+# query, Alg. 4) = 4 INT ops, a pair check (set vs query, Alg. 3: 6 LOP3 + 1 ISETP) = 7
+SURVEY_OPS_PER_TILE_TEST = 4
 SURVEY_OPS_PER_PAIR_CHECK = 7
+# secondary model: the minimum one 64-bit block test per decision = 3 ops
+MIN_OPS_PER_DECISION = 3
 
 
 class _CAI:
@@ -200,7 +205,7 @@ def run_reference(args):
             "data": ("synthetic (seeded sec. 4.4 crafted workload, tmgen.generate_crafted, PAPER.md:391-399)"
                      if args.config.startswith(("C6", "C7")) else
                      "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)"),
-            "config": config_block(c, args, wl),
+            "config": config_block(c, args, wl, args.gpus > 1 and not args.replicated),
             "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
                              "sample": f"{size} of {q_sig.shape[0]} queries per step ("
                                        + (f"O2 brute force over {c['n_sets']} sets" if isinstance(ix, _BruteOracle)
@@ -210,7 +215,7 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
-def config_block(c, args, wl):
+def config_block(c, args, wl, sharded=False):
     return {"workload": args.config, "n_sets": c["n_sets"], "n_queries": c["n_queries"],
             "query_tags": (f"{c['set_tags']}-tag DB sets, {c['query_tags']}-tag queries (PAPER.md:391-399)"
                            if "set_tags" in c else
@@ -219,7 +224,7 @@ def config_block(c, args, wl):
             "tile_filter": ["alg4-prefix", "tile-and", "none"][args.tile_filter],
             "row_order": ["lexicographic", "balanced-splits"][args.row_order],
             "exact_check": bool(args.exact),
-            "parallelism": (f"partition-sharded-{args.gpus} (NCCL exchange)" if args.shard else
+            "parallelism": (f"partition-sharded-{args.gpus} (NCCL exchange)" if sharded else
                             f"replicated-dp{args.gpus}") if args.gpus > 1 else "single",
             "l2": "flushed between timed steps (512 MiB write)", "bloom": "192 bits, k=7 (PAPER.md:106)"}
 
@@ -241,6 +246,101 @@ def memory_block(db, mem0, mem1, dev):
 
 
 # --------------------------------------------------------------------- ours --
+def int_peak(peaks):
+    """INT/logic-pipe peak of this GPU: scripts/int_peak.cu (built by build() as build/int_peak)
+    run now on this GPU (LOP3 thread-ops per SM per clock, x SMs x the max SM clock); else the
+    committed measurement profiles/int_peak.json; else the guide's 64 lanes/clk/SM."""
+    import subprocess
+    mhz = peaks.get("sm_max_mhz", 1965.0)
+    res, src = None, None
+    exe = os.path.join(ROOT, "build", "int_peak")
+    if os.path.exists(exe):
+        try:
+            out = subprocess.run([exe], capture_output=True, text=True, timeout=60).stdout.strip().splitlines()
+            res, src = json.loads(out[-1]), "measured now (build/int_peak)"
+        except Exception:
+            res = None
+    if res is None:
+        try:
+            with open(os.path.join(ROOT, "profiles", "int_peak.json")) as f:
+                res, src = json.load(f), "measured earlier (profiles/int_peak.json)"
+        except Exception:
+            res = None
+    if res is None:
+        return SM_COUNT * ALU_LANES_PER_SM_CLK * mhz * 1e6 / 1e12, \
+            f"fallback: {SM_COUNT} SMs x {ALU_LANES_PER_SM_CLK} lanes/clk (B300_MICROARCH.md) x {mhz} MHz", None
+    per_clk = res["lop3"]["ops_per_clk_per_sm"]
+    return res["sms"] * per_clk * mhz * 1e6 / 1e12, \
+        (f"{src}: LOP3 {per_clk:.1f} thread-ops/clk/SM x {res['sms']} SMs x {mhz} MHz (MEASURED_PEAKS.json "
+         f"sm_max_mhz); measured {res['lop3']['tops']:.2f} Tops/s at ~{res['lop3']['sm_mhz_est']:.0f} MHz"), res
+
+
+def ncu_traffic(config: str, variant: int, build_id: str):
+    """DRAM traffic of k_scan from the committed ncu capture of this config, only if it was
+    taken on the same library build (tm_build_id) and scan variant; else None + why."""
+    path = os.path.join(ROOT, "profiles", f"ncu_scan_traffic_{config}.json")
+    try:
+        with open(path) as f:
+            tr = json.load(f)
+    except Exception:
+        return None, None, f"no committed ncu capture for {config}"
+    if tr.get("build_id") != build_id or tr.get("variant") != variant:
+        return None, None, (f"committed capture {os.path.basename(path)} is from build {tr.get('build_id')} "
+                            f"variant {tr.get('variant')}, this run is build {build_id} variant {variant}")
+    ncu = {k: tr.get(k) for k in ("alu_pipe_pct", "issue_active_pct", "warps_active_pct", "l2_hit_pct")}
+    ncu["report"] = tr.get("report")
+    return tr.get("dram_bytes_per_launch"), ncu, "same build and variant"
+
+
+def hbm_block(wl, dev, stream, flush, Bs=(1, 4, 16)):
+    """The subset scan of the whole table as ONE partition (no partitioning), pre-filter off:
+    every stored signature read from HBM once per call (24 B/set) and checked against B queries
+    (SURVEY 8(d) roofline sweep; the table is larger than L2)."""
+    import torch
+    import paper_conf_eurosys_rogorapkmcc17_b200 as tmb
+    peaks, src = measured_peaks()
+    hbm = float(peaks["hbm_gbs"])
+    t0 = time.perf_counter()
+    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=tmb.TM_NO_PARTITIONING, device=dev,
+                      tile_filter=2, row_order=0)
+    build_s = time.perf_counter() - t0
+    rows = db.stats()["n_rows"]
+    pts = []
+    for B in Bs:
+        q = wl.queries.subset(np.arange(B))
+        arrs = [np.ascontiguousarray(a) for a in (q.vocab_bytes, q.vocab_off.view(np.int64),
+                                                  q.tag_idx.view(np.int32), q.set_off.view(np.int64))]
+        dt = [torch.from_numpy(a).to(f"cuda:{dev}") for a in arrs]
+        dq = tmb.device_tagsets(dt[0].data_ptr(), dt[1].data_ptr(), dt[2].data_ptr(), dt[3].data_ptr(),
+                                arrs[0].size, arrs[1].size - 1, arrs[2].size, B)
+        for _ in range(16):
+            db.match_batch_device(dq, False, stream.cuda_stream)
+            if not db.stats()["tuning"]:
+                break
+        for _ in range(3):
+            db.match_batch_device(dq, False, stream.cuda_stream)
+        scan = []
+        for _ in range(7):
+            flush.zero_()
+            db.match_batch_device(dq, False, stream.cuda_stream)
+            scan.append(db.stats()["scan_ms"])
+        st = db.stats()
+        ms = statistics.median(scan)
+        gbs = 24 * rows / (ms / 1e3) / 1e9
+        pts.append({"B": B, "scan_ms": ms, "GB/s": gbs, "frac": gbs / hbm, "variant": st["scan_variant"],
+                    "pair_checks_per_s": st["pair_checks"] / (ms / 1e3)})
+    db.close()
+    return {"table": f"whole {args_config_name(wl)} table as one partition, {rows} rows x 24 B = "
+                     f"{24 * rows / 1e9:.2f} GB (> 126 MB L2), pre-filter off",
+            "peak_gbs": hbm, "peak_src": f"{src} MEASURED_PEAKS.json hbm_gbs (read+write copy)",
+            "timing": "median of 7 calls, CUDA events around the k_scan launch on the library stream, "
+                      "L2 flushed before each", "points": pts, "build_s": build_s}
+
+
+def args_config_name(wl):
+    return getattr(wl, "name", "")
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -254,24 +354,38 @@ def run_ours(args):
     if world > 1:
         torch.cuda.set_device(local % torch.cuda.device_count())
         if pg == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local % torch.cuda.device_count()))
         else:
             dist.init_process_group(pg)
     else:
         torch.cuda.set_device(0)
     dev = torch.cuda.current_device()
+    cdev = f"cuda:{dev}" if pg == "nccl" else "cpu"
 
     import __graft_entry__
     __graft_entry__.build() if rank == 0 or world == 1 else None
     if world > 1:
         dist.barrier()
     import paper_conf_eurosys_rogorapkmcc17_b200 as tmb
+    from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as tmx
 
-    sharded = args.shard and world > 1
+    sharded = world > 1 and not args.replicated
     # replicated mode: every rank its own batch; sharded mode: the same batch on every rank
     wl, c = load_workload(args.config, 0 if sharded else rank)
     unique = bool(args.unique)
     Q = wl.queries.n_sets
+    peaks, peak_src = measured_peaks()
+    ipeak, ipeak_src, ipeak_raw = int_peak(peaks) if rank == 0 else (None, None, None)
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=f"cuda:{dev}")
+
+    # the scaling base of a sharded run: the same workload on ONE GPU (rank 0), same steps
+    base = None
+    if sharded and rank == 0 and not args.no_scaling_base:
+        base = single_gpu_value(wl, c, args, dev, stream, flush)
+    if world > 1:
+        dist.barrier()
+
     torch.cuda.synchronize(dev)
     mem0 = (torch.cuda.mem_get_info(dev)[0], torch.cuda.memory_reserved(dev))
     t0 = time.perf_counter()
@@ -282,7 +396,6 @@ def run_ours(args):
     torch.cuda.synchronize(dev)
     mem1 = (torch.cuda.mem_get_info(dev)[0], torch.cuda.memory_reserved(dev))
     if sharded:
-        from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as tmx
         uid = [tmx.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
         db.comm_init(uid[0], world, rank)
@@ -297,8 +410,6 @@ def run_ours(args):
     hq = tmb.HostTagSets(pinned[0].numpy(), pinned[1].numpy().view(np.uint64), pinned[2].numpy().view(np.uint32),
                          pinned[3].numpy().view(np.uint64))
     h2d_bytes = sum(a.nbytes for a in qarr)
-    flush = torch.empty(512 << 20, dtype=torch.uint8, device=f"cuda:{dev}")
-    stream = torch.cuda.current_stream()
 
     def step_device():
         if sharded:
@@ -323,19 +434,7 @@ def run_ours(args):
             host[out.n:].copy_(kt)
         return out.n * 8
 
-    # the handle times its scan-kernel variants on its first calls of a batch size (DESIGN.md
-    # sec. 6): finish that before the W warm-up steps, so that no timed step runs a candidate
-    tune_calls = 0
-    for _ in range(16):
-        step_device()
-        tune_calls += 1
-        done = 0 if db.stats()["tuning"] else 1
-        if world > 1:   # the ranks agree (the sharded step has collectives inside)
-            t = torch.tensor([done], device=f"cuda:{dev}" if pg == "nccl" else "cpu", dtype=torch.int32)
-            dist.all_reduce(t, op=dist.ReduceOp.MIN)
-            done = int(t.item())
-        if done:
-            break
+    tune_calls = finish_tuning(db, step_device, world, cdev)
     for _ in range(args.warmup):
         step_device()
         step_e2e()
@@ -343,7 +442,7 @@ def run_ours(args):
 
     # ---- value: device-resident inputs, per-step CUDA events, L2 flushed between steps
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    launches, scan_ms, stats = 0, [], []
+    launches, stats = 0, []
     sampler = ClockSampler(dev)
     if world > 1:
         dist.barrier()
@@ -352,11 +451,10 @@ def run_ours(args):
         for i in range(args.steps):
             flush.zero_()
             ev[i][0].record(stream)
-            out = step_device()
+            step_device()
             ev[i][1].record(stream)
             st = db.stats()
             launches += st["kernel_launches"]
-            scan_ms.append(st["scan_ms"])
             stats.append(st)
         torch.cuda.synchronize()
     if world > 1:
@@ -365,10 +463,30 @@ def run_ours(args):
     t_local = sum(step_ms) / 1000.0
     t_max = t_local
     if world > 1:
-        t = torch.tensor([t_local], device=f"cuda:{dev}" if pg == "nccl" else "cpu", dtype=torch.float64)
+        t = torch.tensor([t_local], device=cdev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         t_max = float(t.item())
     value = (1 if sharded else world) * Q * args.steps / t_max
+    scan_ms = [s["scan_ms"] for s in stats]
+
+    # per-rank view (sharded: scan time, exchange, imbalance)
+    ranks = None
+    if world > 1:
+        mine = torch.tensor([statistics.mean(scan_ms), t_local * 1000 / args.steps,
+                             statistics.mean(s["xchg_ms"] for s in stats),
+                             statistics.mean(s["local_ms"] for s in stats),
+                             float(stats[-1]["xchg_send_bytes"]), float(stats[-1]["xchg_recv_bytes"]),
+                             float(stats[-1]["pair_checks"]), float(stats[-1]["n_rows"])],
+                            device=cdev, dtype=torch.float64)
+        allr = [torch.zeros_like(mine) for _ in range(world)]
+        dist.all_gather(allr, mine)
+        allr = [r.cpu().tolist() for r in allr]
+        sc = [r[0] for r in allr]
+        ranks = {"scan_ms": sc, "step_ms": [r[1] for r in allr], "xchg_ms": [r[2] for r in allr],
+                 "local_ms": [r[3] for r in allr], "xchg_send_bytes": [int(r[4]) for r in allr],
+                 "xchg_recv_bytes": [int(r[5]) for r in allr], "pair_checks": [int(r[6]) for r in allr],
+                 "rows": [int(r[7]) for r in allr],
+                 "scan_imbalance_max_over_mean": max(sc) / max(statistics.mean(sc), 1e-9)}
 
     # ---- e2e: host API, pinned inputs, H2D + D2H inside the timed region
     e2e_t, d2h = [], 0
@@ -383,31 +501,24 @@ def run_ours(args):
         e2e_t.append(time.perf_counter() - t0)
     e2e_local = sum(e2e_t)
     if world > 1:
-        t = torch.tensor([e2e_local], device=f"cuda:{dev}" if pg == "nccl" else "cpu", dtype=torch.float64)
+        t = torch.tensor([e2e_local], device=cdev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_local = float(t.item())
     e2e_value = (1 if sharded else world) * Q * args.steps / e2e_local
 
+    mem = memory_block(db, mem0, mem1, dev)
+    db.close()
+    hbm = None
+    if world == 1 and not args.no_hbm:
+        hbm = hbm_block(wl, dev, stream, flush)
+
     if rank == 0:
-        peaks, peak_src = measured_peaks()
         last = stats[-1]
-        ops = OPS_PER_TILE_TEST * last["tile_tests"] + OPS_PER_PAIR_CHECK * last["pair_checks"]
         scan_s = statistics.mean(scan_ms) / 1000.0
-        peak_tops = SM_COUNT * ALU_LANES_PER_SM_CLK * peaks.get("sm_max_mhz", 1965.0) * 1e6 / 1e12
+        ops = SURVEY_OPS_PER_TILE_TEST * last["tile_tests"] + SURVEY_OPS_PER_PAIR_CHECK * last["pair_checks"]
+        ops_min = MIN_OPS_PER_DECISION * (last["tile_tests"] + last["pair_checks"])
         achieved = ops / scan_s / 1e12
-        traffic, ncu = None, None
-        try:
-            per_cfg = os.path.join(ROOT, "profiles", f"ncu_scan_traffic_{args.config}.json")
-            with open(per_cfg if os.path.exists(per_cfg) else
-                      os.path.join(ROOT, "profiles", "ncu_scan_traffic.json")) as f:
-                tr = json.load(f)
-                if tr.get("config") == args.config:
-                    traffic = tr.get("dram_bytes_per_launch")
-                    ncu = {k: tr.get(k) for k in ("alu_pipe_pct", "issue_active_pct", "warps_active_pct",
-                                                  "l2_hit_pct")}
-                    ncu["report"] = tr.get("report")
-        except Exception:
-            pass
+        traffic, ncu, traffic_note = ncu_traffic(args.config, last["scan_variant"], tmx.build_id())
         line = {
             "metric": METRIC, "value": value, "unit": "queries/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": statistics.mean(step_ms), "higher_is_better": True,
@@ -415,22 +526,18 @@ def run_ours(args):
             "data": ("synthetic (seeded sec. 4.4 crafted workload, tmgen.generate_crafted, PAPER.md:391-399)"
                      if args.config.startswith(("C6", "C7")) else
                      "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)"),
-            "config": config_block(c, args, wl),
-            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak_tops, "unit": "Tops/s",
-                         "frac": achieved / peak_tops, "traffic": traffic,
+            "config": config_block(c, args, wl, sharded),
+            "roofline": {"bound": "alu", "achieved": achieved, "peak": ipeak, "unit": "Tops/s",
+                         "frac": achieved / ipeak, "traffic": traffic, "traffic_note": traffic_note,
                          "kernel": f"k_scan (variant {last['scan_variant']})", "kernel_ms": statistics.mean(scan_ms),
                          "kernel_share_of_step": statistics.mean(scan_ms) / statistics.mean(step_ms),
                          "ops_per_launch": ops,
-                         "ops_model": "3 ALU ops per decision (pre-filter test or pair check): the minimum "
-                                      "one 64-bit block test; DESIGN.md sec. 6",
-                         "frac_survey_model": (SURVEY_OPS_PER_TILE_TEST * last["tile_tests"] +
-                                               SURVEY_OPS_PER_PAIR_CHECK * last["pair_checks"]) / scan_s / 1e12
-                                              / peak_tops,
-                         "survey_model": "SURVEY.md 8(d): 4 ops per tile test + 7 per pair check (the full "
-                                         "three-block check); informational, frac above is the primary",
-                         "ncu_same_kernel": ncu,
-                         "peak_src": f"{SM_COUNT} SMs x {ALU_LANES_PER_SM_CLK} ALU lanes/clk x "
-                                     f"{peaks.get('sm_max_mhz', 1965.0)} MHz ({peak_src} sm_max_mhz)"},
+                         "ops_model": "SURVEY.md 8(d): 4 INT ops per pre-filter test (tm_stats.tile_tests) + 7 per "
+                                      "pair check (6 LOP3 + 1 ISETP, tm_stats.pair_checks), counted by the kernel",
+                         "frac_min_ops_model": ops_min / scan_s / 1e12 / ipeak,
+                         "min_ops_model": "3 ops per decision (one 64-bit block test: the minimum); DESIGN.md sec. 6",
+                         "ncu_same_kernel": ncu, "peak_src": ipeak_src,
+                         "build_id": tmx.build_id()},
             "e2e": {"value": e2e_value, "unit": "queries/s", "h2d_bytes_per_step": h2d_bytes,
                     "d2h_bytes_per_step": d2h},
             "gpu_launches": launches,
@@ -441,9 +548,19 @@ def run_ours(args):
                                                 "pair_checks", "matched_sets", "emitted_pairs", "result_pairs",
                                                 "work_items", "exact_checked", "exact_kept")},
             "build_s": build_s,
-            "memory": memory_block(db, mem0, mem1, dev),
+            "memory": mem,
             "tuning_calls": tune_calls,   # untimed calls that finished the variant tuning before the W warm-ups
         }
+        if ipeak_raw:
+            line["roofline"]["int_peak_microbench"] = {k: ipeak_raw[k] for k in
+                                                      ("lop3", "lop3_imad", "precheck_alu", "precheck_imad")
+                                                      if k in ipeak_raw}
+        if hbm:
+            line["hbm"] = hbm
+        if ranks:
+            line["ranks"] = ranks
+        if base:
+            line["scaling_base_1gpu"] = base
         if not args.no_cpu_baseline and world == 1:
             from oracle import o2
             ix, q_sig, size, obuild = oracle_rate(wl, c, unique, target_s=args.cpu_s)
@@ -459,10 +576,64 @@ def run_ours(args):
                                                f"O2: Alg.1 MAX_P={c['max_partition']} + Alg.2 + linear scan, "
                                                f"{o2.threads(0)} threads; Alg.1 build {obuild:.1f} s excluded") + ")"}
         print(json.dumps(line), flush=True)
-    db.close()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
+
+
+def finish_tuning(db, step, world, cdev):
+    """The handle times its scan-kernel variants on its first calls of a batch size (DESIGN.md
+    sec. 6): finish that before the warm-up steps, so that no timed step runs a candidate."""
+    import torch
+    import torch.distributed as dist
+    calls = 0
+    for _ in range(16):
+        step()
+        calls += 1
+        done = 0 if db.stats()["tuning"] else 1
+        if world > 1:   # the ranks agree (the sharded step has collectives inside)
+            t = torch.tensor([done], device=cdev, dtype=torch.int32)
+            dist.all_reduce(t, op=dist.ReduceOp.MIN)
+            done = int(t.item())
+        if done:
+            break
+    return calls
+
+
+def single_gpu_value(wl, c, args, dev, stream, flush):
+    """Scaling base of a sharded N-GPU line: the whole database on rank 0's GPU, the same batch,
+    tuning + W warm-ups + K timed steps as the sharded run (device-resident inputs)."""
+    import torch
+    import paper_conf_eurosys_rogorapkmcc17_b200 as tmb
+    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], device=dev,
+                      tile_filter=args.tile_filter, row_order=args.row_order, exact=int(args.exact))
+    q = wl.queries
+    arrs = [np.ascontiguousarray(a) for a in (q.vocab_bytes, q.vocab_off.view(np.int64),
+                                              q.tag_idx.view(np.int32), q.set_off.view(np.int64))]
+    dt = [torch.from_numpy(a).to(f"cuda:{dev}") for a in arrs]
+    dq = tmb.device_tagsets(dt[0].data_ptr(), dt[1].data_ptr(), dt[2].data_ptr(), dt[3].data_ptr(),
+                            arrs[0].size, arrs[1].size - 1, arrs[2].size, q.n_sets)
+
+    def step():
+        return db.match_batch_device(dq, bool(args.unique), stream.cuda_stream)
+
+    finish_tuning(db, step, 1, None)
+    for _ in range(args.warmup):
+        step()
+    ms = []
+    for _ in range(args.steps):
+        flush.zero_()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        step()
+        b.record(stream)
+        b.synchronize()
+        ms.append(a.elapsed_time(b))
+    st = db.stats()
+    db.close()
+    return {"value": q.n_sets * len(ms) / (sum(ms) / 1000), "unit": "queries/s", "workload": args.config,
+            "ms_per_step": statistics.mean(ms), "scan_ms": st["scan_ms"],
+            "note": "the same workload and batch unsharded on rank 0's GPU, same K steps (device-resident inputs)"}
 
 
 def main():
@@ -471,10 +642,13 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="C2")
+    ap.add_argument("--config", default=None, help="BASELINE config; default C3 (N = 1), C4 (N > 1)")
     ap.add_argument("--unique", action="store_true", help="match-unique instead of match")
-    ap.add_argument("--shard", action="store_true",
-                    help="N > 1: partition-sharded database + NCCL exchange (strong scaling) instead of replicas")
+    ap.add_argument("--replicated", action="store_true",
+                    help="N > 1: every rank holds the whole database and matches its own batch (weak scaling) "
+                         "instead of the default partition sharding + NCCL exchange")
+    ap.add_argument("--no-hbm", action="store_true", help="skip the one-partition HBM roofline block")
+    ap.add_argument("--no-scaling-base", action="store_true", help="N > 1: skip the 1-GPU base on rank 0")
     # default layout = the B200 one (R18): balanced splits inside partitions +
     # tile AND masks; --tile-filter 0 --row-order 0 is the paper's lexicographic order + Alg. 4 prefix
     ap.add_argument("--tile-filter", type=int, default=1, choices=[0, 1, 2])
@@ -486,8 +660,10 @@ def main():
                     help="override the config's MAX_P (PAPER.md:361-371 sweep); 0 = config value")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-s", type=float, default=10.0, help="seconds of oracle work for cpu_baseline")
-    ap.add_argument("--ref-step-s", type=float, default=8.0, help="seconds per --impl reference step")
+    ap.add_argument("--ref-step-s", type=float, default=4.0, help="seconds per --impl reference step")
     args = ap.parse_args()
+    if args.config is None:
+        args.config = "C3" if int(os.environ.get("WORLD_SIZE", "1")) == 1 else "C4"
     if args.warmup < 3:
         args.warmup = 3
     if args.row_order == 1 and args.tile_filter == 0:

@@ -47,7 +47,7 @@
 extern "C" {
 #endif
 
-#define TM_ABI_VERSION 3u
+#define TM_ABI_VERSION 4u
 /* Bloom filter width and number of hash functions. */
 #define TM_SIG_BITS 192u
 #define TM_SIG_WORDS 3u
@@ -197,6 +197,9 @@ void tm_free(tm_db *db);         /* NULL-safe */
 const char *tm_strerror(tm_status s);
 const char *tm_last_error(void); /* thread-local detail of the last failure ("" if none) */
 uint32_t tm_abi_version(void);
+/* Identifier of the library build: a hash of its CUDA/C++ sources, fixed at compile time
+ * (lets measurement scripts tie a profile to the exact kernels it was taken on). */
+const char *tm_build_id(void);
 
 /* ---------------------------------------------------------- test hooks --- */
 
@@ -235,6 +238,11 @@ typedef struct {
     uint32_t scan_variant;     /* scan-kernel variant of the last call */
     uint32_t tuning;           /* 1: the handle is still timing variants for batches of this size
                                   (ceil log2 class), so later calls may run other variants */
+    /* shard exchange of the last sharded call (tm_match_batch_sharded_device; 0 otherwise) */
+    uint64_t xchg_send_bytes;  /* (query, key) pair bytes this handle sent to other owners        */
+    uint64_t xchg_recv_bytes;  /* ... and received from them                                      */
+    double xchg_ms;            /* CUDA-event time of count all-gather + exchange + owner merge    */
+    double local_ms;           /* CUDA-event time of the local S1-S8 part of a sharded call        */
 } tm_stats_t;
 
 tm_status tm_stats(const tm_db *db, tm_stats_t *out);

@@ -49,10 +49,24 @@ def needs_build() -> bool:
     return any(os.path.getmtime(d) > t for d in _deps())
 
 
-def _compile(src: str, verbose_ptxas: bool) -> str:
+def build_id() -> str:
+    """sha256 (16 hex) of every library source: identifies the kernels a profile was taken on."""
+    import hashlib
+    h = hashlib.sha256()
+    for d in sorted(_deps()):
+        if d.endswith("_build.py"):
+            continue
+        h.update(os.path.basename(d).encode())
+        with open(d, "rb") as f:
+            h.update(f.read())
+    return h.hexdigest()[:16]
+
+
+def _compile(src: str, verbose_ptxas: bool, bid: str) -> str:
     obj = os.path.join(BUILD, os.path.basename(src) + ".o")
     cmd = [NVCC, "-c", src, "-o", obj, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(),
-           "-Xcompiler", "-fPIC,-O3,-Wall", "--expt-relaxed-constexpr", "-DNDEBUG"]
+           "-Xcompiler", "-fPIC,-O3,-Wall", "--expt-relaxed-constexpr", "-DNDEBUG",
+           f"-DTM_BUILD_ID=\"{bid}\""]
     cmd += os.environ.get("TM_NVCC_FLAGS", "").split()  # experiments only (e.g. -DTM_BLOCK_TILES=4)
     if verbose_ptxas and src.endswith(".cu"):
         cmd += ["-Xptxas", "-v"]
@@ -69,7 +83,8 @@ def build(force: bool = False, verbose_ptxas: bool = False) -> str:
         return LIB
     os.makedirs(BUILD, exist_ok=True)
     with cf.ThreadPoolExecutor(max_workers=8) as ex:
-        objs = list(ex.map(lambda s: _compile(s, verbose_ptxas), _sources()))
+        bid = build_id()
+        objs = list(ex.map(lambda s: _compile(s, verbose_ptxas, bid), _sources()))
     tmp = LIB + f".tmp{os.getpid()}"
     cmd = [NVCC, "-shared", *ARCH, "-o", tmp, *objs, "-Xcompiler", "-fPIC", "-lpthread", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -77,6 +92,21 @@ def build(force: bool = False, verbose_ptxas: bool = False) -> str:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
     os.replace(tmp, LIB)
     return LIB
+
+
+def build_tools() -> str:
+    """Measurement tools (not the product): build/int_peak from scripts/int_peak.cu, the INT/logic
+    pipe microbenchmark whose result is bench.py's roofline peak."""
+    src = os.path.join(ROOT, "scripts", "int_peak.cu")
+    exe = os.path.join(ROOT, "build", "int_peak")
+    if os.path.exists(exe) and os.path.getmtime(exe) >= os.path.getmtime(src):
+        return exe
+    os.makedirs(os.path.dirname(exe), exist_ok=True)
+    r = subprocess.run([NVCC, "-O3", *ARCH, "-lineinfo", "-o", exe + ".tmp", src], capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"nvcc failed for {src}:\n{r.stdout}\n{r.stderr}")
+    os.replace(exe + ".tmp", exe)
+    return exe
 
 
 if __name__ == "__main__":

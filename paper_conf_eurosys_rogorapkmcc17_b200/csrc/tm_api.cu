@@ -637,7 +637,7 @@ void destroy_db(tm_db *db) {
     for (DevBuf *b : {&db->planes, &db->tand, &db->wsel, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
                       &db->in_voff, &db->in_tidx, &db->in_soff, &db->vsig, &db->qplanes, &db->bm, &db->word_off,
                       &db->qidx, &db->qoff, &db->item_cnt, &db->item_off, &db->out, &db->out_alt, &db->res_q,
-                      &db->res_k, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,
+                      &db->res_k, &db->res_off, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,
                       &db->mk, &db->xv_bytes, &db->xv_off, &db->xv_hash, &db->xv_pos, &db->xv_canon, &db->xs_off,
                       &db->xs_ids, &db->xk_off, &db->xk_keys, &db->xq_canon, &db->xq_ids, &db->xflag, &db->xcnt,
                       &db->xkoff, &db->xkcnt})
@@ -672,6 +672,11 @@ int check_device(int dev) {
 extern "C" {
 
 uint32_t tm_abi_version(void) { return TM_ABI_VERSION; }
+
+#ifndef TM_BUILD_ID
+#define TM_BUILD_ID "unknown"
+#endif
+const char *tm_build_id(void) { return TM_BUILD_ID; }
 
 const char *tm_strerror(tm_status s) {
     switch (s) {

@@ -655,11 +655,14 @@ void build_gpu(tm_db *db, uint64_t N, const uint64_t *s0, const uint64_t *s1, co
     std::vector<uint32_t> kp_lo(KP), kp_n(KP), row_off(KP + 1, 0);
     db->h_masks.assign(3 * (size_t)KP, 0);
     db->h_sizes.assign(KP, 0);
+    uint64_t rows64 = 0;  // padded rows summed in 64 bits: the table is addressed with u32 row ids
     for (uint32_t j = 0; j < KP; ++j) {
         const Partition &pt = parts[keep[j]];
         kp_lo[j] = (uint32_t)pt.begin;
         kp_n[j] = (uint32_t)(pt.end - pt.begin);
-        row_off[j + 1] = row_off[j] + (kp_n[j] + kTile - 1) / kTile * kTile;
+        rows64 += ((uint64_t)kp_n[j] + kTile - 1) / kTile * kTile;
+        if (rows64 > 0xFFFFFFF0ull) fail(TM_ERANGE, "more than 2^32 rows");
+        row_off[j + 1] = (uint32_t)rows64;
         for (int w = 0; w < 3; ++w) db->h_masks[3 * j + w] = pt.mask.w[w];
         db->h_sizes[j] = kp_n[j];
     }

@@ -32,9 +32,29 @@ struct StatusFail {
 
 [[noreturn]] inline void fail(tm_status s, const std::string &m) { throw StatusFail{s, m}; }
 
+// Device buffer owned by one object: move-only, freed by its destructor (or release()), so no
+// member of a handle can be missed on tm_free (res_off leaked).
 struct DevBuf {
     void *p = nullptr;
     size_t cap = 0;
+    DevBuf() = default;
+    DevBuf(const DevBuf &) = delete;
+    DevBuf &operator=(const DevBuf &) = delete;
+    DevBuf(DevBuf &&o) noexcept : p(o.p), cap(o.cap) {
+        o.p = nullptr;
+        o.cap = 0;
+    }
+    DevBuf &operator=(DevBuf &&o) noexcept {
+        if (this != &o) {
+            release();
+            p = o.p;
+            cap = o.cap;
+            o.p = nullptr;
+            o.cap = 0;
+        }
+        return *this;
+    }
+    ~DevBuf() { release(); }
     template <class T>
     T *as() const { return static_cast<T *>(p); }
     // grows (never shrinks); the caller guarantees the stream is idle w.r.t. the old contents
@@ -137,6 +157,7 @@ void finish_timing(tm_db *db, cudaStream_t s);
 tm_status translate(const CudaFail &f);
 int check_device(int dev);
 void check_tagsets_device(const tm_tagsets *t);
+void check_tagsets_host(const tm_tagsets *t, const char *what);
 int bits_for(uint64_t n);
 std::vector<uint32_t> assign_shards(const std::vector<Partition> &parts, uint32_t n_shards);
 void shard_destroy(tm_db *db);

@@ -301,6 +301,8 @@ tm_status tm_match_batch_sharded_device(tm_db *db, const tm_tagsets *q, int uniq
     // S1-S8 against the local partitions
     match_core(db, &dq, unique, s);
     finish_timing(db, s);
+    db->st.local_ms = db->st.total_ms;
+    TMCK(cudaEventRecord(db->ev[5], s));
     const uint32_t G = (uint32_t)db->nranks;
     const int r = db->rank;
     ncclComm_t comm = static_cast<ncclComm_t>(db->nccl_comm);
@@ -327,6 +329,13 @@ tm_status tm_match_batch_sharded_device(tm_db *db, const tm_tagsets *q, int uniq
     }
     TMNC(a.groupEnd());
     const uint64_t m = merge_pairs(db, db->xrecv.as<uint64_t>(), roff[G], q->n_sets, unique, s);
+    TMCK(cudaEventRecord(db->ev[4], s));
+    TMCK(cudaEventSynchronize(db->ev[4]));
+    float xms = 0;
+    TMCK(cudaEventElapsedTime(&xms, db->ev[5], db->ev[4]));
+    db->st.xchg_ms = xms;
+    db->st.xchg_send_bytes = 8 * (soff[G] - (soff[r + 1] - soff[r]));
+    db->st.xchg_recv_bytes = 8 * (roff[G] - (roff[r + 1] - roff[r]));
     out->n = m;
     out->query = db->mq.as<uint32_t>();
     out->key = db->mk.as<uint32_t>();

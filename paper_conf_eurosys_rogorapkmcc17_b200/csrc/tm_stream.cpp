@@ -26,6 +26,14 @@ uint64_t now_ns() {
         .count();
 }
 
+// One submitted query (its own tag strings), queued until a batch takes it.
+struct Query {
+    std::vector<uint8_t> bytes;
+    std::vector<uint64_t> tag_off{0};  // byte offsets of its tag strings
+    uint64_t ticket = 0, submit_ns = 0;
+};
+
+// A dispatched batch in the tm_tagsets CSR form (vocabulary = the batch's tag strings).
 struct Batch {
     std::vector<uint8_t> bytes;
     std::vector<uint64_t> tag_off{0};   // byte offsets of tag strings
@@ -39,31 +47,23 @@ struct Batch {
         submit_ns.clear();
     }
     size_t size() const { return tickets.size(); }
+    void append(const Query &q) {
+        const uint64_t base = bytes.size();
+        bytes.insert(bytes.end(), q.bytes.begin(), q.bytes.end());
+        for (size_t i = 1; i < q.tag_off.size(); ++i) tag_off.push_back(base + q.tag_off[i]);
+        set_off.push_back(tag_off.size() - 1);
+        tickets.push_back(q.ticket);
+        submit_ns.push_back(q.submit_ns);
+    }
 };
 
-// move the first n queries of src into dst (dst cleared), rebasing src's offsets
-void take_front(Batch &src, size_t n, Batch &dst) {
+// move the first n queued queries into dst (dst cleared): O(n), the rest of the queue stays put
+void take_front(std::deque<Query> &src, size_t n, Batch &dst) {
     dst.clear();
-    if (n >= src.size()) {
-        std::swap(dst, src);
-        src.clear();
-        return;
+    for (size_t i = 0; i < n && !src.empty(); ++i) {
+        dst.append(src.front());
+        src.pop_front();
     }
-    const uint64_t ntag = src.set_off[n], nbyte = src.tag_off[ntag];
-    dst.bytes.assign(src.bytes.begin(), src.bytes.begin() + nbyte);
-    dst.tag_off.assign(src.tag_off.begin(), src.tag_off.begin() + ntag + 1);
-    dst.set_off.assign(src.set_off.begin(), src.set_off.begin() + n + 1);
-    dst.tickets.assign(src.tickets.begin(), src.tickets.begin() + n);
-    dst.submit_ns.assign(src.submit_ns.begin(), src.submit_ns.begin() + n);
-    Batch rest;
-    rest.bytes.assign(src.bytes.begin() + nbyte, src.bytes.end());
-    rest.tag_off.clear();
-    for (size_t i = ntag; i < src.tag_off.size(); ++i) rest.tag_off.push_back(src.tag_off[i] - nbyte);
-    rest.set_off.clear();
-    for (size_t i = n; i < src.set_off.size(); ++i) rest.set_off.push_back(src.set_off[i] - ntag);
-    rest.tickets.assign(src.tickets.begin() + n, src.tickets.end());
-    rest.submit_ns.assign(src.submit_ns.begin() + n, src.submit_ns.end());
-    std::swap(src, rest);
 }
 
 struct Result {
@@ -71,6 +71,7 @@ struct Result {
     std::vector<uint32_t> keys;
     uint64_t dispatch_ns = 0, done_ns = 0;
     tm_status status = TM_OK;
+    std::string error;  // tm_last_error() of the failed batch (the dispatcher thread's detail)
 };
 
 }  // namespace
@@ -81,7 +82,7 @@ struct tm_stream {
     tm_stream_config cfg{};
     std::mutex mu;
     std::condition_variable cv_submit, cv_done;
-    tmb::Batch open;
+    std::deque<tmb::Query> open;  // submitted, not yet dispatched
     std::deque<tmb::Result *> done;
     uint64_t next_ticket = 0;
     uint64_t inflight = 0;  // submitted but not yet published
@@ -106,7 +107,7 @@ void dispatcher(tm_stream *st) {
                     st->cv_submit.wait(lk);
                     continue;
                 }
-                const uint64_t deadline = st->open.submit_ns[0] + (uint64_t)st->cfg.timeout_us * 1000ULL;
+                const uint64_t deadline = st->open.front().submit_ns + (uint64_t)st->cfg.timeout_us * 1000ULL;
                 const uint64_t t = now_ns();
                 if (st->cfg.timeout_us && t >= deadline) break;
                 if (st->cfg.timeout_us)
@@ -131,6 +132,7 @@ void dispatcher(tm_stream *st) {
         q.n_sets = work.size();
         tm_pairs pairs{};
         r->status = tm_match_batch(st->db, &q, st->cfg.unique, &pairs);
+        if (r->status != TM_OK) r->error = tm_last_error();  // thread-local: copy it for the poller
         r->tickets = work.tickets;
         r->submit_ns = work.submit_ns;
         r->key_off.assign(work.size() + 1, 0);
@@ -161,6 +163,7 @@ tm_status tm_stream_open(tm_db *db, const tm_stream_config *cfg, tm_stream **out
     if (!db || !cfg || !out) fail(TM_EINVAL, "NULL argument");
     if (cfg->max_batch == 0) fail(TM_EINVAL, "max_batch must be > 0");
     if (cfg->unique != 0 && cfg->unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
+    if (cfg->reserved) fail(TM_EINVAL, "reserved must be 0");
     tm_stream *st = new tm_stream();
     st->db = db;
     st->cfg = *cfg;
@@ -179,22 +182,20 @@ tm_status tm_stream_submit(tm_stream *st, const uint8_t *bytes, const uint64_t *
         if (tag_off[i + 1] < tag_off[i]) fail(TM_EINVAL, "tag_off not non-decreasing");
     const uint64_t nb = n_tags ? tag_off[n_tags] : 0;
     if (nb && !bytes) fail(TM_EINVAL, "bytes is NULL");
+    tmb::Query q;  // built outside the lock, queued only once complete
+    q.bytes.assign(bytes, bytes + nb);
+    q.tag_off.assign(tag_off, tag_off + (n_tags ? n_tags + 1 : 1));
     bool wake = false;
     {
         std::lock_guard<std::mutex> lk(st->mu);
         if (st->closing) fail(TM_ESTATE, "stream is closing");
-        tmb::Batch &b = st->open;
-        const uint64_t base = b.bytes.size();
-        b.bytes.insert(b.bytes.end(), bytes, bytes + nb);
-        for (uint64_t i = 1; i <= n_tags; ++i) b.tag_off.push_back(base + tag_off[i]);
-        b.set_off.push_back(b.tag_off.size() - 1);
-        *ticket = st->next_ticket++;
-        b.tickets.push_back(*ticket);
-        b.submit_ns.push_back(tmb::now_ns());
+        q.ticket = *ticket = st->next_ticket++;
+        q.submit_ns = tmb::now_ns();
+        st->open.push_back(std::move(q));
         st->inflight++;
-        // wake the dispatcher only when its decision can change: the batch became
+        // wake the dispatcher only when its decision can change: the queue became
         // non-empty (its timeout clock starts) or reached max_batch
-        wake = b.size() == 1 || b.size() >= st->cfg.max_batch;
+        wake = st->open.size() == 1 || st->open.size() >= st->cfg.max_batch;
     }
     if (wake) st->cv_submit.notify_one();
     return TM_OK;
@@ -216,8 +217,9 @@ tm_status tm_stream_poll(tm_stream *st, int wait, tm_stream_result *out) {
     }
     if (r->status != TM_OK) {
         const tm_status s = r->status;
+        const std::string msg = "batch failed on the GPU path: " + r->error;
         delete r;
-        fail(s, "batch failed on the GPU path");
+        fail(s, msg);
     }
     out->n_queries = r->tickets.size();
     out->tickets = r->tickets.data();
@@ -255,9 +257,18 @@ tm_status tm_stream_flush(tm_stream *st) {
 tm_status tm_stream_replay(tm_stream *st, const tm_tagsets *q, const uint64_t *arrival_ns) {
     TM_API_BEGIN
     if (!st || !q || !arrival_ns) fail(TM_EINVAL, "NULL argument");
-    if (q->n_sets && (!q->set_off || (q->n_vocab && !q->vocab_off))) fail(TM_EINVAL, "bad tag sets");
+    // the whole batch is validated before the first query is queued (offsets monotone and in
+    // range, tag indices < n_vocab): a malformed batch queues nothing
+    tmb::check_tagsets_host(q, "queries");
     const uint64_t t0 = tmb::now_ns();
     for (uint64_t i = 0; i < q->n_sets; ++i) {
+        tmb::Query one;
+        for (uint64_t t = q->set_off[i]; t < q->set_off[i + 1]; ++t) {
+            const uint64_t v = q->tag_idx ? q->tag_idx[t] : t;
+            const uint64_t a = q->vocab_off[v], e = q->vocab_off[v + 1];
+            one.bytes.insert(one.bytes.end(), q->vocab_bytes + a, q->vocab_bytes + e);
+            one.tag_off.push_back(one.bytes.size());
+        }
         const uint64_t due = t0 + arrival_ns[i];
         while (tmb::now_ns() < due) {
         }
@@ -265,19 +276,11 @@ tm_status tm_stream_replay(tm_stream *st, const tm_tagsets *q, const uint64_t *a
         {
             std::lock_guard<std::mutex> lk(st->mu);
             if (st->closing) fail(TM_ESTATE, "stream is closing");
-            tmb::Batch &b = st->open;
-            for (uint64_t t = q->set_off[i]; t < q->set_off[i + 1]; ++t) {
-                const uint64_t v = q->tag_idx ? q->tag_idx[t] : t;
-                if (v >= q->n_vocab) fail(TM_EINVAL, "tag_idx out of range");
-                const uint64_t a = q->vocab_off[v], e = q->vocab_off[v + 1];
-                b.bytes.insert(b.bytes.end(), q->vocab_bytes + a, q->vocab_bytes + e);
-                b.tag_off.push_back(b.bytes.size());
-            }
-            b.set_off.push_back(b.tag_off.size() - 1);
-            b.tickets.push_back(st->next_ticket++);
-            b.submit_ns.push_back(tmb::now_ns());
+            one.ticket = st->next_ticket++;
+            one.submit_ns = tmb::now_ns();
+            st->open.push_back(std::move(one));
             st->inflight++;
-            wake = b.size() == 1 || b.size() >= st->cfg.max_batch;
+            wake = st->open.size() == 1 || st->open.size() >= st->cfg.max_batch;
         }
         if (wake) st->cv_submit.notify_one();
     }

@@ -77,7 +77,9 @@ class tm_stats_t(ctypes.Structure):
                [(n, ctypes.c_double) for n in ("encode_ms", "route_ms", "scan_ms", "merge_ms", "total_ms")] + \
                [("scan_launches", ctypes.c_uint32), ("kernel_launches", ctypes.c_uint32),
                 ("exact_checked", ctypes.c_uint64), ("exact_kept", ctypes.c_uint64),
-                ("scan_variant", ctypes.c_uint32), ("tuning", ctypes.c_uint32)]
+                ("scan_variant", ctypes.c_uint32), ("tuning", ctypes.c_uint32),
+                ("xchg_send_bytes", ctypes.c_uint64), ("xchg_recv_bytes", ctypes.c_uint64),
+                ("xchg_ms", ctypes.c_double), ("local_ms", ctypes.c_double)]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
@@ -85,7 +87,7 @@ class tm_stats_t(ctypes.Structure):
 
 EXPORTS = ["tm_build", "tm_match_batch", "tm_match_batch_csr", "tm_match_batch_device", "tm_pairs_free",
            "tm_csr_free", "tm_free", "tm_strerror",
-           "tm_last_error", "tm_abi_version", "tm_encode", "tm_stats", "tm_partitions", "tm_partition_sigs",
+           "tm_last_error", "tm_abi_version", "tm_build_id", "tm_encode", "tm_stats", "tm_partitions", "tm_partition_sigs",
            "tm_owner_range", "tm_shard_plan", "tm_partition_host", "tm_last_result", "tm_shard_counts",
            "tm_shard_merge", "tm_nccl_unique_id", "tm_comm_init", "tm_match_batch_sharded_device",
            "tm_stream_open", "tm_stream_submit", "tm_stream_poll", "tm_stream_result_free", "tm_stream_flush",
@@ -119,6 +121,7 @@ def load(path: str = LIB_PATH):
     L.tm_strerror.argtypes = [ctypes.c_int]
     L.tm_last_error.restype = ctypes.c_char_p
     L.tm_abi_version.restype = ctypes.c_uint32
+    L.tm_build_id.restype = ctypes.c_char_p
     L.tm_encode.restype = ctypes.c_int
     L.tm_encode.argtypes = [P(tm_tagsets), vp, ctypes.c_int]
     L.tm_stats.restype = ctypes.c_int
@@ -352,6 +355,11 @@ def encode(sets, device: int = -1) -> np.ndarray:
 
 def abi_version() -> int:
     return int(load().tm_abi_version())
+
+
+def build_id() -> str:
+    """tm_build_id: hash of the sources the loaded library was compiled from."""
+    return load().tm_build_id().decode()
 
 
 # ------------------------------------------------------------ shard layer --

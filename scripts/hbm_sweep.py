@@ -64,7 +64,7 @@ def main():
             if B == 1 and db_sig is None:
                 db_sig = o2.encode(wl.db)
             ok = None
-            if B <= 8:   # brute-force parity of the B queries (cheap at small B)
+            if True:   # brute-force parity of the B queries at every B (<= 256 queries: seconds)
                 gq, gk = db.match_batch(q, False)
                 wq, wk = o2.match_brute(db_sig, wl.key_off, wl.keys, o2.encode(q), False)
                 ok = bool(np.array_equal(gq, wq) and np.array_equal(gk, wk))

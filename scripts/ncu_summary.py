@@ -83,7 +83,11 @@ def main():
               "alu_pipe_pct": num(m.get("sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active")),
               "issue_active_pct": num(m.get("smsp__issue_active.avg.pct_of_peak_sustained_active")),
               "warps_active_pct": num(m.get("sm__warps_active.avg.pct_of_peak_sustained_active")),
-              "l2_hit_pct": num(m.get("lts__t_sector_hit_rate.pct"))}
+              "l2_hit_pct": num(m.get("lts__t_sector_hit_rate.pct")),
+              # the library build and scan variant the capture was taken on (bench.py only uses the
+              # traffic for a line of the same build and variant)
+              "build_id": sys.argv[sys.argv.index("--build-id") + 1] if "--build-id" in sys.argv else None,
+              "variant": int(sys.argv[sys.argv.index("--variant") + 1]) if "--variant" in sys.argv else None}
         with open(sys.argv[sys.argv.index("--json") + 1], "w") as f:
             json.dump(js, f, indent=1)
 
