@@ -161,8 +161,8 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
     db->last_n = 0;
     db->last_Q = Q;
     if (Q == 0 || P == 0) return 0;
-    const uint64_t QW = (Q + 31) / 32;
-    const uint64_t n_words = (uint64_t)P * QW;
+    const uint64_t NB = route_blocks(Q);          // route blocks of 512 queries
+    const uint64_t n_words = (uint64_t)P * NB;    // (partition, route block) counts
     uint32_t launches = 0, cub_calls = 0;
 
     db->ctr.ensure(sizeof(DevCounters));
@@ -189,15 +189,17 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
     launches += 2;
     TMCK(cudaEventRecord(db->ev[1], s));
 
-    // S2: route (bitmap of mask_p subset-of q, scanned to a partition-major CSR)
+    // S2: route (Alg. 2, bit-sliced): per (partition, route block) counts, scanned to the
+    // offsets of a partition-major CSR of ascending query ids
     db->bm.ensure(n_words * 4);
     db->word_off.ensure((n_words + 1) * 8);
-    TMCK(launch_route_bitmap(db->masks.as<uint64_t>(), P, q0, q1, q2, Q, db->bm.as<uint32_t>(), s));
+    TMCK(launch_route(0, db->masks.as<uint64_t>(), P, q0, q1, q2, Q, db->bm.as<uint32_t>(), nullptr, nullptr, 0, s));
     launches++;
     size_t tb = 0;
-    TMCK(cub_exclusive_popc_scan(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words, nullptr, &tb, s));
-    TMCK(cub_exclusive_popc_scan(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words,
-                                 cub_tmp(db, tb), &tb, s));
+    TMCK(cub_exclusive_scan_u32_u64(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words, nullptr,
+                                    &tb, s));
+    TMCK(cub_exclusive_scan_u32_u64(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words,
+                                    cub_tmp(db, tb), &tb, s));
     cub_calls++;
     db->qoff.ensure((uint64_t)(P + 1) * 8);
     db->item_cnt.ensure((uint64_t)(P + 1) * 8);
@@ -209,11 +211,11 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         db->qidx.ensure(db->cap_qidx * 4);
         db->out.ensure(db->cap_out * 8);
         TMCK(cudaMemsetAsync(ctr, 0, offsetof(DevCounters, input_err), s));
-        TMCK(launch_route_scatter(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words,
-                                  (uint32_t)QW, db->qidx.as<uint32_t>(), db->cap_qidx, s));
+        TMCK(launch_route(1, db->masks.as<uint64_t>(), P, q0, q1, q2, Q, nullptr,
+                          db->word_off.as<unsigned long long>(), db->qidx.as<uint32_t>(), db->cap_qidx, s));
         // S3: per-partition batches -> work items
         const uint32_t range_rows = range_rows_env(db->n_rows);
-        TMCK(launch_items(db->word_off.as<unsigned long long>(), (uint32_t)QW, db->part_row.as<uint32_t>(),
+        TMCK(launch_items(db->word_off.as<unsigned long long>(), NB, db->part_row.as<uint32_t>(),
                           db->part_n.as<uint32_t>(), P, db->qoff.as<unsigned long long>(),
                           db->item_cnt.as<unsigned long long>(), ctr, range_rows, s));
         launches += 2;
@@ -250,6 +252,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         sp.filter = db->cfg.tile_filter;
         sp.wsel = db->wsel.as<uint8_t>();
         sp.range_rows = range_rows;
+        sp.one = 1;
         // variant: TM_SCAN_VARIANT if set; else a call whose partition batches are all small
         // (Q <= kSmallBatch) takes the streaming path only, in the streaming-only kernels (small
         // shared memory: 8 CTAs/SM) -- up to four queries checked directly (variant 6), 5-8
@@ -259,7 +262,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         const int forced = scan_variant_env();
         int var = forced;
         // the streaming-only kernels cannot take a filtered batch: a forced 6 / 7 maps to 0 / 5 then
-        if (var >= 6 && Q > (uint64_t)kSmallBatch) var = var == 6 ? 0 : 5;
+        if ((var == 6 || var == 7) && Q > (uint64_t)kSmallBatch) var = var == 6 ? 0 : 5;
         db->call_tunes = false;
         if (var < 0) {
             if (Q <= (uint64_t)kSmallBatch) {
@@ -270,7 +273,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
                 // batches below kTuneMinQ queries keep the default variant: a tuning round there
                 // would put slow candidates into a latency-bound stream for little gain
                 if (Q >= (uint64_t)kTuneMinQ && db->tune_calls[c] < 2 * kTuneN) {
-                    var = kTune[db->tune_calls[c] % kTuneN];
+                    var = db->tune[db->tune_calls[c] % kTuneN];
                     db->call_tunes = true;
                 } else {
                     var = db->variant[c];
@@ -377,9 +380,9 @@ void finish_timing(tm_db *db, cudaStream_t s) {
         const int c = db->call_class;
         if (db->tune_calls[c] >= kTuneN) db->tune_cost[c][db->call_variant] = ms * 1e6 / dec;
         if (++db->tune_calls[c] == 2 * kTuneN) {
-            int best = kTune[0];
+            int best = db->tune[0];
             for (int i = 1; i < kTuneN; ++i)
-                if (db->tune_cost[c][kTune[i]] < db->tune_cost[c][best]) best = kTune[i];
+                if (db->tune_cost[c][db->tune[i]] < db->tune_cost[c][best]) best = db->tune[i];
             db->variant[c] = best;
         }
     }
@@ -621,6 +624,7 @@ tm_db *new_db(const tm_config *cfg) {
     if (cfg) db->cfg = *cfg;
     if (db->cfg.max_partition == 0) db->cfg.max_partition = TM_DEFAULT_MAX_PARTITION;
     if (db->cfg.n_shards == 0) db->cfg.n_shards = 1;
+    if (db->cfg.tile_filter == 2) db->set_tune(kTuneDense);  // no pre-filter: the dense scan
     return db;
 }
 

@@ -109,11 +109,17 @@ struct tm_db {
     static constexpr int kClasses = 33;
     int variant[kClasses], tune_calls[kClasses] = {};
     double tune_cost[kClasses][kScanVariants] = {};
+    const int *tune = kTune;      // the candidates of this table (kTune, or kTuneDense without a pre-filter)
     int call_variant = kTune[0];  // the variant the last call launched
     int call_class = 0;           // the batch-size class of the last call
     bool call_tunes = false;      // the last call is a tuning sample
     tm_db() {
         for (int &v : variant) v = kTune[0];
+    }
+    void set_tune(const int *t) {
+        tune = t;
+        call_variant = t[0];
+        for (int &v : variant) v = t[0];
     }
     int grid_of[kScanVariants] = {};
     // database (device)

@@ -28,9 +28,10 @@ constexpr int kScanWarps = 4;      // warps per CTA
 constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch); 640 fits 7 CTAs/SM of shared memory and measured 1.3% faster than 512 (profiles/r1v34_ab.txt)
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
-constexpr int kScanVariants = 8;    // k_scan variants (TM_SCAN_VARIANT)
+constexpr int kScanVariants = 13;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {5, 0};  // variants the handle times on its first calls (first = default); 2 never won
 constexpr int kTuneN = 2;
+constexpr int kTuneDense[] = {10, 9};  // tables without a pre-filter (tile_filter = 2): the dense scan
 constexpr int kTuneMinQ = 4096;     // smaller calls are not tuned (default variant kTune[0])
 
 struct DevCounters {            // zeroed at the start of every match call
@@ -65,6 +66,7 @@ struct ScanParams {
     uint32_t filter;                  // 0 prefix, 1 AND, 2 none
     const uint8_t *wsel;              // [rows] pre-check word per row (variant 5)
     uint32_t range_rows;              // rows per work item (multiple of 256)
+    uint32_t one;                     // 1 (a run-time operand, so the FMA-pipe accumulate stays an IMAD)
 };
 
 // ------------------------------------------------------------ launchers --
@@ -74,11 +76,13 @@ cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_
 cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, const uint64_t *set_off,
                                uint64_t n_sets, uint64_t n_tags, uint64_t n_vocab, uint64_t *w0, uint64_t *w1,
                                uint64_t *w2, unsigned int *err, cudaStream_t s);
-cudaError_t launch_route_bitmap(const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
-                                const uint64_t *q2, uint64_t n_q, uint32_t *bm, cudaStream_t s);
-cudaError_t launch_route_scatter(const uint32_t *bm, const unsigned long long *word_off, uint64_t n_words,
-                                 uint32_t qw, uint32_t *qidx, unsigned long long cap, cudaStream_t s);
-cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const uint32_t *part_row,
+// S2, bit-sliced Alg. 2 in two passes: pass 0 writes counts[p * NB + blk] (NB = route_blocks(n_q)),
+// pass 1 scatters query ids at the scanned offsets off[p * NB + blk] into qidx (capacity cap).
+uint64_t route_blocks(uint64_t n_q);
+cudaError_t launch_route(int pass, const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
+                         const uint64_t *q2, uint64_t n_q, uint32_t *counts, const unsigned long long *off,
+                         uint32_t *qidx, unsigned long long cap, cudaStream_t s);
+cudaError_t launch_items(const unsigned long long *word_off, uint64_t qw, const uint32_t *part_row,
                          const uint32_t *part_n, uint32_t n_parts, unsigned long long *qoff,
                          unsigned long long *item_cnt, DevCounters *ctr, uint32_t range_rows, cudaStream_t s);
 uint32_t range_rows_env(uint64_t n_rows);  // TM_RANGE_ROWS (multiple of 256), else by table size
@@ -97,8 +101,8 @@ cudaError_t launch_gather_u64(const uint64_t *src, const uint32_t *idx, uint64_t
 cudaError_t launch_iota(uint32_t *v, uint64_t n, cudaStream_t s);
 
 // CUB wrappers (temp storage managed by the caller through `tmp`/`tmp_bytes`).
-cudaError_t cub_exclusive_popc_scan(const uint32_t *bm, unsigned long long *out, uint64_t n, void *tmp,
-                                    size_t *tmp_bytes, cudaStream_t s);
+cudaError_t cub_exclusive_scan_u32_u64(const uint32_t *in, unsigned long long *out, uint64_t n, void *tmp,
+                                      size_t *tmp_bytes, cudaStream_t s);
 cudaError_t cub_exclusive_scan_u64(const unsigned long long *in, unsigned long long *out, uint64_t n, void *tmp,
                                    size_t *tmp_bytes, cudaStream_t s);
 cudaError_t cub_sort_pairs_u64_u32(const uint64_t *kin, uint64_t *kout, const uint32_t *vin, uint32_t *vout,

@@ -104,63 +104,123 @@ __global__ void k_encode_sets(const uint64_t *__restrict__ vsig, const uint32_t 
 }
 
 // ------------------------------------------------------------------ S2 ---
-// Warp w of the grid owns 32 consecutive queries (one per lane) and tests them
-// against every partition mask staged in shared memory; bitmap word
-// bm[p * QW + qw] = ballot(mask_p subset-of q) for query word qw.
-constexpr int kRouteWarps = 8;
-constexpr int kRouteMaskTile = 512;
+// Alg. 2 bit-sliced: partition p is routed to query q iff mask_p is a subset
+// of sig(q), i.e. iff no one-bit of mask_p is a zero-bit of q.  A warp owns a route block of
+// kRouteWB query words (32 queries each) and first transposes them into
+//   Z[pos][i] = ballot over the 32 queries of word i of "bit pos of q is 0"   (pos = 64 w + j)
+// in shared memory; then lane l takes partition p = g + l and ORs Z[pos] over the one-bits pos
+// of its mask (a mask has ~2-5 bits): ~Z-OR is the 32-query routing word of (p, word i), for
+// all kRouteWB words at once (four LDS.128 per mask bit).  Per (partition, 32 queries) that is
+// a few instructions per LANE instead of a 6-op test per (partition, query): routing cost stays
+// small when MAX_P is small and partitions are many.
+// Two passes over the same function: count (per (partition, route block) counts, scanned into
+// the partition-major CSR offsets) and scatter (ascending query ids per partition).  Scratch:
+// 12 B per (partition, 512 queries) instead of a dense P x Q bitmap.
+constexpr int kRouteWB = 16;                 // query words per route block (one warp)
+constexpr int kRouteBlockQ = 32 * kRouteWB;  // 512 queries
+constexpr int kRouteWarps = 4;               // warps per CTA (48 KB of Z)
 
-__global__ void __launch_bounds__(kRouteWarps * 32) k_route_bitmap(const uint64_t *__restrict__ masks,
-                                                                   uint32_t n_parts, const uint64_t *__restrict__ q0,
-                                                                   const uint64_t *__restrict__ q1,
-                                                                   const uint64_t *__restrict__ q2, uint64_t n_q,
-                                                                   uint32_t *__restrict__ bm, uint64_t qw_total) {
-    __shared__ uint64_t sm[3 * kRouteMaskTile];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint64_t qw = (uint64_t)blockIdx.x * kRouteWarps + warp;
-    const uint64_t q = qw * 32 + lane;
-    const bool valid = q < n_q;
-    uint64_t a0 = 0, a1 = 0, a2 = 0;
-    if (valid) {
-        a0 = q0[q];
-        a1 = q1[q];
-        a2 = q2[q];
-    }
-    for (uint32_t base = 0; base < n_parts; base += kRouteMaskTile) {
-        const uint32_t nm = min((uint32_t)kRouteMaskTile, n_parts - base);
-        __syncthreads();
-        for (uint32_t i = threadIdx.x; i < 3 * nm; i += blockDim.x) sm[i] = masks[3 * (uint64_t)base + i];
-        __syncthreads();
-        if (qw >= qw_total) continue;
-        for (uint32_t g = 0; g < nm; g += 32) {
-            uint32_t mine = 0;
-            const uint32_t ng = min(32u, nm - g);
-            for (uint32_t j = 0; j < ng; ++j) {
-                const uint64_t *m = sm + 3 * (g + j);
-                const bool ok = valid && (((m[0] & ~a0) | (m[1] & ~a1) | (m[2] & ~a2)) == 0);
-                const uint32_t b = __ballot_sync(0xffffffffu, ok);
-                if ((uint32_t)lane == j) mine = b;
+__device__ __forceinline__ void route_build_z(uint32_t *__restrict__ z, const uint64_t *__restrict__ q0,
+                                              const uint64_t *__restrict__ q1, const uint64_t *__restrict__ q2,
+                                              uint64_t qb, uint64_t n_q, int lane) {
+    for (int i = 0; i < kRouteWB; ++i) {
+        const uint64_t q = qb + (uint64_t)i * 32 + lane;
+        uint64_t a[3] = {~0ULL, ~0ULL, ~0ULL};  // past the batch: all ones (no zero bits); masked by `valid`
+        if (q < n_q) {
+            a[0] = __ldg(q0 + q);
+            a[1] = __ldg(q1 + q);
+            a[2] = __ldg(q2 + q);
+        }
+#pragma unroll
+        for (int w = 0; w < 3; ++w) {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const uint32_t x = (uint32_t)(a[w] >> (32 * h));
+                uint32_t mine = 0;
+#pragma unroll
+                for (int t = 0; t < 32; ++t) {
+                    const uint32_t b = __ballot_sync(0xffffffffu, ((x >> t) & 1u) == 0u);
+                    if (lane == t) mine = b;
+                }
+                z[(64 * w + 32 * h + lane) * kRouteWB + i] = mine;
             }
-            if ((uint32_t)lane < ng) bm[(uint64_t)(base + g + lane) * qw_total + qw] = mine;
         }
     }
 }
 
-// One thread per bitmap word: write the word's query ids at its scanned offset.
-__global__ void k_route_scatter(const uint32_t *__restrict__ bm, const unsigned long long *__restrict__ word_off,
-                                uint64_t n_words, uint32_t qw_total, uint32_t *__restrict__ qidx,
-                                unsigned long long cap) {
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i >= n_words) return;
-    uint32_t b = bm[i];
-    if (!b) return;
-    unsigned long long o = word_off[i];
-    const uint32_t qbase = (uint32_t)(i % qw_total) * 32u;
-    while (b) {
-        const int l = __ffs(b) - 1;
-        b &= b - 1;
-        if (o < cap) qidx[o] = qbase + (uint32_t)l;
-        ++o;
+// PASS 0: counts[p * NB + blk] = routed queries of partition p in route block blk.
+// PASS 1: scatter the routed query ids of (p, blk) at off[p * NB + blk] (ascending query order).
+template <int PASS>
+__global__ void __launch_bounds__(kRouteWarps * 32) k_route(const uint64_t *__restrict__ masks, uint32_t n_parts,
+                                                            const uint64_t *__restrict__ q0,
+                                                            const uint64_t *__restrict__ q1,
+                                                            const uint64_t *__restrict__ q2, uint64_t n_q,
+                                                            uint64_t n_blocks, uint32_t *__restrict__ counts,
+                                                            const unsigned long long *__restrict__ off,
+                                                            uint32_t *__restrict__ qidx, unsigned long long cap) {
+    extern __shared__ __align__(16) uint32_t zsm[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint64_t blk = (uint64_t)blockIdx.x * kRouteWarps + warp;
+    if (blk >= n_blocks) return;  // warp-uniform; no CTA barrier below
+    uint32_t *z = zsm + warp * (192 * kRouteWB);
+    const uint64_t qb = blk * kRouteBlockQ;
+    route_build_z(z, q0, q1, q2, qb, n_q, lane);
+    __syncwarp();
+    // valid-query mask of each word of the block (warp-uniform)
+    const uint64_t nvq = n_q - qb;  // > 0
+    for (uint32_t g = 0; g < n_parts; g += 32) {
+        const uint32_t p = g + lane;
+        uint64_t m[3] = {0, 0, 0};
+        if (p < n_parts) {
+            m[0] = __ldg(masks + 3 * (uint64_t)p);
+            m[1] = __ldg(masks + 3 * (uint64_t)p + 1);
+            m[2] = __ldg(masks + 3 * (uint64_t)p + 2);
+        }
+        uint32_t acc[kRouteWB];
+#pragma unroll
+        for (int i = 0; i < kRouteWB; ++i) acc[i] = 0;
+#pragma unroll
+        for (int w = 0; w < 3; ++w) {
+            uint64_t mw = m[w];
+            while (mw) {
+                const int j = __ffsll((long long)mw) - 1;
+                mw &= mw - 1;
+                const uint4 *zz = reinterpret_cast<const uint4 *>(z + (64 * w + j) * kRouteWB);
+#pragma unroll
+                for (int v = 0; v < kRouteWB / 4; ++v) {
+                    const uint4 x = zz[v];
+                    acc[4 * v + 0] |= x.x;
+                    acc[4 * v + 1] |= x.y;
+                    acc[4 * v + 2] |= x.z;
+                    acc[4 * v + 3] |= x.w;
+                }
+            }
+        }
+        if (p >= n_parts) continue;
+        if constexpr (PASS == 0) {
+            uint32_t c = 0;
+#pragma unroll
+            for (int i = 0; i < kRouteWB; ++i) {
+                const uint64_t lo = 32ULL * i;
+                const uint32_t vm = nvq > lo ? (nvq - lo >= 32 ? ~0u : ((1u << (nvq - lo)) - 1u)) : 0u;
+                c += __popc(~acc[i] & vm);
+            }
+            counts[(uint64_t)p * n_blocks + blk] = c;
+        } else {
+            unsigned long long o = off[(uint64_t)p * n_blocks + blk];
+#pragma unroll
+            for (int i = 0; i < kRouteWB; ++i) {
+                const uint64_t lo = 32ULL * i;
+                const uint32_t vm = nvq > lo ? (nvq - lo >= 32 ? ~0u : ((1u << (nvq - lo)) - 1u)) : 0u;
+                uint32_t r = ~acc[i] & vm;
+                while (r) {
+                    const int t = __ffs(r) - 1;
+                    r &= r - 1;
+                    if (o < cap) qidx[o] = (uint32_t)(qb + lo + (uint32_t)t);
+                    ++o;
+                }
+            }
+        }
     }
 }
 
@@ -179,7 +239,7 @@ __device__ __forceinline__ uint32_t part_range_rows(unsigned long long nq, uint3
 
 // Per partition: routed query count -> (chunks of kChunk queries) x (ranges of
 // range_rows rows) work items.
-__global__ void k_items(const unsigned long long *__restrict__ word_off, uint32_t qw_total,
+__global__ void k_items(const unsigned long long *__restrict__ word_off, uint64_t qw_total,
                         const uint32_t *__restrict__ part_row, const uint32_t *__restrict__ part_n, uint32_t n_parts,
                         unsigned long long *__restrict__ qoff, unsigned long long *__restrict__ item_cnt,
                         DevCounters *ctr, uint32_t range_rows) {
@@ -293,9 +353,27 @@ __device__ __forceinline__ void store_survivor(uint32_t *sw, uint16_t *sbi, uint
 
 // Four independent accumulators (one per survivor lane of the uint4) keep the predicated ORs
 // off a single serial dependency chain; the caller ORs them together.
-template <int B>
+// IMAD = true: the predicated accumulate is an integer multiply-add (acc += one * bit; the bits of an
+// accumulator are disjoint, so + is |), which runs on the FMA pipe instead of the ALU pipe: the
+// pre-check then puts 2 of its 3 ops per pair on the ALU pipe (scripts/int_peak.cu measures both).
+template <int B, bool IMAD = false>
 __device__ __forceinline__ void precheck4x2(uint32_t &c0, uint32_t &c1, uint32_t &c2, uint32_t &c3, uint32_t a,
-                                            uint4 v, uint32_t b, uint4 u) {
+                                            uint4 v, uint32_t b, uint4 u, uint32_t one = 1u) {
+    if constexpr (IMAD) {
+        asm("{\n\t.reg .pred p0, p1, p2, p3;\n\t.reg .b32 t0, t1, t2, t3, s0, s1, s2, s3;\n\t"
+            "not.b32 t0, %5;\n\tnot.b32 t1, %6;\n\tnot.b32 t2, %7;\n\tnot.b32 t3, %8;\n\t"
+            "and.b32 t0, t0, %4;\n\tand.b32 t1, t1, %4;\n\tand.b32 t2, t2, %4;\n\tand.b32 t3, t3, %4;\n\t"
+            "not.b32 s0, %10;\n\tnot.b32 s1, %11;\n\tnot.b32 s2, %12;\n\tnot.b32 s3, %13;\n\t"
+            "and.b32 s0, s0, %9;\n\tand.b32 s1, s1, %9;\n\tand.b32 s2, s2, %9;\n\tand.b32 s3, s3, %9;\n\t"
+            "or.b32 t0, t0, s0;\n\tor.b32 t1, t1, s1;\n\tor.b32 t2, t2, s2;\n\tor.b32 t3, t3, s3;\n\t"
+            "setp.eq.u32 p0, t0, 0;\n\tsetp.eq.u32 p1, t1, 0;\n\tsetp.eq.u32 p2, t2, 0;\n\tsetp.eq.u32 p3, t3, 0;\n\t"
+            "@p0 mad.lo.u32 %0, %18, %14, %0;\n\t@p1 mad.lo.u32 %1, %18, %15, %1;\n\t"
+            "@p2 mad.lo.u32 %2, %18, %16, %2;\n\t@p3 mad.lo.u32 %3, %18, %17, %3;\n\t}"
+            : "+r"(c0), "+r"(c1), "+r"(c2), "+r"(c3)
+            : "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "r"(b), "r"(u.x), "r"(u.y), "r"(u.z), "r"(u.w), "n"(B),
+              "n"(B << 1), "n"(B << 2), "n"(B << 3), "r"(one));
+        return;
+    }
     asm("{\n\t.reg .pred p0, p1, p2, p3;\n\t.reg .b32 t0, t1, t2, t3, s0, s1, s2, s3;\n\t"
         "not.b32 t0, %5;\n\tnot.b32 t1, %6;\n\tnot.b32 t2, %7;\n\tnot.b32 t3, %8;\n\t"
         "and.b32 t0, t0, %4;\n\tand.b32 t1, t1, %4;\n\tand.b32 t2, t2, %4;\n\tand.b32 t3, t3, %4;\n\t"
@@ -465,8 +543,10 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // MINB: resident CTAs per SM the register allocator must allow (__launch_bounds__); shared memory
 // caps residency at 8 CTAs, which ptxas cannot see (the scan's shared memory is dynamic).
 // STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
-template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8, bool STREAM = false>
+// OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>).
+template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
+    constexpr bool kImad = (OPT & 1) != 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -803,7 +883,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                             // ---- pre-check: the lane's word against 32 survivors, pass bits in acc
                             uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0;
                             const uint32_t pa = my_plane + k0 * 4, pa2 = my_plane2 + k0 * 4;
-#define TM_PRE(B, o) precheck4x2<B>(c0, c1, c2, c3, aw, lds128(pa + (o)), aw2, lds128(pa2 + (o)))
+#define TM_PRE(B, o) precheck4x2<B, kImad>(c0, c1, c2, c3, aw, lds128(pa + (o)), aw2, lds128(pa2 + (o)), p.one)
                             TM_PRE(1u << 0, 0);
                             TM_PRE(1u << 4, 16);
                             if (cnt > 8) {
@@ -987,6 +1067,267 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
     }
 }
 
+// ------------------------------------------------------------ dense scan ---
+// Unfiltered subset scan (tables built with tile_filter = 2: the plain Alg. 3 scan, and the HBM
+// roofline sweep of SURVEY 8(d)).  No pre-filter, so no survivor compaction: the item's query
+// batch is staged once as six 32-bit word planes, every lane holds two consecutive rows, and the
+// two-word pre-check of the filtered path (necessary condition, 3 ops per (row, query), four
+// queries per LDS.128 pair) runs against the whole batch in groups of 32 queries; only passing
+// (row, query) pairs get the full six-word check (Alg. 3) and are emitted.
+// BULK = false: lanes load their rows straight from HBM (16-B non-allocating loads).
+// BULK = true : each warp streams its 64-row units through a ring of kDenseStages shared-memory
+//               stages filled by 1-D bulk copies (cp.async.bulk, completion on an mbarrier):
+//               the next units are in flight while the current one is checked, with no
+//               registers held for outstanding loads (north_star's "TMA staging of a
+//               partition tile").
+constexpr int kDenseStages = 3;
+constexpr int kDenseRows = 64;                  // rows per unit (two per lane)
+constexpr int kDpStride = kChunk + 4;           // word-plane stride: 16 B mod 128 -> planes on disjoint bank quads
+
+struct DenseSmemBase {
+    uint32_t dp[6][kDpStride];                  // the batch as word planes
+    const uint32_t *qid;
+    unsigned long long item;
+    unsigned int unit_ctr;
+    unsigned long long cnt[3];
+    uint2 pend[kScanWarps][kPend];
+};
+struct DenseSmemBulk : DenseSmemBase {
+    __align__(16) uint64_t stage[kScanWarps][kDenseStages][3 * kDenseRows];  // per warp: ring of row tiles
+    __align__(16) uint8_t wstage[kScanWarps][kDenseStages][kDenseRows];      // their pre-check word bytes
+    __align__(8) unsigned long long bar[kScanWarps][kDenseStages];           // one mbarrier per stage
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(unsigned long long *bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long *bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ bool mbar_try_wait(unsigned long long *bar, uint32_t parity) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred P1;\n\tmbarrier.try_wait.parity.shared::cta.b64 P1, [%1], %2;\n\tselp.u32 %0, 1, 0, P1;\n\t}"
+        : "=r"(ok)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    return ok != 0;
+}
+
+// 1-D bulk copy global -> shared (TMA engine), completing `bytes` on the mbarrier
+__device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t bytes, unsigned long long *bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     smem_u32(dst)),
+                 "l"(src), "r"(bytes), "r"(smem_u32(bar))
+                 : "memory");
+}
+
+template <bool BULK, int OPT = 0>
+__global__ void __launch_bounds__(kScanWarps * 32, BULK ? 6 : 7) k_dense(const ScanParams p) {
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    using Smem = typename std::conditional<BULK, DenseSmemBulk, DenseSmemBase>::type;
+    Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
+    constexpr bool kImad = (OPT & 1) != 0;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    uint32_t st_checks = 0, st_matched = 0;
+    uint32_t npend = 0;
+    uint32_t par = 0;  // BULK: expected phase parity of each of the warp's stages (bit s)
+    const unsigned long long n_items = p.item_off[p.n_parts];
+    if (blockIdx.x == 0 && threadIdx.x == 0) p.ctr->n_items = n_items;
+    if (p.ctr->routed > p.qcap) return;
+    if (threadIdx.x < 3) sm.cnt[threadIdx.x] = 0;
+    if constexpr (BULK) {
+        if (lane == 0)
+            for (int i = 0; i < kDenseStages; ++i) mbar_init(&sm.bar[warp][i], 1);
+    }
+    const uint32_t dp_base = smem_u32(sm.dp[0]);
+    constexpr uint32_t kPl = kDpStride * 4;
+
+    for (;;) {
+        if (lane == 0 && (st_checks | st_matched)) {
+            atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
+            atomicAdd(&sm.cnt[2], (unsigned long long)st_matched);
+        }
+        st_checks = st_matched = 0;
+        if (threadIdx.x == 0) {
+            sm.item = atomicAdd(&p.ctr->item_ctr, 1ULL);
+            sm.unit_ctr = 0;
+        }
+        __syncthreads();  // also orders the mbarrier inits before their first use
+        const unsigned long long item = sm.item;
+        if (item >= n_items) break;
+        uint32_t lo = 0, hi = p.n_parts;
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (__ldg(p.item_off + mid) <= item) lo = mid; else hi = mid;
+        }
+        const uint32_t part = lo;
+        const uint32_t prow = __ldg(p.part_row + part);
+        const uint32_t rows = __ldg(p.part_row + part + 1) - prow;
+        const uint32_t real_end = prow + __ldg(p.part_n + part);
+        const unsigned long long pq0 = __ldg(p.qoff + part), pq1 = __ldg(p.qoff + part + 1);
+        const uint32_t rr = part_range_rows(pq1 - pq0, p.range_rows);
+        const uint32_t nrange = (rows + rr - 1) / rr;
+        const unsigned long long local = item - __ldg(p.item_off + part);
+        const uint32_t chunk = (uint32_t)(local / nrange), range = (uint32_t)(local % nrange);
+        const unsigned long long qbeg = pq0 + (unsigned long long)chunk * kChunk;
+        const uint32_t nq = (uint32_t)min((unsigned long long)kChunk, pq1 - qbeg);
+        const uint32_t rlo = prow + range * rr;
+        const uint32_t rhi = min(rlo + rr, prow + rows);
+        const uint32_t vend = min(real_end, rhi);
+        if (threadIdx.x == 0) sm.qid = p.qidx + qbeg;
+        // the batch as six word planes
+        for (uint32_t i = threadIdx.x; i < nq; i += blockDim.x) {
+            const uint32_t q = __ldg(p.qidx + qbeg + i);
+            const uint64_t a0 = __ldg(p.q0 + q), a1 = __ldg(p.q1 + q), a2 = __ldg(p.q2 + q);
+            sm.dp[0][i] = (uint32_t)a0;
+            sm.dp[1][i] = (uint32_t)(a0 >> 32);
+            sm.dp[2][i] = (uint32_t)a1;
+            sm.dp[3][i] = (uint32_t)(a1 >> 32);
+            sm.dp[4][i] = (uint32_t)a2;
+            sm.dp[5][i] = (uint32_t)(a2 >> 32);
+        }
+        __syncthreads();
+        const uint32_t nunit = (rhi - rlo + kDenseRows - 1) / kDenseRows;
+        auto take = [&]() {
+            uint32_t u = 0;
+            if (lane == 0) u = atomicAdd(&sm.unit_ctr, 1u);
+            return __shfl_sync(0xffffffffu, u, 0);
+        };
+        // BULK: fill stage si with unit u (lane 0): 3 planes + the word bytes, nr = 32 or 64 rows
+        auto issue = [&](uint32_t si, uint32_t u) {
+            if constexpr (BULK) {
+                if (lane == 0) {
+                    const uint32_t r0 = rlo + u * kDenseRows;
+                    const uint32_t nr = min((uint32_t)kDenseRows, rhi - r0);
+                    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // prior generic reads of the stage
+                    mbar_expect_tx(&sm.bar[warp][si], nr * 25);
+                    bulk_g2s(&sm.stage[warp][si][0], p.w0 + r0, nr * 8, &sm.bar[warp][si]);
+                    bulk_g2s(&sm.stage[warp][si][kDenseRows], p.w1 + r0, nr * 8, &sm.bar[warp][si]);
+                    bulk_g2s(&sm.stage[warp][si][2 * kDenseRows], p.w2 + r0, nr * 8, &sm.bar[warp][si]);
+                    bulk_g2s(&sm.wstage[warp][si][0], p.wsel + r0, nr, &sm.bar[warp][si]);
+                }
+            }
+        };
+        // BULK: the warp's reserved units in issue order (stage of ring0 = si, ring1 = si + 1, ...);
+        // rotated by value so no array is indexed dynamically (no local memory)
+        static_assert(kDenseStages == 3, "the ring below is written for three stages");
+        uint32_t ring0 = 0, ring1 = 0, ring2 = 0;
+        if constexpr (BULK) {
+            ring0 = take();
+            if (ring0 < nunit) issue(0, ring0);
+            ring1 = take();
+            if (ring1 < nunit) issue(1, ring1);
+            ring2 = take();
+            if (ring2 < nunit) issue(2, ring2);
+        }
+        uint32_t si = 0;
+        for (;;) {
+            uint32_t u;
+            ulonglong2 v0, v1, v2;
+            uint32_t wab;
+            if constexpr (BULK) {
+                u = ring0;
+                if (u >= nunit) break;  // later reservations are larger: nothing is in flight
+                while (!mbar_try_wait(&sm.bar[warp][si], (par >> si) & 1u)) {
+                }
+                par ^= 1u << si;
+                const uint64_t *st = sm.stage[warp][si];
+                v0 = *reinterpret_cast<const ulonglong2 *>(st + 2 * lane);
+                v1 = *reinterpret_cast<const ulonglong2 *>(st + kDenseRows + 2 * lane);
+                v2 = *reinterpret_cast<const ulonglong2 *>(st + 2 * kDenseRows + 2 * lane);
+                wab = *reinterpret_cast<const unsigned short *>(&sm.wstage[warp][si][2 * lane]);
+                __syncwarp();  // every lane has read the stage: refill it now
+                const uint32_t nu = take();
+                if (nu < nunit) issue(si, nu);
+                ring0 = ring1;
+                ring1 = ring2;
+                ring2 = nu;
+                si = si == kDenseStages - 1 ? 0 : si + 1;
+            } else {
+                u = take();
+                if (u >= nunit) break;
+                const uint32_t ra0 = rlo + u * kDenseRows + 2 * (uint32_t)lane;
+                v0 = v1 = v2 = make_ulonglong2(~0ULL, ~0ULL);
+                wab = 0x1010u;
+                if (ra0 < rhi) {
+                    v0 = ldg_stream2(p.w0 + ra0);
+                    v1 = ldg_stream2(p.w1 + ra0);
+                    v2 = ldg_stream2(p.w2 + ra0);
+                    wab = __ldg(reinterpret_cast<const unsigned short *>(p.wsel + ra0));
+                }
+            }
+            const uint32_t u0 = rlo + u * kDenseRows;
+            const uint32_t ra = u0 + 2 * (uint32_t)lane, rb = ra + 1;
+            const uint64_t a0 = v0.x, a1 = v1.x, a2 = v2.x, b0 = v0.y, b1 = v1.y, b2 = v2.y;
+            const bool va = ra < vend, vb = rb < vend;
+            const uint32_t wa = wab & 0xffu, wb = wab >> 8;
+            const uint32_t xa = pick_word(a0, a1, a2, wa & 15u, va), ya = pick_word(a0, a1, a2, wa >> 4, va);
+            const uint32_t xb = pick_word(b0, b1, b2, wb & 15u, vb), yb = pick_word(b0, b1, b2, wb >> 4, vb);
+            const uint32_t pxa = dp_base + (wa & 15u) * kPl, pya = dp_base + (wa >> 4) * kPl;
+            const uint32_t pxb = dp_base + (wb & 15u) * kPl, pyb = dp_base + (wb >> 4) * kPl;
+            for (uint32_t k0 = 0; k0 < nq; k0 += 32) {
+                uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0, d0 = 0, d1 = 0, d2 = 0, d3 = 0;
+                const uint32_t o = k0 * 4;
+#define TM_DPRE(B, g)                                                                                        \
+    precheck4x2<B, kImad>(c0, c1, c2, c3, xa, lds128(pxa + o + 16 * (g)), ya, lds128(pya + o + 16 * (g)), p.one); \
+    precheck4x2<B, kImad>(d0, d1, d2, d3, xb, lds128(pxb + o + 16 * (g)), yb, lds128(pyb + o + 16 * (g)), p.one)
+                const uint32_t left = nq - k0;
+                TM_DPRE(1u << 0, 0);
+                if (left > 4) { TM_DPRE(1u << 4, 1); }
+                if (left > 8) { TM_DPRE(1u << 8, 2); }
+                if (left > 12) { TM_DPRE(1u << 12, 3); }
+                if (left > 16) { TM_DPRE(1u << 16, 4); }
+                if (left > 20) { TM_DPRE(1u << 20, 5); }
+                if (left > 24) { TM_DPRE(1u << 24, 6); }
+                if (left > 28) { TM_DPRE(1u << 28, 7); }
+#undef TM_DPRE
+                const uint32_t qmask = left >= 32 ? ~0u : ((1u << left) - 1u);
+                uint32_t acc_a = va ? ((c0 | c1) | (c2 | c3)) & qmask : 0u;
+                uint32_t acc_b = vb ? ((d0 | d1) | (d2 | d3)) & qmask : 0u;
+                // Alg. 3 on the pairs that passed: all six words, then emit (keys fused, S7)
+                while (__any_sync(0xffffffffu, (acc_a | acc_b) != 0)) {
+                    bool m = false;
+                    uint32_t j = 0, row = ra;
+                    if (acc_a | acc_b) {
+                        const bool isb = acc_a == 0;
+                        uint32_t &acc = isb ? acc_b : acc_a;
+                        j = k0 + (uint32_t)(__ffs(acc) - 1);
+                        acc &= acc - 1;
+                        row = isb ? rb : ra;
+                        const uint64_t s0 = isb ? b0 : a0, s1 = isb ? b1 : a1, s2 = isb ? b2 : a2;
+                        m = (((uint32_t)s0 & ~sm.dp[0][j]) | ((uint32_t)(s0 >> 32) & ~sm.dp[1][j]) |
+                             ((uint32_t)s1 & ~sm.dp[2][j]) | ((uint32_t)(s1 >> 32) & ~sm.dp[3][j]) |
+                             ((uint32_t)s2 & ~sm.dp[4][j]) | ((uint32_t)(s2 >> 32) & ~sm.dp[5][j])) == 0;
+                    }
+                    const uint32_t bm = __ballot_sync(0xffffffffu, m);
+                    if (bm) {
+                        st_matched += __popc(bm);
+                        emit_keys(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane, sm.pend[warp], npend);
+                    }
+                }
+            }
+            st_checks += nq * (vend > u0 ? min((uint32_t)kDenseRows, vend - u0) : 0u);
+        }
+        __syncthreads();
+    }
+    flush_pend(sm.pend[warp], npend, p, lane);
+    if (lane == 0 && (st_checks | st_matched)) {
+        atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
+        atomicAdd(&sm.cnt[2], (unsigned long long)st_matched);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (sm.cnt[1]) atomicAdd(&p.ctr->pair_checks, sm.cnt[1]);
+        if (sm.cnt[2]) atomicAdd(&p.ctr->matched_sets, sm.cnt[2]);
+    }
+}
+
 // ------------------------------------------------------------------ S8 ---
 __global__ void k_split(const uint64_t *__restrict__ pairs, uint64_t n, uint32_t *__restrict__ q,
                         uint32_t *__restrict__ k) {
@@ -1068,11 +1409,11 @@ __global__ void k_word_select(const uint64_t *__restrict__ w0, const uint64_t *_
     wsel[r] = (uint8_t)(best | (second << 4));
 }
 
-struct PopcAt {
-    const uint32_t *bm;
+struct WidenAt {
+    const uint32_t *v;
     uint64_t n;
     __device__ unsigned long long operator()(const uint64_t &i) const {
-        return i < n ? (unsigned long long)__popc(bm[i]) : 0ULL;
+        return i < n ? (unsigned long long)v[i] : 0ULL;
     }
 };
 
@@ -1095,22 +1436,22 @@ cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, co
     return cudaGetLastError();
 }
 
-cudaError_t launch_route_bitmap(const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
-                                const uint64_t *q2, uint64_t n_q, uint32_t *bm, cudaStream_t s) {
-    const uint64_t qw = (n_q + 31) / 32;
-    if (!qw || !n_parts) return cudaSuccess;
-    k_route_bitmap<<<grid_for(qw, kRouteWarps), kRouteWarps * 32, 0, s>>>(masks, n_parts, q0, q1, q2, n_q, bm, qw);
+uint64_t route_blocks(uint64_t n_q) { return (n_q + kRouteBlockQ - 1) / kRouteBlockQ; }
+
+cudaError_t launch_route(int pass, const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
+                         const uint64_t *q2, uint64_t n_q, uint32_t *counts, const unsigned long long *off,
+                         uint32_t *qidx, unsigned long long cap, cudaStream_t s) {
+    const uint64_t nb = route_blocks(n_q);
+    if (!nb || !n_parts) return cudaSuccess;
+    const size_t smem = (size_t)kRouteWarps * 192 * kRouteWB * 4;  // 48 KB: within the default dynamic limit
+    static_assert((size_t)kRouteWarps * 192 * kRouteWB * 4 <= 48 * 1024, "route Z needs the opt-in attribute");
+    auto f = pass == 0 ? k_route<0> : k_route<1>;
+    f<<<grid_for(nb, kRouteWarps), kRouteWarps * 32, smem, s>>>(masks, n_parts, q0, q1, q2, n_q, nb, counts, off, qidx,
+                                                                cap);
     return cudaGetLastError();
 }
 
-cudaError_t launch_route_scatter(const uint32_t *bm, const unsigned long long *word_off, uint64_t n_words,
-                                 uint32_t qw, uint32_t *qidx, unsigned long long cap, cudaStream_t s) {
-    if (!n_words) return cudaSuccess;
-    k_route_scatter<<<grid_for(n_words, 256), 256, 0, s>>>(bm, word_off, n_words, qw, qidx, cap);
-    return cudaGetLastError();
-}
-
-cudaError_t launch_items(const unsigned long long *word_off, uint32_t qw, const uint32_t *part_row,
+cudaError_t launch_items(const unsigned long long *word_off, uint64_t qw, const uint32_t *part_row,
                          const uint32_t *part_n, uint32_t n_parts, unsigned long long *qoff,
                          unsigned long long *item_cnt, DevCounters *ctr, uint32_t range_rows, cudaStream_t s) {
     k_items<<<grid_for((uint64_t)n_parts + 1, 256), 256, 0, s>>>(word_off, qw, part_row, part_n, n_parts, qoff,
@@ -1131,13 +1472,20 @@ ScanFn scan_fn(int variant) {
         case 5: return k_scan<4, false, false, true, 7>;
         case 6: return k_scan<4, false, false, false, 8, true>;  // streaming only, direct check
         case 7: return k_scan<4, false, false, true, 8, true>;   // streaming only, word pre-check
+        case 8: return k_scan<4, false, false, true, 7, false, 1>;  // 5 + pre-check accumulate on the FMA pipe
+        case 9: return k_dense<false, 1>;   // unfiltered dense scan, direct loads, FMA-pipe accumulate
+        case 10: return k_dense<true, 1>;   // unfiltered dense scan, bulk-copy (TMA) staged rows
+        case 11: return k_dense<false, 0>;
+        case 12: return k_dense<true, 0>;
         default: return k_scan<4, false>;
     }
 }
 }  // namespace
 
 size_t scan_smem(int variant) {
-    return variant >= 6 ? sizeof(StreamSmem) : sizeof(ScanSmem);
+    if (variant == 9 || variant == 11) return sizeof(DenseSmemBase);
+    if (variant == 10 || variant == 12) return sizeof(DenseSmemBulk);
+    return (variant == 6 || variant == 7) ? sizeof(StreamSmem) : sizeof(ScanSmem);
 }
 
 int scan_variant_env() {
@@ -1221,12 +1569,12 @@ cudaError_t launch_iota(uint32_t *v, uint64_t n, cudaStream_t s) {
 }
 
 // ----------------------------------------------------------------- CUB ---
-cudaError_t cub_exclusive_popc_scan(const uint32_t *bm, unsigned long long *out, uint64_t n, void *tmp,
-                                    size_t *tmp_bytes, cudaStream_t s) {
-    // out[0..n] = exclusive prefix of popc(bm[i]); out[n] = total
+cudaError_t cub_exclusive_scan_u32_u64(const uint32_t *in, unsigned long long *out, uint64_t n, void *tmp,
+                                      size_t *tmp_bytes, cudaStream_t s) {
+    // out[0..n] = exclusive prefix of in[0..n) widened to 64 bits; out[n] = total
     cub::CountingInputIterator<uint64_t> cnt(0);
-    cub::TransformInputIterator<unsigned long long, PopcAt, cub::CountingInputIterator<uint64_t>> it(cnt,
-                                                                                                    PopcAt{bm, n});
+    cub::TransformInputIterator<unsigned long long, WidenAt, cub::CountingInputIterator<uint64_t>> it(cnt,
+                                                                                                     WidenAt{in, n});
     return cub::DeviceScan::ExclusiveSum(tmp, *tmp_bytes, it, out, (int64_t)(n + 1), s);
 }
 

@@ -39,7 +39,12 @@ def main():
         db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=tmb.TM_NO_PARTITIONING, tile_filter=filt)
         build_s = time.time() - t0
         rows = db.stats()["n_rows"]
-        for B in [int(x) for x in os.environ.get("HBM_B", "1,2,4,8,16,32,64,128,256").split(",")]:
+        for B, var in [(int(b), v) for b in os.environ.get("HBM_B", "1,2,4,8,16,32,64,128,256").split(",")
+                       for v in os.environ.get("HBM_VARIANTS", "auto").split(",")]:
+            if var == "auto":
+                os.environ.pop("TM_SCAN_VARIANT", None)
+            else:
+                os.environ["TM_SCAN_VARIANT"] = var
             q = wl.queries.subset(np.arange(B))
             arrs = [np.ascontiguousarray(a) for a in (q.vocab_bytes, q.vocab_off.view(np.int64),
                                                       q.tag_idx.view(np.int32), q.set_off.view(np.int64))]
@@ -68,7 +73,7 @@ def main():
                 gq, gk = db.match_batch(q, False)
                 wq, wk = o2.match_brute(db_sig, wl.key_off, wl.keys, o2.encode(q), False)
                 ok = bool(np.array_equal(gq, wq) and np.array_equal(gk, wk))
-            print(json.dumps({"B": B, "tile_filter": filt, "n_sets": n_sets, "rows": rows, "scan_ms": ms,
+            print(json.dumps({"B": B, "forced": var, "tile_filter": filt, "n_sets": n_sets, "rows": rows, "scan_ms": ms,
                               "table_gbs": gbs, "frac_of_measured_hbm": gbs / hbm,
                               "pair_checks": st["pair_checks"], "tile_tests": st["tile_tests"],
                               "checks_per_s": st["pair_checks"] / (ms / 1e3), "parity": ok,
