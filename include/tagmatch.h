@@ -57,6 +57,11 @@ extern "C" {
 /* max_partition value meaning "no partitioning": one partition with the empty
  * mask, routed to every query (reading R8; BASELINE config C1). */
 #define TM_NO_PARTITIONING 0xFFFFFFFFu
+/* max_partition value meaning "choose MAX_P from the database size": clamp(n_sets / 10^4,
+ * 5,000, 200,000) (reading R8b: the paper's optimum of ~200K
+ * comes from its CPU pipeline's per-partition cost; with the bit-sliced GPU router the
+ * measured optimum is ~10^4 partitions: C2 best at 5K, C3 at 10K). */
+#define TM_AUTO_MAX_PARTITION 0xFFFFFFFEu
 
 typedef struct tm_db tm_db; /* opaque, owned by the library */
 
@@ -243,6 +248,8 @@ typedef struct {
     uint64_t xchg_recv_bytes;  /* ... and received from them                                      */
     double xchg_ms;            /* CUDA-event time of count all-gather + exchange + owner merge    */
     double local_ms;           /* CUDA-event time of the local S1-S8 part of a sharded call        */
+    uint32_t max_partition;    /* MAX_P the database was partitioned with (TM_AUTO_MAX_PARTITION resolved) */
+    uint32_t n_gpus;           /* GPUs behind the handle (1, or n_gpus of an in-process multi-GPU database) */
 } tm_stats_t;
 
 tm_status tm_stats(const tm_db *db, tm_stats_t *out);

@@ -6,4 +6,4 @@ thin ctypes binding (tagmatch.py).  Every step of the matching path runs in the
 library's sm_100a kernels; there is no CPU fallback.
 """
 from .tagmatch import (Database, HostTagSets, TagMatchError, abi_version, device_tagsets, encode, load,  # noqa: F401
-                       TM_DEFAULT_MAX_PARTITION, TM_NO_PARTITIONING, EXPORTS, LIB_PATH)
+                       TM_DEFAULT_MAX_PARTITION, TM_NO_PARTITIONING, TM_AUTO_MAX_PARTITION, EXPORTS, LIB_PATH)

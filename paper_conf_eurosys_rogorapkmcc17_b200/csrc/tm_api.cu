@@ -151,17 +151,25 @@ void *cub_tmp(tm_db *db, size_t bytes) {
 }
 
 // Run the whole path for device-resident queries; leaves n results in db->res_q/res_k.
-uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) {
+// Every query of the batch is encoded; queries [qlo, qlo + qn) are matched (the share of one GPU
+// of a replicated multi-GPU database; default: all), with their batch-global indices.
+uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, uint64_t qlo, uint64_t qn) {
     tm_stats_t &st = db->st;
-    const uint64_t Q = q->n_sets;
+    const uint64_t Qall = q->n_sets;
+    if (qlo > Qall) qlo = Qall;
+    if (qn > Qall - qlo) qn = Qall - qlo;
+    const uint64_t Qm = qn;                        // queries matched
     const uint32_t P = (uint32_t)db->n_parts;
     std::memset(&st.n_queries, 0, sizeof(tm_stats_t) - offsetof(tm_stats_t, n_queries));
-    st.n_queries = Q;
+    st.n_queries = Qm;
     db->last_sorted = nullptr;
     db->last_n = 0;
-    db->last_Q = Q;
-    if (Q == 0 || P == 0) return 0;
-    const uint64_t NB = route_blocks(Q);          // route blocks of 512 queries
+    db->last_Q = Qall;
+    db->last_qlo = qlo;
+    db->last_qn = Qm;
+    if (Qm == 0 || P == 0) return 0;
+    const uint64_t Q = Qall;                       // encoded (and the sort width)
+    const uint64_t NB = route_blocks(Qm);          // route blocks of 512 queries
     const uint64_t n_words = (uint64_t)P * NB;    // (partition, route block) counts
     uint32_t launches = 0, cub_calls = 0;
 
@@ -193,7 +201,8 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
     // offsets of a partition-major CSR of ascending query ids
     db->bm.ensure(n_words * 4);
     db->word_off.ensure((n_words + 1) * 8);
-    TMCK(launch_route(0, db->masks.as<uint64_t>(), P, q0, q1, q2, Q, db->bm.as<uint32_t>(), nullptr, nullptr, 0, s));
+    TMCK(launch_route(0, db->masks.as<uint64_t>(), P, q0 + qlo, q1 + qlo, q2 + qlo, Qm, db->bm.as<uint32_t>(), nullptr,
+                      nullptr, 0, s));
     launches++;
     size_t tb = 0;
     TMCK(cub_exclusive_scan_u32_u64(db->bm.as<uint32_t>(), db->word_off.as<unsigned long long>(), n_words, nullptr,
@@ -204,15 +213,16 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
     db->qoff.ensure((uint64_t)(P + 1) * 8);
     db->item_cnt.ensure((uint64_t)(P + 1) * 8);
     db->item_off.ensure((uint64_t)(P + 1) * 8);
-    if (db->cap_qidx == 0) db->cap_qidx = std::max<unsigned long long>(Q * 32, 1 << 16);
-    if (db->cap_out == 0) db->cap_out = std::max<unsigned long long>(Q * 32, 1 << 16);
+    if (db->cap_qidx == 0) db->cap_qidx = std::max<unsigned long long>(Qm * 32, 1 << 16);
+    if (db->cap_out == 0) db->cap_out = std::max<unsigned long long>(Qm * 32, 1 << 16);
 
     for (int attempt = 0;; ++attempt) {
         db->qidx.ensure(db->cap_qidx * 4);
         db->out.ensure(db->cap_out * 8);
         TMCK(cudaMemsetAsync(ctr, 0, offsetof(DevCounters, input_err), s));
-        TMCK(launch_route(1, db->masks.as<uint64_t>(), P, q0, q1, q2, Q, nullptr,
-                          db->word_off.as<unsigned long long>(), db->qidx.as<uint32_t>(), db->cap_qidx, s));
+        TMCK(launch_route(1, db->masks.as<uint64_t>(), P, q0 + qlo, q1 + qlo, q2 + qlo, Qm, nullptr,
+                          db->word_off.as<unsigned long long>(), db->qidx.as<uint32_t>(), db->cap_qidx, s,
+                          (uint32_t)qlo));
         // S3: per-partition batches -> work items
         const uint32_t range_rows = range_rows_env(db->n_rows);
         TMCK(launch_items(db->word_off.as<unsigned long long>(), NB, db->part_row.as<uint32_t>(),
@@ -253,6 +263,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         sp.wsel = db->wsel.as<uint8_t>();
         sp.range_rows = range_rows;
         sp.one = 1;
+        sp.pmask = db->masks.as<uint64_t>();
         // variant: TM_SCAN_VARIANT if set; else a call whose partition batches are all small
         // (Q <= kSmallBatch) takes the streaming path only, in the streaming-only kernels (small
         // shared memory: 8 CTAs/SM) -- up to four queries checked directly (variant 6), 5-8
@@ -262,17 +273,17 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s) 
         const int forced = scan_variant_env();
         int var = forced;
         // the streaming-only kernels cannot take a filtered batch: a forced 6 / 7 maps to 0 / 5 then
-        if ((var == 6 || var == 7) && Q > (uint64_t)kSmallBatch) var = var == 6 ? 0 : 5;
+        if ((var == 6 || var == 7) && Qm > (uint64_t)kSmallBatch) var = var == 6 ? 0 : 5;
         db->call_tunes = false;
         if (var < 0) {
-            if (Q <= (uint64_t)kSmallBatch) {
-                var = Q <= 4 ? 6 : 7;
+            if (Qm <= (uint64_t)kSmallBatch) {
+                var = Qm <= 4 ? 6 : 7;
             } else {
-                const int c = 63 - __builtin_clzll(Q);
+                const int c = 63 - __builtin_clzll(Qm);
                 db->call_class = c;
                 // batches below kTuneMinQ queries keep the default variant: a tuning round there
                 // would put slow candidates into a latency-bound stream for little gain
-                if (Q >= (uint64_t)kTuneMinQ && db->tune_calls[c] < 2 * kTuneN) {
+                if (Qm >= (uint64_t)kTuneMinQ && db->tune_calls[c] < 2 * kTuneN) {
                     var = db->tune[db->tune_calls[c] % kTuneN];
                     db->call_tunes = true;
                 } else {
@@ -455,6 +466,8 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
     if (K > 0 && !keys) fail(TM_EINVAL, "keys is NULL");
     db->n_sets = N;
     db->n_entries = K;
+    if (db->cfg.max_partition == TM_AUTO_MAX_PARTITION)  // reading R8b: ~10^4 partitions
+        db->cfg.max_partition = (uint32_t)std::min<uint64_t>(200000, std::max<uint64_t>(5000, N / 10000));
 
     // S0a: encode every set on the GPU
     DevBuf d_bytes, d_voff, d_tidx, d_soff, d_vsig, d_planes, d_sorted, d_idx, d_idx2, d_key, d_key2;
@@ -827,7 +840,7 @@ tm_status tm_match_batch_csr(tm_db *db, const tm_tagsets *q, int unique, tm_csr 
     const uint64_t Q = q->n_sets;
     db->res_off.ensure((Q + 1) * 8);
     const uint64_t *sorted = n ? db->last_sorted : nullptr;
-    TMCK(launch_query_offsets(sorted, n, Q, db->res_off.as<uint64_t>(), s));
+    TMCK(launch_query_offsets(sorted, n, 0, Q, 0, db->res_off.as<uint64_t>(), s));
     PinnedBlock *blk = pinned_get((Q + 1) * 8 + std::max<uint64_t>(n, 1) * 4);
     uint64_t *hoff = static_cast<uint64_t *>(blk->p);
     uint32_t *hk = reinterpret_cast<uint32_t *>(hoff + Q + 1);
@@ -953,6 +966,8 @@ tm_status tm_stats(const tm_db *db, tm_stats_t *out) {
     out->n_partitions = db->n_parts;
     out->n_partitions_total = db->n_parts_total;
     out->build_ms = db->build_ms;
+    out->max_partition = db->cfg.max_partition;
+    out->n_gpus = 1;
     return TM_OK;
     TM_API_END
 }

@@ -145,6 +145,7 @@ struct tm_db {
     // last call's merged result before the split (sorted (q<<32|key)), for the shard exchange
     uint64_t *last_sorted = nullptr;
     uint64_t last_n = 0, last_Q = 0;
+    uint64_t last_qlo = 0, last_qn = 0;  // the query range the last call matched
     // shard layer (tm_shard.cu)
     void *nccl_comm = nullptr;
     int nranks = 1, rank = 0;
@@ -158,7 +159,8 @@ struct tm_db {
 
 namespace tmb {
 void *cub_tmp(tm_db *db, size_t bytes);
-uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s);
+uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, uint64_t qlo = 0,
+                    uint64_t qn = ~0ULL);
 void finish_timing(tm_db *db, cudaStream_t s);
 tm_status translate(const CudaFail &f);
 int check_device(int dev);

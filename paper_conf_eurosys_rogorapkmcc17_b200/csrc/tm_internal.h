@@ -28,7 +28,7 @@ constexpr int kScanWarps = 4;      // warps per CTA
 constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch); 640 fits 7 CTAs/SM of shared memory and measured 1.3% faster than 512 (profiles/r1v34_ab.txt)
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
-constexpr int kScanVariants = 13;    // k_scan variants (TM_SCAN_VARIANT)
+constexpr int kScanVariants = 15;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {5, 0};  // variants the handle times on its first calls (first = default); 2 never won
 constexpr int kTuneN = 2;
 constexpr int kTuneDense[] = {10, 9};  // tables without a pre-filter (tile_filter = 2): the dense scan
@@ -67,6 +67,7 @@ struct ScanParams {
     const uint8_t *wsel;              // [rows] pre-check word per row (variant 5)
     uint32_t range_rows;              // rows per work item (multiple of 256)
     uint32_t one;                     // 1 (a run-time operand, so the FMA-pipe accumulate stays an IMAD)
+    const uint64_t *pmask;            // [P][3] partition masks (bits every routed query contains)
 };
 
 // ------------------------------------------------------------ launchers --
@@ -81,7 +82,7 @@ cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, co
 uint64_t route_blocks(uint64_t n_q);
 cudaError_t launch_route(int pass, const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
                          const uint64_t *q2, uint64_t n_q, uint32_t *counts, const unsigned long long *off,
-                         uint32_t *qidx, unsigned long long cap, cudaStream_t s);
+                         uint32_t *qidx, unsigned long long cap, cudaStream_t s, uint32_t qbase = 0);
 cudaError_t launch_items(const unsigned long long *word_off, uint64_t qw, const uint32_t *part_row,
                          const uint32_t *part_n, uint32_t n_parts, unsigned long long *qoff,
                          unsigned long long *item_cnt, DevCounters *ctr, uint32_t range_rows, cudaStream_t s);
@@ -92,7 +93,9 @@ int scan_variant_env();  // -1 = auto-tune
 cudaError_t launch_word_select(const uint64_t *planes, const uint64_t *tand, uint64_t rows, uint8_t *wsel,
                                cudaStream_t s);
 cudaError_t launch_split(const uint64_t *pairs, uint64_t n, uint32_t *q, uint32_t *k, cudaStream_t s);
-cudaError_t launch_query_offsets(const uint64_t *pairs, uint64_t n, uint64_t Q, uint64_t *q_off, cudaStream_t s);
+// q_off[i] = base + (first pair of query qlo + i), i < nq; q_off[nq] = base + n
+cudaError_t launch_query_offsets(const uint64_t *pairs, uint64_t n, uint64_t qlo, uint64_t nq, uint64_t base,
+                                 uint64_t *q_off, cudaStream_t s);
 cudaError_t launch_gather_planes(const uint64_t *src0, const uint64_t *src1, const uint64_t *src2,
                                  const uint32_t *idx, uint64_t n, uint64_t *d0, uint64_t *d1, uint64_t *d2,
                                  cudaStream_t s);

@@ -194,6 +194,8 @@ tm_status tm_partition_host(const uint64_t *sigs, uint64_t n, uint32_t max_parti
     TM_API_BEGIN
     if ((n && !sigs) || !masks_out || !sizes_out || !n_parts_out || !n_unique_out) fail(TM_EINVAL, "NULL argument");
     if (max_partition == 0) max_partition = TM_DEFAULT_MAX_PARTITION;
+    if (max_partition == TM_AUTO_MAX_PARTITION)  // reading R8b, as tm_build
+        max_partition = (uint32_t)std::min<uint64_t>(200000, std::max<uint64_t>(5000, n / 10000));
     std::vector<Sig> v(n);
     for (uint64_t i = 0; i < n; ++i) v[i] = Sig{{sigs[3 * i], sigs[3 * i + 1], sigs[3 * i + 2]}};
     auto lt = [](const Sig &a, const Sig &b) {

@@ -19,6 +19,7 @@ LIB_PATH = os.path.join(_PKG, "libtagmatch.so")
 
 TM_DEFAULT_MAX_PARTITION = 200_000
 TM_NO_PARTITIONING = 0xFFFFFFFF
+TM_AUTO_MAX_PARTITION = 0xFFFFFFFE
 STATUS = {0: "TM_OK", -1: "TM_EINVAL", -2: "TM_ENOMEM", -3: "TM_ECUDA", -4: "TM_ENCCL", -5: "TM_ERANGE",
           -6: "TM_ESTATE"}
 
@@ -79,7 +80,8 @@ class tm_stats_t(ctypes.Structure):
                 ("exact_checked", ctypes.c_uint64), ("exact_kept", ctypes.c_uint64),
                 ("scan_variant", ctypes.c_uint32), ("tuning", ctypes.c_uint32),
                 ("xchg_send_bytes", ctypes.c_uint64), ("xchg_recv_bytes", ctypes.c_uint64),
-                ("xchg_ms", ctypes.c_double), ("local_ms", ctypes.c_double)]
+                ("xchg_ms", ctypes.c_double), ("local_ms", ctypes.c_double),
+                ("max_partition", ctypes.c_uint32), ("n_gpus", ctypes.c_uint32)]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
