@@ -20,11 +20,14 @@ hbm    : (N = 1) the subset scan of the whole table as ONE partition, pre-filter
          copy bandwidth (the BASELINE metric's "subset-scan HBM GB/s vs roofline").
 roofline: the dominant kernel (k_scan) against the INT/logic-pipe peak measured on
          this box by build/int_peak (scripts/int_peak.cu), SURVEY 8(d) ops model.
-N > 1  : one process per GPU (torchrun).  Default: the database is partition-sharded
-         over the ranks: every rank matches the same batch against
-         its partitions and the pairs go to query owners over NCCL
-         (tm_match_batch_sharded_device) -> "scaling": "strong".  --replicated: every
-         rank holds the whole database and matches its own batch -> "weak".
+N > 1  : one process per GPU (torchrun), the same batch on every rank, "scaling": "strong".
+         Default: the database is partition-sharded over the ranks (plan
+         weighted by a routed 10K-query sample): every rank matches the batch against its
+         partitions and the pairs go to query owners over NCCL (tm_match_batch_sharded_device).
+         --replicated: every rank holds the whole database and matches its owner range of the
+         batch, no exchange (NEXT-1; the library's TM_SHARD_REPLICATED).
+MAX_P  : auto (TM_AUTO_MAX_PARTITION: clamp(N / 10^4, 5K, 200K), R8b) unless
+         --max-partition N (--max-partition 200000 = the paper's value).
 --impl reference : the oracle (oracle/o2.c, the paper's CPU method) on the
          host cores, on a bounded sample of the same workload per step.
 """
@@ -125,13 +128,21 @@ def load_workload(name: str, rank: int = 0):
     """BASELINE config `name`; rank r > 0 matches its own query batch (query seed + 7919 r)."""
     import tmgen
     if name in tmgen.CRAFTED:  # sec. 4.4 crafted workloads (PAPER.md:391-399)
-        c = dict(tmgen.CRAFTED[name], max_partition=getattr(load_workload, "max_partition", 0) or 200_000, total_tags=0)
+        mp = getattr(load_workload, "max_partition", -1)
+        c = dict(tmgen.CRAFTED[name], max_partition=0xFFFFFFFE if mp == -1 else (mp or 200_000), total_tags=0,
+                 oracle_max_partition=200_000)
+        c["resolved_max_partition"] = min(200_000, max(5_000, c["n_sets"] // 10_000))
         wl = tmgen.config(name, max_partition=c["max_partition"],
                           query_seed=c["seed"] + (1 << 32) + 7919 * rank)
         return wl, c
     c = dict(tmgen.CONFIGS[name])
-    if getattr(load_workload, "max_partition", 0):
-        c["max_partition"] = load_workload.max_partition
+    c["oracle_max_partition"] = c["max_partition"]   # O2's own MAX_P (the paper's 200K)
+    mp = getattr(load_workload, "max_partition", -1)
+    if mp == -1:
+        c["max_partition"] = 0xFFFFFFFE   # TM_AUTO_MAX_PARTITION
+        c["resolved_max_partition"] = min(200_000, max(5_000, c["n_sets"] // 10_000))  # the library's rule
+    elif mp:
+        c["max_partition"] = mp
     wl = tmgen.generate(c["n_sets"], c["n_queries"], c["seed"], total_tags=c["total_tags"],
                         max_partition=c["max_partition"], name=name,
                         query_seed=(c.get("query_seed") or c["seed"] + (1 << 32)) + 7919 * rank)
@@ -147,7 +158,7 @@ def oracle_rate(wl, c, unique: bool, target_s: float = 8.0, max_q: int | None = 
     q_sig = o2.encode(wl.queries)
     t0 = time.perf_counter()
     if c["n_sets"] <= 20_000_000:
-        ix = o2.Index(db_sig, c["max_partition"])
+        ix = o2.Index(db_sig, c.get("oracle_max_partition", 200_000))
     else:
         # O2's single-threaded Alg. 1 takes minutes beyond ~20M sets (213 s at 100M):
         # the baseline is then O2's brute-force scan on all cores
@@ -205,11 +216,11 @@ def run_reference(args):
             "data": ("synthetic (seeded sec. 4.4 crafted workload, tmgen.generate_crafted, PAPER.md:391-399)"
                      if args.config.startswith(("C6", "C7")) else
                      "synthetic (seeded Twitter-like generator tmgen, PAPER.md:258-282)"),
-            "config": config_block(c, args, wl, args.gpus > 1 and not args.replicated),
+            "config": config_block(c, args, wl, args.gpus > 1),
             "cpu_baseline": {"value": value, "unit": "queries/s", "cores": cores, "kind": "oracle",
                              "sample": f"{size} of {q_sig.shape[0]} queries per step ("
                                        + (f"O2 brute force over {c['n_sets']} sets" if isinstance(ix, _BruteOracle)
-                                          else f"O2: Alg.1 MAX_P={c['max_partition']} + Alg.2 + linear scan; "
+                                          else f"O2: Alg.1 MAX_P={c.get('oracle_max_partition')} + Alg.2 + linear scan; "
                                                f"Alg.1 build {build_s:.1f} s excluded") + ")"},
             "e2e": {"value": value, "unit": "queries/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -220,12 +231,15 @@ def config_block(c, args, wl, sharded=False):
             "query_tags": (f"{c['set_tags']}-tag DB sets, {c['query_tags']}-tag queries (PAPER.md:391-399)"
                            if "set_tags" in c else
                            "base set + 2..4 extra" if not c["total_tags"] else f"total {c['total_tags']}"),
-            "max_partition": c["max_partition"], "mode": "match-unique" if args.unique else "match",
+            "max_partition": (f"auto: clamp(N/1e4, 5000, 200000) = {c['resolved_max_partition']}"
+                              if c["max_partition"] == 0xFFFFFFFE else c["max_partition"]),
+            "mode": "match-unique" if args.unique else "match",
             "tile_filter": ["alg4-prefix", "tile-and", "none"][args.tile_filter],
             "row_order": ["lexicographic", "balanced-splits"][args.row_order],
             "exact_check": bool(args.exact),
-            "parallelism": (f"partition-sharded-{args.gpus} (NCCL exchange)" if sharded else
-                            f"replicated-dp{args.gpus}") if args.gpus > 1 else "single",
+            "parallelism": (f"replicated-{args.gpus} (each rank: owner range of the batch, whole table)"
+                            if args.replicated else f"partition-sharded-{args.gpus} (NCCL exchange)")
+                           if args.gpus > 1 else "single",
             "l2": "flushed between timed steps (512 MiB write)", "bloom": "192 bits, k=7 (PAPER.md:106)"}
 
 
@@ -369,9 +383,11 @@ def run_ours(args):
     import paper_conf_eurosys_rogorapkmcc17_b200 as tmb
     from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as tmx
 
-    sharded = world > 1 and not args.replicated
-    # replicated mode: every rank its own batch; sharded mode: the same batch on every rank
-    wl, c = load_workload(args.config, 0 if sharded else rank)
+    # N > 1: one batch on every rank; partitioned (default) or replicated database (library
+    # shard_mode: each rank matches its owner range of the batch against the whole table)
+    sharded = world > 1
+    mode = tmx.TM_SHARD_REPLICATED if args.replicated else tmx.TM_SHARD_PARTITIONED
+    wl, c = load_workload(args.config, 0)
     unique = bool(args.unique)
     Q = wl.queries.n_sets
     peaks, peak_src = measured_peaks()
@@ -389,13 +405,17 @@ def run_ours(args):
     torch.cuda.synchronize(dev)
     mem0 = (torch.cuda.mem_get_info(dev)[0], torch.cuda.memory_reserved(dev))
     t0 = time.perf_counter()
+    # the shard plan weighs partitions by the routing of a 10K-query sample of the stream
+    sample = wl.queries.subset(np.arange(min(10_000, Q))) if sharded else None
     db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], device=dev,
                       tile_filter=args.tile_filter, row_order=args.row_order, exact=int(args.exact),
-                      n_shards=world if sharded else 1, shard=rank if sharded else 0)
+                      n_shards=world if sharded else 1, shard=rank if sharded else 0, shard_mode=mode,
+                      plan_sample=sample)
     build_s = time.perf_counter() - t0
+    c["resolved_max_partition"] = db.stats()["max_partition"]
     torch.cuda.synchronize(dev)
     mem1 = (torch.cuda.mem_get_info(dev)[0], torch.cuda.memory_reserved(dev))
-    if sharded:
+    if sharded and mode == tmx.TM_SHARD_PARTITIONED:
         uid = [tmx.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
         db.comm_init(uid[0], world, rank)
@@ -466,7 +486,7 @@ def run_ours(args):
         t = torch.tensor([t_local], device=cdev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         t_max = float(t.item())
-    value = (1 if sharded else world) * Q * args.steps / t_max
+    value = Q * args.steps / t_max
     scan_ms = [s["scan_ms"] for s in stats]
 
     # per-rank view (sharded: scan time, exchange, imbalance)
@@ -504,7 +524,7 @@ def run_ours(args):
         t = torch.tensor([e2e_local], device=cdev, dtype=torch.float64)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         e2e_local = float(t.item())
-    e2e_value = (1 if sharded else world) * Q * args.steps / e2e_local
+    e2e_value = Q * args.steps / e2e_local
 
     mem = memory_block(db, mem0, mem1, dev)
     db.close()
@@ -573,7 +593,7 @@ def run_ours(args):
                                     "sample": f"{size} of {Q} queries (" +
                                               (f"O2 brute force over {c['n_sets']} sets, {o2.threads(0)} threads"
                                                if isinstance(ix, _BruteOracle) else
-                                               f"O2: Alg.1 MAX_P={c['max_partition']} + Alg.2 + linear scan, "
+                                               f"O2: Alg.1 MAX_P={c.get('oracle_max_partition')} + Alg.2 + linear scan, "
                                                f"{o2.threads(0)} threads; Alg.1 build {obuild:.1f} s excluded") + ")"}
         print(json.dumps(line), flush=True)
     if world > 1:
@@ -656,8 +676,9 @@ def main():
                     help="exact subset post-check (PAPER.md:106; removes Bloom false positives)")
     ap.add_argument("--row-order", type=int, default=1, choices=[0, 1],
                     help="1: balanced-split order inside partitions (DESIGN.md R18; needs --tile-filter 1)")
-    ap.add_argument("--max-partition", type=int, default=0,
-                    help="override the config's MAX_P (PAPER.md:361-371 sweep); 0 = config value")
+    ap.add_argument("--max-partition", type=int, default=-1,
+                    help="MAX_P (PAPER.md:361-371 sweep): -1 = auto (TM_AUTO_MAX_PARTITION, default), "
+                         "0 = the config's (the paper's 200K), N = N")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-s", type=float, default=10.0, help="seconds of oracle work for cpu_baseline")
     ap.add_argument("--ref-step-s", type=float, default=4.0, help="seconds per --impl reference step")

@@ -126,8 +126,30 @@ typedef struct {
                                kept only if every tag string of the entry's set occurs in
                                the query, which removes Bloom false positives; 0 = the
                                Bloom result (default)                                  */
+    uint32_t n_gpus;        /* in-process multi-GPU database (one process drives several GPUs,
+                               no launcher needed; sec. "Multi-GPU"): 0/1 = one device
+                               (`device`); k > 1 = k sub-databases on device_ids[0..k)  */
+    uint32_t shard_mode;    /* how a multi-GPU database uses its GPUs (n_gpus > 1, or one process
+                               per GPU with n_shards > 1): TM_SHARD_PARTITIONED (default) or
+                               TM_SHARD_REPLICATED (see below)                          */
     uint32_t reserved;      /* must be 0                                               */
+    const int32_t *device_ids; /* n_gpus device ordinals, or NULL for 0 .. n_gpus-1; a device may
+                               repeat (several sub-databases on one GPU: functional testing) */
+    const tm_tagsets *plan_sample; /* optional host query sample (e.g. 10K queries of the expected
+                               stream) for the partition -> shard plan: partition p
+                               weighs |P_p| x (sample queries routed to p); NULL: |P_p| x 4^-|mask_p| */
 } tm_config;
+
+/* shard_mode values.
+ * TM_SHARD_PARTITIONED: the partitions are split into contiguous ranges of the partition table
+ *   of ~equal estimated work, one per GPU ("partition an extremely large tagset
+ *   table on multiple GPUs"); every GPU matches the whole batch against its partitions and the
+ *   (query, key) pairs are exchanged so that GPU g holds the queries of owner range g
+ *   (tm_owner_range), where they are merged (sorted / de-duplicated).
+ * TM_SHARD_REPLICATED: every GPU holds the whole table and matches owner range g of the batch;
+ *   no exchange ("maximal inter-GPU parallelism in the case of full replication"). */
+#define TM_SHARD_PARTITIONED 0u
+#define TM_SHARD_REPLICATED 1u
 
 /* Result pairs in host memory, allocated by the library (pinned), released by
  * tm_pairs_free().  query[i] is a 0-based index into the call's query batch. */
@@ -281,11 +303,23 @@ tm_status tm_partition_sigs(const tm_db *db, uint64_t p, uint64_t *sig_out);
 /* Query owner ranges: owner g holds queries [floor(Q*g/G), floor(Q*(g+1)/G)). Host only. */
 tm_status tm_owner_range(uint64_t n_queries, uint32_t n_owners, uint32_t owner, uint64_t *lo, uint64_t *hi);
 
-/* Partition -> shard plan (host only, deterministic): greedy longest-processing-
- * time over the estimated work |P| * 4^-|mask|.  masks: n_parts*3 words,
- * sizes: n_parts set counts, owner_out: n_parts shard ids. */
-tm_status tm_shard_plan(const uint64_t *masks, const uint64_t *sizes, uint64_t n_parts, uint32_t n_shards,
-                        uint32_t *owner_out);
+/* Partition -> shard plan (host only, deterministic): the partitions, in table
+ * order, are cut into n_shards contiguous ranges of ~equal estimated work w_p = sizes[p] x
+ * routed[p] (routed[p] = sample queries routed to p), or, with routed NULL or all zero,
+ * w_p = sizes[p] x 4^-|mask_p| (a mask bit is in a query with probability ~1/4).  Partition p
+ * goes to the shard whose share of the total work contains the middle of p's work.
+ * masks: n_parts*3 words, sizes: n_parts set counts, routed: n_parts or NULL,
+ * owner_out: n_parts shard ids (non-decreasing). */
+tm_status tm_shard_plan(const uint64_t *masks, const uint64_t *sizes, const uint64_t *routed, uint64_t n_parts,
+                        uint32_t n_shards, uint32_t *owner_out);
+
+/* Exchange plan of one rank (host only): counts[s * n_ranks + d] = pairs rank s holds for owner
+ * d (the all-gathered count matrix).  send_off[0..n_ranks]: where this rank's pairs for owner d
+ * start in its sorted local result (prefix over d of counts[rank][d]); recv_off[0..n_ranks]:
+ * where pairs from source s land in this rank's receive buffer (prefix over s of
+ * counts[s][rank]); send_off[n_ranks] / recv_off[n_ranks] = totals. */
+tm_status tm_exchange_plan(const uint64_t *counts, uint32_t n_ranks, uint32_t rank, uint64_t *send_off,
+                           uint64_t *recv_off);
 
 /* Algorithm 1 on the host (test hook, no GPU): signatures sigs[n*3] (any
  * order, duplicates allowed) are sorted and de-duplicated, then partitioned
@@ -310,6 +344,18 @@ tm_status tm_shard_counts(tm_db *db, uint32_t n_owners, uint64_t *counts_out);
 tm_status tm_shard_merge(tm_db *db, const uint64_t *pairs, uint64_t n, uint64_t n_queries, int unique,
                          tm_dev_pairs *out, void *stream);
 
+/* In-process multi-GPU databases (tm_config.n_gpus > 1).  tm_build builds one sub-database per
+ * device (in parallel, one host thread each); tm_match_batch / tm_match_batch_csr run the batch
+ * on all of them and return one result, sorted by (query, key) as always; the exchange of a
+ * partitioned database is peer-to-peer copies between the GPUs (cudaMemcpyPeerAsync over
+ * NVLink; peer access is enabled at build), the per-owner merge runs on the owner's GPU.
+ * tm_stats sums the counters and takes the maximum of the times over the GPUs.  Calls taking
+ * device pointers (tm_match_batch_device, the shard hooks) return TM_ESTATE on such a handle.
+ * tm_group_size: number of sub-databases (1 for a single-GPU handle); tm_group_member: the
+ * read-only sub-database g (for tm_stats / tm_partitions; owned by the group). */
+tm_status tm_group_size(const tm_db *db, uint32_t *n);
+tm_status tm_group_member(const tm_db *db, uint32_t g, const tm_db **sub);
+
 /* NCCL communicator of a shard handle.  id: 128 bytes from tm_nccl_unique_id
  * on one rank, distributed by the caller (e.g. torch.distributed). */
 tm_status tm_nccl_unique_id(void *id_out, uint64_t len);
@@ -317,7 +363,9 @@ tm_status tm_comm_init(tm_db *db, const void *id, uint64_t len, int nranks, int 
 
 /* match / match-unique of a batch resident in device memory (the same batch on
  * every rank) against this rank's partitions, exchanged over NCCL: *out holds
- * this rank's owner slice of the global sorted result (query ids global). */
+ * this rank's owner slice of the global sorted result (query ids global).
+ * shard_mode TM_SHARD_REPLICATED (every rank holds the whole table): the rank matches
+ * only its owner range of the batch, no exchange and no communicator needed. */
 tm_status tm_match_batch_sharded_device(tm_db *db, const tm_tagsets *queries, int unique, tm_dev_pairs *out,
                                         void *stream);
 

@@ -28,10 +28,6 @@ void set_error(const std::string &msg) { g_err = msg; }
 
 
 // -------------------------------------------- pinned host result blocks --
-struct PinnedBlock {
-    void *p;
-    size_t cap;
-};
 std::mutex g_pin_mu;
 std::multimap<size_t, void *> g_pin_cache;
 size_t g_pin_cached = 0;
@@ -414,32 +410,6 @@ tm_status translate(const CudaFail &f) {
     return TM_ECUDA;
 }
 
-// Partition -> shard assignment (n_shards > 1): greedy longest-processing-time
-// over the estimated work |P| * 4^-|mask| (routing probability of a mask of
-// |mask| bits for queries with one-bit density ~1/4), ties by partition id.
-std::vector<uint32_t> assign_shards(const std::vector<Partition> &parts, uint32_t n_shards) {
-    std::vector<uint32_t> owner(parts.size(), 0);
-    if (n_shards <= 1) return owner;
-    std::vector<double> w(parts.size());
-    for (size_t i = 0; i < parts.size(); ++i) {
-        int pc = __builtin_popcountll(parts[i].mask.w[0]) + __builtin_popcountll(parts[i].mask.w[1]) +
-                 __builtin_popcountll(parts[i].mask.w[2]);
-        w[i] = (double)(parts[i].end - parts[i].begin) * std::pow(0.25, pc);
-    }
-    std::vector<uint32_t> ord(parts.size());
-    std::iota(ord.begin(), ord.end(), 0u);
-    std::stable_sort(ord.begin(), ord.end(), [&](uint32_t a, uint32_t b) { return w[a] > w[b]; });
-    std::vector<double> load(n_shards, 0.0);
-    for (uint32_t i : ord) {
-        uint32_t best = 0;
-        for (uint32_t s = 1; s < n_shards; ++s)
-            if (load[s] < load[best]) best = s;
-        owner[i] = best;
-        load[best] += w[i];
-    }
-    return owner;
-}
-
 void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys) {
     auto t0 = std::chrono::steady_clock::now();
     const bool trace = getenv("TM_TRACE_BUILD") != nullptr;
@@ -558,7 +528,7 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
     if (db->cfg.row_order == 1) refine_order(usig.data(), order, parts, 8);
     mark("row order");
     db->n_parts_total = parts.size();
-    const std::vector<uint32_t> owner = assign_shards(parts, std::max(1u, db->cfg.n_shards));
+    const std::vector<uint32_t> owner = plan_shards(db, parts);
 
     // S0d: layout -- kept partitions in acceptance order, each padded to 32 rows
     std::vector<uint32_t> keep;
@@ -643,6 +613,8 @@ tm_db *new_db(const tm_config *cfg) {
 
 void destroy_db(tm_db *db) {
     if (!db) return;
+    for (tm_db *sub : db->subs) destroy_db(sub);
+    db->subs.clear();
     int prev = -1;
     cudaGetDevice(&prev);
     cudaSetDevice(db->device);
@@ -710,12 +682,11 @@ const char *tm_strerror(tm_status s) {
 
 const char *tm_last_error(void) { return tmb::g_err.c_str(); }
 
-tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys, const tm_config *cfg,
-                   tm_db **out) {
-    tm_db *db = nullptr;
-    TM_API_BEGIN
-    if (!out) fail(TM_EINVAL, "out is NULL");
-    check_tagsets_host(sets, "sets");
+}  // extern "C"
+
+namespace tmb {
+// Validates the config and builds a single-GPU database (throws; the caller owns the result).
+tm_db *build_db(const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys, const tm_config *cfg) {
     if (cfg) {
         if (cfg->n_shards > 1 && cfg->shard >= cfg->n_shards) fail(TM_EINVAL, "shard >= n_shards");
         if (cfg->tile_filter > 2) fail(TM_EINVAL, "tile_filter must be 0, 1 or 2");
@@ -723,47 +694,34 @@ tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32
         if (cfg->row_order == 1 && cfg->tile_filter == 0)
             fail(TM_EINVAL, "row_order 1 needs tile_filter 1 or 2 (the first/last prefix needs lexicographic order)");
         if (cfg->exact > 1) fail(TM_EINVAL, "exact must be 0 or 1");
+        if (cfg->shard_mode > 1) fail(TM_EINVAL, "shard_mode must be TM_SHARD_PARTITIONED or TM_SHARD_REPLICATED");
         if (cfg->reserved) fail(TM_EINVAL, "reserved fields must be 0");
+        if (cfg->plan_sample) check_tagsets_host(cfg->plan_sample, "plan_sample");
     }
     const int dev = check_device(cfg ? cfg->device : -1);
     DeviceGuard g(dev);
-    db = new_db(cfg);
-    db->device = dev;
-    TMCK(cudaStreamCreateWithFlags(&db->stream, cudaStreamNonBlocking));
-    for (auto &e : db->ev) TMCK(cudaEventCreate(&e));
-    TMCK(cudaMallocHost((void **)&db->h_ctr, sizeof(DevCounters)));
-    TMCK(cudaMallocHost((void **)&db->h_nuniq, 8));
-    db->scan_grid = 0;
-    build_impl(db, sets, key_off, keys);
-    // load every scan-kernel variant now (lazy module loading would otherwise put ~10-30 ms into
-    // the first call that picks a variant: a latency spike inside a stream, profiles/r1v46_stream_*)
-    for (int v = 0; v < kScanVariants; ++v) db->grid_of[v] = scan_grid(db->device, v);
-    db->st.n_sets = db->n_sets;
-    *out = db;
-    db = nullptr;
-    return TM_OK;
+    tm_db *db = new_db(cfg);
+    try {
+        db->device = dev;
+        TMCK(cudaStreamCreateWithFlags(&db->stream, cudaStreamNonBlocking));
+        for (auto &e : db->ev) TMCK(cudaEventCreate(&e));
+        TMCK(cudaMallocHost((void **)&db->h_ctr, sizeof(DevCounters)));
+        TMCK(cudaMallocHost((void **)&db->h_nuniq, 8));
+        db->scan_grid = 0;
+        build_impl(db, sets, key_off, keys);
+        // load every scan-kernel variant now (lazy module loading would otherwise put ~10-30 ms into
+        // the first call that picks a variant: a latency spike inside a stream, profiles/r1v46_stream_*)
+        for (int v = 0; v < kScanVariants; ++v) db->grid_of[v] = scan_grid(db->device, v);
+        db->st.n_sets = db->n_sets;
+        db->cfg.plan_sample = nullptr;  // borrowed for the build only
+        db->cfg.device_ids = nullptr;
+    } catch (...) {
+        destroy_db(db);
+        throw;
     }
-    catch (const tmb::StatusFail &f) {
-        tmb::set_error(f.msg);
-        tmb::destroy_db(db);
-        return f.s;
-    }
-    catch (const tmb::CudaFail &f) {
-        tm_status s = tmb::translate(f);
-        tmb::destroy_db(db);
-        return s;
-    }
-    catch (const std::bad_alloc &) {
-        tmb::set_error("host allocation failed");
-        tmb::destroy_db(db);
-        return TM_ENOMEM;
-    }
-    catch (...) {
-        tmb::set_error("unexpected exception");
-        tmb::destroy_db(db);
-        return TM_ESTATE;
-    }
+    return db;
 }
+}  // namespace tmb
 
 namespace tmb {
 // H2D of a host query batch into the handle's input buffers; returns the device-side tagsets.
@@ -795,11 +753,40 @@ tm_tagsets upload_queries(tm_db *db, const tm_tagsets *q, cudaStream_t s) {
 }
 }  // namespace tmb
 
+extern "C" {
+
+tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys, const tm_config *cfg,
+                   tm_db **out) {
+    TM_API_BEGIN
+    if (!out) fail(TM_EINVAL, "out is NULL");
+    check_tagsets_host(sets, "sets");
+    if (cfg && cfg->n_gpus > 1) {  // in-process multi-GPU database (tm_group.cu)
+        tm_db *top = new_db(cfg);
+        try {
+            group_build(top, sets, key_off, keys, cfg);
+        } catch (...) {
+            destroy_db(top);
+            throw;
+        }
+        *out = top;
+        return TM_OK;
+    }
+    *out = build_db(sets, key_off, keys, cfg);
+    return TM_OK;
+    TM_API_END
+}
+
+
+
 tm_status tm_match_batch(tm_db *db, const tm_tagsets *q, int unique, tm_pairs *out) {
     TM_API_BEGIN
     if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
     if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
     check_tagsets_shape(q, "queries");
+    if (!db->subs.empty()) {
+        group_match(db, q, unique, out, nullptr);
+        return TM_OK;
+    }
     DeviceGuard g(db->device);
     cudaStream_t s = db->stream;
     const tm_tagsets dq = upload_queries(db, q, s);  // one H2D copy of the query batch
@@ -833,6 +820,10 @@ tm_status tm_match_batch_csr(tm_db *db, const tm_tagsets *q, int unique, tm_csr 
     if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
     if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
     check_tagsets_shape(q, "queries");
+    if (!db->subs.empty()) {
+        group_match(db, q, unique, nullptr, out);
+        return TM_OK;
+    }
     DeviceGuard g(db->device);
     cudaStream_t s = db->stream;
     const tm_tagsets dq = upload_queries(db, q, s);
@@ -868,6 +859,7 @@ tm_status tm_match_batch_csr(tm_db *db, const tm_tagsets *q, int unique, tm_csr 
 tm_status tm_match_batch_device(tm_db *db, const tm_tagsets *q, int unique, tm_dev_pairs *out, void *stream) {
     TM_API_BEGIN
     if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
+    if (!db->subs.empty()) fail(TM_ESTATE, "device-pointer calls are not available on an in-process multi-GPU handle");
     if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
     check_tagsets_device(q);
     DeviceGuard g(db->device);
@@ -958,6 +950,10 @@ tm_status tm_encode(const tm_tagsets *sets, uint64_t *sig_out, int device) {
 tm_status tm_stats(const tm_db *db, tm_stats_t *out) {
     TM_API_BEGIN
     if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
+    if (!db->subs.empty()) {
+        group_stats(db, out);
+        return TM_OK;
+    }
     *out = db->st;
     out->n_sets = db->n_sets;
     out->n_entries = db->n_entries;
@@ -975,6 +971,7 @@ tm_status tm_stats(const tm_db *db, tm_stats_t *out) {
 tm_status tm_partitions(const tm_db *db, uint64_t *masks, uint64_t *sizes) {
     TM_API_BEGIN
     if (!db) fail(TM_EINVAL, "db is NULL");
+    if (!db->subs.empty()) fail(TM_ESTATE, "use tm_group_member on an in-process multi-GPU handle");
     if (masks && !db->h_masks.empty()) std::memcpy(masks, db->h_masks.data(), db->h_masks.size() * 8);
     if (sizes && !db->h_sizes.empty()) std::memcpy(sizes, db->h_sizes.data(), db->h_sizes.size() * 8);
     return TM_OK;
@@ -984,6 +981,7 @@ tm_status tm_partitions(const tm_db *db, uint64_t *masks, uint64_t *sizes) {
 tm_status tm_partition_sigs(const tm_db *db, uint64_t p, uint64_t *sig_out) {
     TM_API_BEGIN
     if (!db || !sig_out) fail(TM_EINVAL, "db or sig_out is NULL");
+    if (!db->subs.empty()) fail(TM_ESTATE, "use tm_group_member on an in-process multi-GPU handle");
     if (p >= db->n_parts) fail(TM_EINVAL, "partition index out of range");
     DeviceGuard g(db->device);
     const uint64_t r0 = db->h_part_row[p], n = db->h_sizes[p];

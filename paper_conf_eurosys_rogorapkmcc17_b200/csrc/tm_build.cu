@@ -647,7 +647,7 @@ void build_gpu(tm_db *db, uint64_t N, const uint64_t *s0, const uint64_t *s1, co
         parts[i].begin = h_lo[i];
         parts[i].end = h_hi[i];
     }
-    const std::vector<uint32_t> owner = assign_shards(parts, std::max(1u, db->cfg.n_shards));
+    const std::vector<uint32_t> owner = plan_shards(db, parts);
     std::vector<uint32_t> keep;
     for (uint32_t i = 0; i < P; ++i)
         if (owner[i] == db->cfg.shard) keep.push_back(i);

@@ -147,6 +147,10 @@ struct tm_db {
     uint64_t last_n = 0, last_Q = 0;
     uint64_t last_qlo = 0, last_qn = 0;  // the query range the last call matched
     // shard layer (tm_shard.cu)
+    uint64_t *merged = nullptr;  // merge_pairs: the owner's sorted (q<<32|key) pairs (mq/mk split)
+    uint64_t merged_n = 0;
+    // in-process multi-GPU database (tm_group.cu): sub-databases, one per device
+    std::vector<tm_db *> subs;
     void *nccl_comm = nullptr;
     int nranks = 1, rank = 0;
     DevBuf xcounts, xall, xrecv, xalt, mq, mk;
@@ -167,7 +171,33 @@ int check_device(int dev);
 void check_tagsets_device(const tm_tagsets *t);
 void check_tagsets_host(const tm_tagsets *t, const char *what);
 int bits_for(uint64_t n);
-std::vector<uint32_t> assign_shards(const std::vector<Partition> &parts, uint32_t n_shards);
+// partition -> shard plan of the handle's config (tm_shard.cu): contiguous ranges of ~equal
+// estimated work; all zeros for one shard or a replicated database
+std::vector<uint32_t> plan_shards(tm_db *db, const std::vector<Partition> &parts);
+std::vector<uint32_t> plan_ranges(const std::vector<double> &w, uint32_t n_shards);
+std::vector<double> model_weights(const std::vector<Partition> &parts);
+void exchange_plan(const uint64_t *counts, uint32_t G, uint32_t r, uint64_t *send_off, uint64_t *recv_off);
+inline uint64_t owner_start(uint64_t Q, uint32_t G, uint32_t g) { return (Q * g) / G; }
+// sorts / de-duplicates n received (q<<32|key) pairs into db->mq / db->mk (db->merged: the sorted
+// u64 pairs); synchronous
+uint64_t merge_pairs(tm_db *db, uint64_t *in, uint64_t n, uint64_t Q, int unique, cudaStream_t s);
+// db->xcounts[g] = pairs of the last local result owned by g (G owner ranges of the last batch)
+void owner_counts(tm_db *db, uint32_t G, cudaStream_t s);
+tm_tagsets upload_queries(tm_db *db, const tm_tagsets *q, cudaStream_t s);
+// pinned host result blocks (cached; tm_api.cu)
+struct PinnedBlock {
+    void *p;
+    size_t cap;
+};
+PinnedBlock *pinned_get(size_t bytes);
+void pinned_put(PinnedBlock *b);
+// in-process multi-GPU databases (tm_group.cu)
+void group_build(tm_db *top, const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys,
+                 const tm_config *cfg);
+void group_match(tm_db *top, const tm_tagsets *q, int unique, tm_pairs *pout, tm_csr *cout);
+void group_stats(const tm_db *top, tm_stats_t *out);
+tm_db *build_db(const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys, const tm_config *cfg);
+void destroy_db(tm_db *db);
 void shard_destroy(tm_db *db);
 // exact subset post-check (tm_exact.cu)
 void exact_build(tm_db *db, const uint8_t *d_bytes, uint64_t n_bytes, const uint64_t *d_voff, uint64_t V,

@@ -546,10 +546,12 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // MINB: resident CTAs per SM the register allocator must allow (__launch_bounds__); shared memory
 // caps residency at 8 CTAs, which ptxas cannot see (the scan's shared memory is dynamic).
 // STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
-// OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>).
+// OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>); bit 3 = lazy row
+// loads (a tile's sets are loaded only when level B found a survivor; AND-mask tables).
 template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     constexpr bool kImad = (OPT & 1) != 0;
+    constexpr bool kLazy = (OPT & 8) != 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -819,8 +821,15 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                 const uint32_t row = row0 + lane;
                 const uint32_t nvalid = min(32u, real_end - row0);
                 const bool valid = (uint32_t)lane < nvalid;
-                // rows are padded to whole tiles: every lane may load
-                const uint64_t s0 = __ldg(p.w0 + row), s1 = __ldg(p.w1 + row), s2 = __ldg(p.w2 + row);
+                // rows are padded to whole tiles: every lane may load.  kLazy (AND-mask tables): the
+                // rows are loaded only once level B has found a survivor (most visited tiles have none)
+                const bool lazy = kLazy && WORD1 && p.filter != 0;
+                uint64_t s0 = ~0ULL, s1 = ~0ULL, s2 = ~0ULL;
+                if (!lazy) {
+                    s0 = __ldg(p.w0 + row);
+                    s1 = __ldg(p.w1 + row);
+                    s2 = __ldg(p.w2 + row);
+                }
                 uint64_t g0 = 0, g1 = 0, g2 = 0;
                 if (p.filter == 0) {
                     tile_prefix(shfl64(s0, 0), shfl64(s1, 0), shfl64(s2, 0), shfl64(s0, nvalid - 1),
@@ -830,21 +839,35 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     g1 = sm.tmask[warp][1][t - t_first];
                     g2 = sm.tmask[warp][2][t - t_first];
                 }
-                // 32-bit halves of the lane's set (invalid lanes: all ones, never pass)
-                const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
-                const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
-                const uint32_t a2l = valid ? (uint32_t)s2 : ~0u, a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
                 if constexpr (WORD1) {
-                    const uint32_t wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
-                    const uint32_t wl = wsel & 15u, wl2 = wsel >> 4;
-                    // branch-free word select: block wl >> 1, half wl & 1 (invalid lanes: all ones)
-                    const uint32_t aw = pick_word(s0, s1, s2, wl, valid);
-                    const uint32_t aw2 = pick_word(s0, s1, s2, wl2, valid);
-                    st_tests += na;
+                    // 32-bit halves of the lane's set (invalid lanes: all ones, never pass), its two
+                    // pre-check words and their planes: set up by row_setup() (at once, or lazily)
+                    uint32_t a0l, a0h, a1l, a1h, a2l, a2h, aw, aw2, my_plane, my_plane2;
                     const uint32_t *swp = sm.sw[warp][0];
                     const uint32_t sw_base = (uint32_t)__cvta_generic_to_shared(swp);
-                    const uint32_t my_plane = sw_base + wl * (uint32_t)(kSubWStride * 4);
-                    const uint32_t my_plane2 = sw_base + wl2 * (uint32_t)(kSubWStride * 4);
+                    auto row_setup = [&]() {
+                        if (lazy) {
+                            s0 = __ldg(p.w0 + row);
+                            s1 = __ldg(p.w1 + row);
+                            s2 = __ldg(p.w2 + row);
+                        }
+                        a0l = valid ? (uint32_t)s0 : ~0u;
+                        a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
+                        a1l = valid ? (uint32_t)s1 : ~0u;
+                        a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
+                        a2l = valid ? (uint32_t)s2 : ~0u;
+                        a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
+                        const uint32_t wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
+                        const uint32_t wl = wsel & 15u, wl2 = wsel >> 4;
+                        // branch-free word select: block wl >> 1, half wl & 1 (invalid lanes: all ones)
+                        aw = pick_word(s0, s1, s2, wl, valid);
+                        aw2 = pick_word(s0, s1, s2, wl2, valid);
+                        my_plane = sw_base + wl * (uint32_t)(kSubWStride * 4);
+                        my_plane2 = sw_base + wl2 * (uint32_t)(kSubWStride * 4);
+                    };
+                    bool have_rows = !lazy;
+                    if (!lazy) row_setup();
+                    st_tests += na;
                     for (uint32_t j = 0; j < na;) {
                         // ---- level B: level-A survivors that contain the tile's mask -> word planes,
                         // 32 at a time until the buffer cannot take another 32 (full pre-check groups)
@@ -881,6 +904,10 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                         }
                         st_checks += nb * nvalid;
                         __syncwarp();
+                        if (nb && !have_rows) {  // warp-uniform
+                            row_setup();
+                            have_rows = true;
+                        }
                         for (uint32_t k0 = 0; k0 < nb; k0 += 32) {
                             const uint32_t cnt = min(32u, nb - k0);
                             // ---- pre-check: the lane's word against 32 survivors, pass bits in acc
@@ -928,6 +955,10 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     }
                     continue;
                 }
+                // 32-bit halves of the lane's set (invalid lanes: all ones, never pass)
+                const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
+                const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
+                const uint32_t a2l = valid ? (uint32_t)s2 : ~0u, a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
                 for (uint32_t pb = 0; pb < na; pb += kPiece) {
                     const uint32_t pe = min(na, pb + kPiece);
                     // ---- level B: level-A survivors that contain the tile's mask
@@ -1056,292 +1087,6 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
         __syncthreads();
     }
     // the loop ends for all warps together (after the barrier that read the last item)
-    flush_pend(sm.pend[warp], npend, p, lane);
-    if (lane == 0 && (st_tests | st_checks | st_matched)) {
-        atomicAdd(&sm.cnt[0], (unsigned long long)st_tests);
-        atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
-        atomicAdd(&sm.cnt[2], (unsigned long long)st_matched);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        if (sm.cnt[0]) atomicAdd(&p.ctr->tile_tests, sm.cnt[0]);
-        if (sm.cnt[1]) atomicAdd(&p.ctr->pair_checks, sm.cnt[1]);
-        if (sm.cnt[2]) atomicAdd(&p.ctr->matched_sets, sm.cnt[2]);
-    }
-}
-
-// ---------------------------------------------------- bit-sliced filter ---
-// The filtered scan with Alg. 4's pre-filter evaluated bit-sliced.  The item's
-// batch is transposed once into Z[pos][w] (bit t = query 32 w + t LACKS position pos).  A query
-// contains a mask m iff no one-bit of m is one of its zero bits, so for the 32 queries of word w
-//     survivors(m) = ~OR_{pos in m} Z[pos][w]
-// -- one shared load + one OR per mask bit for 32 queries at once, lane w taking word w.  Level A
-// tests the 256-row block's AND mask (minus the partition mask, which every routed query already
-// contains), level B each 32-row tile's extra bits (tile AND minus the block AND) on the level-A
-// survivor words; a tile with no survivor costs ~2 instructions per extra bit and loads nothing.
-// Survivors of a tile are compacted into the per-warp word planes and go through the same two-word
-// pre-check + full check (Alg. 3) + fused emission as variant 5.
-constexpr int kZW = (kChunk + 31) / 32;   // query words per batch
-
-struct FiltSmem {
-    uint64_t q0[kChunk], q1[kChunk], q2[kChunk];   // the item's batch (SoA): plane fills, full checks
-    uint32_t z[192][kZW];                          // the batch bit-transposed (zero bits)
-    uint32_t sw[kScanWarps][6][kSubWStride];       // per-warp survivor word planes
-    uint16_t sbi[kScanWarps][kSubW];               // their batch slots
-    uint64_t tmask[kScanWarps][3][kBlockTiles];    // the unit's tile AND masks
-    const uint32_t *qid;
-    unsigned long long item;
-    unsigned int unit_ctr;
-    unsigned long long cnt[3];
-    uint2 pend[kScanWarps][kPend];
-};
-
-// OR of Z[pos][w] over the one-bits pos of the 192-bit mask (m0, m1, m2): warp-uniform bit loop
-__device__ __forceinline__ uint32_t zor(const uint32_t *__restrict__ zw, uint64_t m0, uint64_t m1, uint64_t m2) {
-    uint32_t acc = 0;
-    while (m0) {
-        const int j = __ffsll((long long)m0) - 1;
-        m0 &= m0 - 1;
-        acc |= zw[j * kZW];
-    }
-    while (m1) {
-        const int j = __ffsll((long long)m1) - 1;
-        m1 &= m1 - 1;
-        acc |= zw[(64 + j) * kZW];
-    }
-    while (m2) {
-        const int j = __ffsll((long long)m2) - 1;
-        m2 &= m2 - 1;
-        acc |= zw[(128 + j) * kZW];
-    }
-    return acc;
-}
-
-__device__ __forceinline__ uint32_t warp_sum(uint32_t v) { return __reduce_add_sync(0xffffffffu, v); }
-
-template <int OPT = 1>
-__global__ void __launch_bounds__(kScanWarps * 32, 5) k_filt(const ScanParams p) {
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    FiltSmem &sm = *reinterpret_cast<FiltSmem *>(smem_raw);
-    constexpr bool kImad = (OPT & 1) != 0;
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    uint32_t st_tests = 0, st_checks = 0, st_matched = 0;
-    uint32_t npend = 0;
-    const unsigned long long n_items = p.item_off[p.n_parts];
-    if (blockIdx.x == 0 && threadIdx.x == 0) p.ctr->n_items = n_items;
-    if (p.ctr->routed > p.qcap) return;
-    if (threadIdx.x < 3) sm.cnt[threadIdx.x] = 0;
-    uint16_t *sbi = sm.sbi[warp];
-    uint32_t *swk = sm.sw[warp][0];
-    const uint32_t sw_base = smem_u32(swk);
-    const uint32_t lt_mask = (1u << lane) - 1u;
-
-    for (;;) {
-        if (lane == 0 && (st_tests | st_checks | st_matched)) {
-            atomicAdd(&sm.cnt[0], (unsigned long long)st_tests);
-            atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
-            atomicAdd(&sm.cnt[2], (unsigned long long)st_matched);
-        }
-        st_tests = st_checks = st_matched = 0;
-        if (threadIdx.x == 0) {
-            sm.item = atomicAdd(&p.ctr->item_ctr, 1ULL);
-            sm.unit_ctr = 0;
-        }
-        __syncthreads();
-        const unsigned long long item = sm.item;
-        if (item >= n_items) break;
-        uint32_t lo = 0, hi = p.n_parts;
-        while (hi - lo > 1) {
-            const uint32_t mid = (lo + hi) >> 1;
-            if (__ldg(p.item_off + mid) <= item) lo = mid; else hi = mid;
-        }
-        const uint32_t part = lo;
-        const uint32_t prow = __ldg(p.part_row + part);
-        const uint32_t rows = __ldg(p.part_row + part + 1) - prow;
-        const uint32_t real_end = prow + __ldg(p.part_n + part);
-        const unsigned long long pq0 = __ldg(p.qoff + part), pq1 = __ldg(p.qoff + part + 1);
-        const uint32_t rr = part_range_rows(pq1 - pq0, p.range_rows);
-        const uint32_t nrange = (rows + rr - 1) / rr;
-        const unsigned long long local = item - __ldg(p.item_off + part);
-        const uint32_t chunk = (uint32_t)(local / nrange), range = (uint32_t)(local % nrange);
-        const unsigned long long qbeg = pq0 + (unsigned long long)chunk * kChunk;
-        const uint32_t nq = (uint32_t)min((unsigned long long)kChunk, pq1 - qbeg);
-        const uint32_t rlo = prow + range * rr;
-        const uint32_t rhi = min(rlo + rr, prow + rows);
-        const uint64_t pm0 = __ldg(p.pmask + 3 * part), pm1 = __ldg(p.pmask + 3 * part + 1),
-                       pm2 = __ldg(p.pmask + 3 * part + 2);
-        if (threadIdx.x == 0) sm.qid = p.qidx + qbeg;
-        // stage the batch, then transpose it: warp v builds query words v, v+4, ...
-        for (uint32_t i = threadIdx.x; i < nq; i += blockDim.x) {
-            const uint32_t q = __ldg(p.qidx + qbeg + i);
-            sm.q0[i] = __ldg(p.q0 + q);
-            sm.q1[i] = __ldg(p.q1 + q);
-            sm.q2[i] = __ldg(p.q2 + q);
-        }
-        __syncthreads();
-        const uint32_t nw = (nq + 31) / 32;
-        for (uint32_t w = warp; w < nw; w += kScanWarps) {
-            const uint32_t i = w * 32 + lane;
-            uint64_t a[3] = {~0ULL, ~0ULL, ~0ULL};  // past the batch: no zero bits (masked by validity)
-            if (i < nq) {
-                a[0] = sm.q0[i];
-                a[1] = sm.q1[i];
-                a[2] = sm.q2[i];
-            }
-#pragma unroll
-            for (int wd = 0; wd < 3; ++wd) {
-#pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                    const uint32_t x = (uint32_t)(a[wd] >> (32 * h));
-                    uint32_t mine = 0;
-#pragma unroll
-                    for (int t = 0; t < 32; ++t) {
-                        const uint32_t b = __ballot_sync(0xffffffffu, ((x >> t) & 1u) == 0u);
-                        if (lane == t) mine = b;
-                    }
-                    sm.z[64 * wd + 32 * h + lane][w] = mine;
-                }
-            }
-        }
-        __syncthreads();
-
-        const uint32_t ntile = (rhi - rlo) / kTile;
-        const uint32_t nblock = (ntile + kBlockTiles - 1) / kBlockTiles;
-        // unit = (256-row block, word-aligned query sub-range); few blocks: split the batch
-        const uint32_t nsplit = nblock >= (uint32_t)kScanWarps ? 1u : (uint32_t)kScanWarps / max(nblock, 1u);
-        const uint32_t subsz = ((nq + nsplit - 1) / nsplit + 31) & ~31u;
-        const uint32_t units = nblock * nsplit;
-        for (;;) {
-            uint32_t u = 0;
-            if (lane == 0) u = atomicAdd(&sm.unit_ctr, 1u);
-            u = __shfl_sync(0xffffffffu, u, 0);
-            if (u >= units) break;
-            const uint32_t blk = u / nsplit, sub = u % nsplit;
-            const uint32_t qs = sub * subsz, qe = min(nq, qs + subsz);
-            if (qs >= qe) continue;
-            const uint32_t t_first = blk * kBlockTiles, t_end = min(ntile, t_first + kBlockTiles);
-            const uint32_t brow0 = rlo + t_first * kTile;
-            // the unit's tile AND masks (lane = tile), staged for level B; block mask = their AND
-            const uint32_t t = brow0 / kTile + lane;
-            const bool in = (uint32_t)lane < t_end - t_first;
-            const uint64_t m0 = in ? __ldg(p.t0 + t) : ~0ULL, m1 = in ? __ldg(p.t1 + t) : ~0ULL,
-                           m2 = in ? __ldg(p.t2 + t) : ~0ULL;
-            const uint64_t f0 = warp_and(m0), f1 = warp_and(m1), f2 = warp_and(m2);
-            if ((uint32_t)lane < (uint32_t)kBlockTiles) {  // each tile's extra bits over the block mask
-                sm.tmask[warp][0][lane] = m0 & ~f0;
-                sm.tmask[warp][1][lane] = m1 & ~f1;
-                sm.tmask[warp][2][lane] = m2 & ~f2;
-            }
-            // ---- level A (bit-sliced): lane = query word of the sub-range
-            const uint32_t w = qs / 32 + lane;
-            const bool wv = w * 32 < qe;
-            const uint32_t *zw = &sm.z[0][0] + (wv ? w : 0);
-            const uint32_t vmask = wv ? (qe - w * 32 >= 32 ? ~0u : ((1u << (qe - w * 32)) - 1u)) : 0u;
-            const uint32_t sa = ~zor(zw, f0 & ~pm0, f1 & ~pm1, f2 & ~pm2) & vmask;
-            st_tests += qe - qs;
-            __syncwarp();
-            if (!__any_sync(0xffffffffu, sa != 0)) continue;
-            const uint32_t na = warp_sum(__popc(sa));
-            // ---- per tile of the block
-            for (uint32_t tt = t_first; tt < t_end; ++tt) {
-                const uint32_t row0 = rlo + tt * kTile;
-                const uint32_t k = tt - t_first;
-                // level B (bit-sliced): the tile's extra mask bits on the level-A survivor words
-                const uint32_t sb = sa & ~zor(zw, sm.tmask[warp][0][k], sm.tmask[warp][1][k], sm.tmask[warp][2][k]);
-                st_tests += na;
-                const uint32_t cnt_l = __popc(sb);
-                if (!__any_sync(0xffffffffu, cnt_l != 0)) continue;  // no survivor: no row is loaded
-                // exclusive prefix of the per-word survivor counts: where lane w's survivors go
-                uint32_t incl = cnt_l;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const uint32_t x = __shfl_up_sync(0xffffffffu, incl, o);
-                    if (lane >= o) incl += x;
-                }
-                const uint32_t nb = __shfl_sync(0xffffffffu, incl, 31);
-                const uint32_t excl = incl - cnt_l;
-                // the tile's sets, one per lane (rows are padded to whole tiles: every lane may load)
-                const uint32_t row = row0 + lane;
-                const uint32_t nvalid = min(32u, real_end - row0);
-                const bool valid = (uint32_t)lane < nvalid;
-                const uint64_t s0 = __ldg(p.w0 + row), s1 = __ldg(p.w1 + row), s2 = __ldg(p.w2 + row);
-                const uint32_t wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
-                const uint32_t wl = wsel & 15u, wl2 = wsel >> 4;
-                const uint32_t aw = pick_word(s0, s1, s2, wl, valid);
-                const uint32_t aw2 = pick_word(s0, s1, s2, wl2, valid);
-                const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
-                const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
-                const uint32_t a2l = valid ? (uint32_t)s2 : ~0u, a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
-                const uint32_t my_plane = sw_base + wl * (uint32_t)(kSubWStride * 4);
-                const uint32_t my_plane2 = sw_base + wl2 * (uint32_t)(kSubWStride * 4);
-                st_checks += nb * nvalid;
-                // passes of at most kSubW survivors through the word planes
-                for (uint32_t kb0 = 0; kb0 < nb; kb0 += kSubW) {
-                    const uint32_t npass = min((uint32_t)kSubW, nb - kb0);
-                    // compaction: lane w writes its survivors with rank in [kb0, kb0 + npass)
-                    if (excl < kb0 + npass && incl > kb0) {
-                        uint32_t r = sb, kk = excl;
-                        while (r) {
-                            const uint32_t bit = (uint32_t)(__ffs(r) - 1);
-                            r &= r - 1;
-                            if (kk >= kb0 + npass) break;
-                            if (kk >= kb0) {
-                                const uint32_t i = w * 32 + bit;
-                                store_survivor(swk, sbi, kk - kb0, sm.q0[i], sm.q1[i], sm.q2[i], i);
-                            }
-                            ++kk;
-                        }
-                    }
-                    __syncwarp();
-                    for (uint32_t k0 = 0; k0 < npass; k0 += 32) {
-                        const uint32_t cnt = min(32u, npass - k0);
-                        uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0;
-                        const uint32_t pa = my_plane + k0 * 4, pa2 = my_plane2 + k0 * 4;
-#define TM_FPRE(B, o) precheck4x2<B, kImad>(c0, c1, c2, c3, aw, lds128(pa + (o)), aw2, lds128(pa2 + (o)), p.one)
-                        TM_FPRE(1u << 0, 0);
-                        TM_FPRE(1u << 4, 16);
-                        if (cnt > 8) {
-                            TM_FPRE(1u << 8, 32);
-                            TM_FPRE(1u << 12, 48);
-                        }
-                        if (cnt > 16) {
-                            TM_FPRE(1u << 16, 64);
-                            TM_FPRE(1u << 20, 80);
-                        }
-                        if (cnt > 24) {
-                            TM_FPRE(1u << 24, 96);
-                            TM_FPRE(1u << 28, 112);
-                        }
-#undef TM_FPRE
-                        uint32_t acc = (c0 | c1) | (c2 | c3);
-                        if (cnt < 32) acc &= (1u << cnt) - 1u;
-                        if (!valid) acc = 0;
-                        while (__any_sync(0xffffffffu, acc != 0)) {
-                            bool m = false;
-                            uint32_t e = 0;
-                            if (acc) {
-                                e = k0 + (uint32_t)(__ffs(acc) - 1);
-                                acc &= acc - 1;
-                                const uint32_t *c = swk + e;
-                                m = ((a0l & ~c[0]) | (a0h & ~c[kSubWStride]) | (a1l & ~c[2 * kSubWStride]) |
-                                     (a1h & ~c[3 * kSubWStride]) | (a2l & ~c[4 * kSubWStride]) |
-                                     (a2h & ~c[5 * kSubWStride])) == 0;
-                            }
-                            const uint32_t bm = __ballot_sync(0xffffffffu, m);
-                            if (bm) {
-                                st_matched += __popc(bm);
-                                emit_keys(m, bm, row, m ? __ldg(sm.qid + sbi[e]) : 0u, p, lane, sm.pend[warp],
-                                          npend);
-                            }
-                        }
-                    }
-                    __syncwarp();
-                }
-            }
-            (void)lt_mask;
-        }
-        __syncthreads();
-    }
     flush_pend(sm.pend[warp], npend, p, lane);
     if (lane == 0 && (st_tests | st_checks | st_matched)) {
         atomicAdd(&sm.cnt[0], (unsigned long long)st_tests);
@@ -1792,7 +1537,7 @@ ScanFn scan_fn(int variant) {
         case 11: return k_dense<false, 0>;
         case 12: return k_dense<true, 0>;
         case 13: return k_dense<false, 5>;  // 9 + register prefetch of the next unit
-        case 14: return k_filt<1>;          // bit-sliced level A / B pre-filter (tile AND masks)
+        case 14: return k_scan<4, false, false, true, 7, false, 9>;  // 8 + lazy row loads
         default: return k_scan<4, false>;
     }
 }
@@ -1800,7 +1545,7 @@ ScanFn scan_fn(int variant) {
 
 size_t scan_smem(int variant) {
     if (variant == 9 || variant == 11 || variant == 13) return sizeof(DenseSmemBase);
-    if (variant == 14) return sizeof(FiltSmem);
+
     if (variant == 10 || variant == 12) return sizeof(DenseSmemBulk);
     return (variant == 6 || variant == 7) ? sizeof(StreamSmem) : sizeof(ScanSmem);
 }

@@ -16,6 +16,7 @@
 // NCCL is loaded at run time (dlopen), so the library loads without it.
 #include <dlfcn.h>
 
+#include <cmath>
 #include <cstring>
 #include <mutex>
 
@@ -85,8 +86,6 @@ NcclApi &nccl() {
         if (_r != ncclSuccess) fail(TM_ENCCL, std::string("NCCL: ") + nccl().errorString(_r) + " in " #call); \
     } while (0)
 
-inline uint64_t owner_start(uint64_t Q, uint32_t G, uint32_t g) { return (Q * g) / G; }
-
 // counts[g] = number of sorted (q<<32|key) pairs with owner(q) == g (one thread per owner)
 __global__ void k_owner_counts(const uint64_t *__restrict__ sorted, uint64_t n, uint64_t Q, uint32_t G,
                                unsigned long long *__restrict__ counts) {
@@ -104,6 +103,8 @@ __global__ void k_owner_counts(const uint64_t *__restrict__ sorted, uint64_t n, 
     const uint64_t b = (g + 1 == G) ? n : lower((Q * (g + 1) / G) << 32);
     counts[g] = b - a;
 }
+
+}  // namespace
 
 // Sort (query, key) pairs received by this owner, de-duplicate for match-unique,
 // split into db->mq / db->mk.  `in` may alias db->xrecv.
@@ -134,6 +135,8 @@ uint64_t merge_pairs(tm_db *db, uint64_t *in, uint64_t n, uint64_t Q, int unique
     db->mk.ensure(std::max<uint64_t>(n, 1) * 4);
     TMCK(launch_split(sorted, n, db->mq.as<uint32_t>(), db->mk.as<uint32_t>(), s));
     TMCK(cudaStreamSynchronize(s));
+    db->merged = sorted;
+    db->merged_n = n;
     return n;
 }
 
@@ -148,7 +151,88 @@ void owner_counts(tm_db *db, uint32_t G, cudaStream_t s) {
     TMCK(cudaGetLastError());
 }
 
+// ---------------------------------------------------------------- plan ---
+// Contiguous ranges of the partition table with ~equal work: partition i goes to
+// the shard whose 1/G share of the total work contains the middle of partition i's work.
+std::vector<uint32_t> plan_ranges(const std::vector<double> &w, uint32_t G) {
+    const size_t P = w.size();
+    std::vector<uint32_t> owner(P, 0);
+    if (G <= 1 || P == 0) return owner;
+    double W = 0;
+    for (double x : w) W += x;
+    double acc = 0;
+    for (size_t i = 0; i < P; ++i) {
+        const double mid = W > 0 ? (acc + 0.5 * w[i]) / W : (i + 0.5) / (double)P;
+        acc += w[i];
+        owner[i] = std::min<uint32_t>(G - 1, (uint32_t)(mid * G));
+    }
+    return owner;
+}
+
+// |P| x 4^-|mask|: the chance that a query contains a mask of |mask| bits when ~1/4 of a query's
+// positions are set (an 8-tag query sets ~49 of 192 bits, fn.3 / PAPER.md:132)
+std::vector<double> model_weights(const std::vector<Partition> &parts) {
+    std::vector<double> w(parts.size());
+    for (size_t i = 0; i < parts.size(); ++i) {
+        const int pc = __builtin_popcountll(parts[i].mask.w[0]) + __builtin_popcountll(parts[i].mask.w[1]) +
+                       __builtin_popcountll(parts[i].mask.w[2]);
+        w[i] = (double)(parts[i].end - parts[i].begin) * std::pow(0.25, pc);
+    }
+    return w;
+}
+
+namespace {
+// queries of the config's plan sample routed to each partition (Alg. 2 on the GPU: the library's
+// encoder and bit-sliced router, pass 0)
+std::vector<uint64_t> sample_routes(tm_db *db, const std::vector<Partition> &parts, cudaStream_t s) {
+    const tm_tagsets *smp = db->cfg.plan_sample;
+    const uint64_t P = parts.size(), Qs = smp ? smp->n_sets : 0;
+    std::vector<uint64_t> routed(P, 0);
+    if (!Qs || !P) return routed;
+    const tm_tagsets dq = upload_queries(db, smp, s);
+    DevBuf vsig, planes, masks, counts;
+    vsig.ensure(std::max<uint64_t>(dq.n_vocab, 1) * 24);
+    planes.ensure(Qs * 24);
+    uint64_t *q0 = planes.as<uint64_t>(), *q1 = q0 + Qs, *q2 = q1 + Qs;
+    TMCK(launch_hash_vocab(dq.vocab_bytes, dq.vocab_off, dq.n_vocab, dq.n_bytes, vsig.as<uint64_t>(), nullptr, s));
+    TMCK(launch_encode_sets(vsig.as<uint64_t>(), dq.n_tags ? dq.tag_idx : nullptr, dq.set_off, Qs, dq.n_tags,
+                            dq.n_vocab, q0, q1, q2, nullptr, s));
+    std::vector<uint64_t> hm(3 * P);
+    for (uint64_t i = 0; i < P; ++i)
+        for (int w = 0; w < 3; ++w) hm[3 * i + w] = parts[i].mask.w[w];
+    masks.ensure(P * 24);
+    TMCK(cudaMemcpyAsync(masks.p, hm.data(), P * 24, cudaMemcpyHostToDevice, s));
+    const uint64_t NB = route_blocks(Qs);
+    counts.ensure(P * NB * 4);
+    TMCK(launch_route(0, masks.as<uint64_t>(), (uint32_t)P, q0, q1, q2, Qs, counts.as<uint32_t>(), nullptr, nullptr, 0,
+                      s));
+    std::vector<uint32_t> hc(P * NB);
+    TMCK(cudaMemcpyAsync(hc.data(), counts.p, P * NB * 4, cudaMemcpyDeviceToHost, s));
+    TMCK(cudaStreamSynchronize(s));
+    for (uint64_t i = 0; i < P; ++i)
+        for (uint64_t b = 0; b < NB; ++b) routed[i] += hc[i * NB + b];
+    return routed;
+}
 }  // namespace
+
+std::vector<uint32_t> plan_shards(tm_db *db, const std::vector<Partition> &parts) {
+    const uint32_t G = std::max(1u, db->cfg.n_shards);
+    if (G <= 1 || db->cfg.shard_mode == TM_SHARD_REPLICATED) return std::vector<uint32_t>(parts.size(), 0);
+    const std::vector<uint64_t> routed = sample_routes(db, parts, db->stream);
+    std::vector<double> w(parts.size(), 0.0);
+    double W = 0;
+    for (size_t i = 0; i < parts.size(); ++i) W += (w[i] = (double)(parts[i].end - parts[i].begin) * routed[i]);
+    if (W <= 0) w = model_weights(parts);
+    return plan_ranges(w, G);
+}
+
+void exchange_plan(const uint64_t *counts, uint32_t G, uint32_t r, uint64_t *send_off, uint64_t *recv_off) {
+    send_off[0] = recv_off[0] = 0;
+    for (uint32_t p = 0; p < G; ++p) {
+        send_off[p + 1] = send_off[p] + counts[(size_t)r * G + p];
+        recv_off[p + 1] = recv_off[p] + counts[(size_t)p * G + r];
+    }
+}
 
 void shard_destroy(tm_db *db) {
     if (db && db->nccl_comm) {
@@ -171,8 +255,8 @@ tm_status tm_owner_range(uint64_t n_queries, uint32_t n_owners, uint32_t owner, 
     TM_API_END
 }
 
-tm_status tm_shard_plan(const uint64_t *masks, const uint64_t *sizes, uint64_t n_parts, uint32_t n_shards,
-                        uint32_t *owner_out) {
+tm_status tm_shard_plan(const uint64_t *masks, const uint64_t *sizes, const uint64_t *routed, uint64_t n_parts,
+                        uint32_t n_shards, uint32_t *owner_out) {
     TM_API_BEGIN
     if ((n_parts && (!masks || !sizes || !owner_out)) || n_shards == 0) fail(TM_EINVAL, "bad shard plan arguments");
     std::vector<Partition> parts(n_parts);
@@ -183,8 +267,22 @@ tm_status tm_shard_plan(const uint64_t *masks, const uint64_t *sizes, uint64_t n
         b += sizes[i];
         parts[i].end = b;
     }
-    const std::vector<uint32_t> own = assign_shards(parts, n_shards);
-    std::memcpy(owner_out, own.data(), own.size() * 4);
+    std::vector<double> w(n_parts, 0.0);
+    double W = 0;
+    if (routed)
+        for (uint64_t i = 0; i < n_parts; ++i) W += (w[i] = (double)sizes[i] * (double)routed[i]);
+    if (W <= 0) w = model_weights(parts);
+    const std::vector<uint32_t> own = plan_ranges(w, n_shards);
+    if (n_parts) std::memcpy(owner_out, own.data(), own.size() * 4);
+    return TM_OK;
+    TM_API_END
+}
+
+tm_status tm_exchange_plan(const uint64_t *counts, uint32_t n_ranks, uint32_t rank, uint64_t *send_off,
+                           uint64_t *recv_off) {
+    TM_API_BEGIN
+    if (!counts || !send_off || !recv_off || n_ranks == 0 || rank >= n_ranks) fail(TM_EINVAL, "bad exchange plan arguments");
+    tmb::exchange_plan(counts, n_ranks, rank, send_off, recv_off);
     return TM_OK;
     TM_API_END
 }
@@ -227,6 +325,7 @@ tm_status tm_partition_host(const uint64_t *sigs, uint64_t n, uint32_t max_parti
 tm_status tm_last_result(const tm_db *db, const uint64_t **pairs, uint64_t *n) {
     TM_API_BEGIN
     if (!db || !pairs || !n) fail(TM_EINVAL, "NULL argument");
+    if (!db->subs.empty()) fail(TM_ESTATE, "not available on an in-process multi-GPU handle");
     *pairs = db->last_sorted;
     *n = db->last_n;
     return TM_OK;
@@ -236,6 +335,7 @@ tm_status tm_last_result(const tm_db *db, const uint64_t **pairs, uint64_t *n) {
 tm_status tm_shard_counts(tm_db *db, uint32_t n_owners, uint64_t *counts_out) {
     TM_API_BEGIN
     if (!db || !counts_out || n_owners == 0) fail(TM_EINVAL, "bad arguments");
+    if (!db->subs.empty()) fail(TM_ESTATE, "not available on an in-process multi-GPU handle");
     DeviceGuard g(db->device);
     owner_counts(db, n_owners, db->stream);
     TMCK(cudaMemcpyAsync(counts_out, db->xcounts.p, n_owners * 8, cudaMemcpyDeviceToHost, db->stream));
@@ -248,6 +348,7 @@ tm_status tm_shard_merge(tm_db *db, const uint64_t *pairs, uint64_t n, uint64_t 
                          tm_dev_pairs *out, void *stream) {
     TM_API_BEGIN
     if (!db || !out || (n && !pairs)) fail(TM_EINVAL, "bad arguments");
+    if (!db->subs.empty()) fail(TM_ESTATE, "not available on an in-process multi-GPU handle");
     DeviceGuard g(db->device);
     cudaStream_t s = stream ? static_cast<cudaStream_t>(stream) : db->stream;
     db->xrecv.ensure(std::max<uint64_t>(n, 1) * 8);
@@ -274,6 +375,7 @@ tm_status tm_comm_init(tm_db *db, const void *id, uint64_t len, int nranks, int 
     TM_API_BEGIN
     if (!db || !id || len < sizeof(ncclUniqueId) || nranks < 1 || rank < 0 || rank >= nranks)
         fail(TM_EINVAL, "bad communicator arguments");
+    if (!db->subs.empty()) fail(TM_ESTATE, "not available on an in-process multi-GPU handle");
     if (db->cfg.n_shards != (uint32_t)nranks || db->cfg.shard != (uint32_t)rank)
         fail(TM_ESTATE, "the handle must be built with n_shards == nranks and shard == rank");
     DeviceGuard g(db->device);
@@ -293,13 +395,28 @@ tm_status tm_match_batch_sharded_device(tm_db *db, const tm_tagsets *q, int uniq
                                         void *stream) {
     TM_API_BEGIN
     if (!db || !out) fail(TM_EINVAL, "db or out is NULL");
-    if (!db->nccl_comm) fail(TM_ESTATE, "tm_comm_init was not called");
+    if (!db->subs.empty()) fail(TM_ESTATE, "not available on an in-process multi-GPU handle");
     if (unique != 0 && unique != 1) fail(TM_EINVAL, "unique must be 0 or 1");
     check_tagsets_device(q);
     DeviceGuard g(db->device);
     cudaStream_t s = stream ? static_cast<cudaStream_t>(stream) : db->stream;
     tm_tagsets dq = *q;
     if (!dq.n_tags) dq.tag_idx = nullptr;
+    if (db->cfg.shard_mode == TM_SHARD_REPLICATED) {
+        // the whole table on every rank: match this rank's owner range only, no exchange
+        const uint32_t G = std::max(1u, db->cfg.n_shards);
+        const uint64_t lo = owner_start(q->n_sets, G, db->cfg.shard), hi = owner_start(q->n_sets, G, db->cfg.shard + 1);
+        const uint64_t n = match_core(db, &dq, unique, s, lo, hi - lo);
+        finish_timing(db, s);
+        db->st.local_ms = db->st.total_ms;
+        db->st.xchg_ms = 0;
+        db->st.xchg_send_bytes = db->st.xchg_recv_bytes = 0;
+        out->n = n;
+        out->query = db->res_q.as<uint32_t>();
+        out->key = db->res_k.as<uint32_t>();
+        return TM_OK;
+    }
+    if (!db->nccl_comm) fail(TM_ESTATE, "tm_comm_init was not called");
     // S1-S8 against the local partitions
     match_core(db, &dq, unique, s);
     finish_timing(db, s);
@@ -317,10 +434,7 @@ tm_status tm_match_batch_sharded_device(tm_db *db, const tm_tagsets *q, int uniq
     TMCK(cudaMemcpyAsync(all.data(), db->xall.p, (size_t)G * G * 8, cudaMemcpyDeviceToHost, s));
     TMCK(cudaStreamSynchronize(s));
     std::vector<uint64_t> soff(G + 1, 0), roff(G + 1, 0);
-    for (uint32_t p = 0; p < G; ++p) {
-        soff[p + 1] = soff[p] + all[(size_t)r * G + p];
-        roff[p + 1] = roff[p] + all[(size_t)p * G + r];
-    }
+    exchange_plan(all.data(), G, (uint32_t)r, soff.data(), roff.data());
     db->xrecv.ensure(std::max<uint64_t>(roff[G], 1) * 8);
     // all-to-all-v of (q<<32|key) pairs to query owners
     TMNC(a.groupStart());

@@ -39,7 +39,13 @@ class tm_tagsets(ctypes.Structure):
 class tm_config(ctypes.Structure):
     _fields_ = [("max_partition", ctypes.c_uint32), ("device", ctypes.c_int32), ("n_shards", ctypes.c_uint32),
                 ("shard", ctypes.c_uint32), ("tile_filter", ctypes.c_uint32), ("row_order", ctypes.c_uint32),
-                ("exact", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+                ("exact", ctypes.c_uint32), ("n_gpus", ctypes.c_uint32), ("shard_mode", ctypes.c_uint32),
+                ("reserved", ctypes.c_uint32), ("device_ids", ctypes.c_void_p),
+                ("plan_sample", ctypes.POINTER(tm_tagsets))]
+
+
+TM_SHARD_PARTITIONED = 0
+TM_SHARD_REPLICATED = 1
 
 
 class tm_pairs(ctypes.Structure):
@@ -90,7 +96,7 @@ class tm_stats_t(ctypes.Structure):
 EXPORTS = ["tm_build", "tm_match_batch", "tm_match_batch_csr", "tm_match_batch_device", "tm_pairs_free",
            "tm_csr_free", "tm_free", "tm_strerror",
            "tm_last_error", "tm_abi_version", "tm_build_id", "tm_encode", "tm_stats", "tm_partitions", "tm_partition_sigs",
-           "tm_owner_range", "tm_shard_plan", "tm_partition_host", "tm_last_result", "tm_shard_counts",
+           "tm_owner_range", "tm_shard_plan", "tm_exchange_plan", "tm_group_size", "tm_group_member", "tm_partition_host", "tm_last_result", "tm_shard_counts",
            "tm_shard_merge", "tm_nccl_unique_id", "tm_comm_init", "tm_match_batch_sharded_device",
            "tm_stream_open", "tm_stream_submit", "tm_stream_poll", "tm_stream_result_free", "tm_stream_flush",
            "tm_stream_replay", "tm_stream_close"]
@@ -134,7 +140,10 @@ def load(path: str = LIB_PATH):
     L.tm_partition_sigs.argtypes = [vp, ctypes.c_uint64, vp]
     u64, u32, i32 = ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
     for name, args in [("tm_owner_range", [u64, u32, u32, vp, vp]),
-                       ("tm_shard_plan", [vp, vp, u64, u32, vp]),
+                       ("tm_shard_plan", [vp, vp, vp, u64, u32, vp]),
+                       ("tm_exchange_plan", [vp, u32, u32, vp, vp]),
+                       ("tm_group_size", [vp, vp]),
+                       ("tm_group_member", [vp, u32, vp]),
                        ("tm_partition_host", [vp, u64, u32, vp, vp, vp, vp, vp]),
                        ("tm_last_result", [vp, vp, vp]),
                        ("tm_shard_counts", [vp, u32, vp]),
@@ -193,7 +202,7 @@ def device_tagsets(vocab_bytes_ptr, vocab_off_ptr, tag_idx_ptr, set_off_ptr, n_b
 
 
 def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0, row_order=0,
-                exact=0) -> tm_config:
+                exact=0, n_gpus=0, shard_mode=0) -> tm_config:
     c = tm_config()
     c.max_partition = max_partition
     c.device = device
@@ -202,6 +211,8 @@ def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0, 
     c.tile_filter = tile_filter
     c.row_order = row_order
     c.exact = exact
+    c.n_gpus = n_gpus
+    c.shard_mode = shard_mode
     return c
 
 
@@ -209,17 +220,28 @@ class Database:
     """A tm_db handle: tm_build on construction, tm_free on close()."""
 
     def __init__(self, sets, key_off=None, keys=None, max_partition=0, device=-1, n_shards=1, shard=0,
-                 tile_filter=0, row_order=0, exact=0):
+                 tile_filter=0, row_order=0, exact=0, n_gpus=0, shard_mode=0, device_ids=None, plan_sample=None):
+        """n_gpus > 1: an in-process multi-GPU database on device_ids (default 0..n_gpus-1; repeats
+        allowed); shard_mode TM_SHARD_PARTITIONED / TM_SHARD_REPLICATED; plan_sample: host query
+        batch whose routing weighs the partition -> shard plan."""
         L = load()
         self._sets = sets if isinstance(sets, HostTagSets) else HostTagSets.of(sets)
         self._ko = None if key_off is None else np.ascontiguousarray(key_off, dtype=np.uint64)
         self._ks = np.ascontiguousarray(keys if keys is not None else np.zeros(0), dtype=np.uint32)
-        cfg = make_config(max_partition, device, n_shards, shard, tile_filter, row_order, exact)
+        cfg = make_config(max_partition, device, n_shards, shard, tile_filter, row_order, exact, n_gpus, shard_mode)
+        ids = None
+        if device_ids is not None:
+            ids = np.ascontiguousarray(device_ids, dtype=np.int32)
+            cfg.device_ids = ctypes.c_void_p(ids.ctypes.data)
+        smp = None
+        if plan_sample is not None:
+            smp = plan_sample if isinstance(plan_sample, HostTagSets) else HostTagSets.of(plan_sample)
+            cfg.plan_sample = ctypes.pointer(smp.c)
         h = ctypes.c_void_p()
         _check(L.tm_build(ctypes.byref(self._sets.c), _ptr(self._ko), _ptr(self._ks) if self._ks.size else None,
                           ctypes.byref(cfg), ctypes.byref(h)))
         self.h = h
-        del self._sets  # inputs are not retained by the library
+        del self._sets, ids, smp  # inputs are not retained by the library
 
     def match_batch(self, queries, unique: bool) -> tuple[np.ndarray, np.ndarray]:
         """tm_match_batch: host queries -> sorted (query, key) arrays (copies out of pinned memory)."""
@@ -278,6 +300,19 @@ class Database:
         _check(load().tm_match_batch_device(self.h, ctypes.byref(dq), int(bool(unique)), ctypes.byref(out),
                                             ctypes.c_void_p(stream) if stream else None))
         return out
+
+    def group_size(self) -> int:
+        n = ctypes.c_uint32()
+        _check(load().tm_group_size(self.h, ctypes.byref(n)))
+        return n.value
+
+    def member_stats(self, g: int) -> dict:
+        """tm_stats of sub-database g of an in-process multi-GPU handle (tm_group_member)."""
+        sub = ctypes.c_void_p()
+        _check(load().tm_group_member(self.h, g, ctypes.byref(sub)))
+        s = tm_stats_t()
+        _check(load().tm_stats(sub, ctypes.byref(s)))
+        return s.as_dict()
 
     def stats(self) -> dict:
         s = tm_stats_t()
@@ -371,12 +406,26 @@ def owner_range(n_queries: int, n_owners: int, owner: int) -> tuple[int, int]:
     return lo.value, hi.value
 
 
-def shard_plan(masks: np.ndarray, sizes: np.ndarray, n_shards: int) -> np.ndarray:
+def shard_plan(masks: np.ndarray, sizes: np.ndarray, n_shards: int, routed: np.ndarray | None = None) -> np.ndarray:
+    """tm_shard_plan: contiguous partition ranges of ~equal work |P| x routed (or |P| x 4^-|mask|)."""
     masks = np.ascontiguousarray(masks, dtype=np.uint64).reshape(-1, 3)
     sizes = np.ascontiguousarray(sizes, dtype=np.uint64)
+    r = None if routed is None else np.ascontiguousarray(routed, dtype=np.uint64)
     out = np.zeros(masks.shape[0], np.uint32)
-    _check(load().tm_shard_plan(_ptr(masks), _ptr(sizes), masks.shape[0], n_shards, _ptr(out)))
+    _check(load().tm_shard_plan(_ptr(masks), _ptr(sizes), _ptr(r) if r is not None else None, masks.shape[0],
+                                n_shards, _ptr(out)))
     return out
+
+
+def exchange_plan(counts: np.ndarray, rank: int) -> tuple[np.ndarray, np.ndarray]:
+    """tm_exchange_plan: (send_off [G+1], recv_off [G+1]) of `rank` from the G x G count matrix
+    counts[s, d] = pairs rank s holds for owner d."""
+    c = np.ascontiguousarray(counts, dtype=np.uint64)
+    G = c.shape[0]
+    so = np.zeros(G + 1, np.uint64)
+    ro = np.zeros(G + 1, np.uint64)
+    _check(load().tm_exchange_plan(_ptr(c), G, rank, _ptr(so), _ptr(ro)))
+    return so, ro
 
 
 def partition_host(sigs: np.ndarray, max_partition: int = 0):

@@ -66,7 +66,7 @@ def main():
             ms = float(np.median(scan))
             table_bytes = 24 * rows
             gbs = table_bytes / (ms / 1e3) / 1e9
-            if B == 1 and db_sig is None:
+            if db_sig is None:
                 db_sig = o2.encode(wl.db)
             ok = None
             if True:   # brute-force parity of the B queries at every B (<= 256 queries: seconds)

@@ -44,15 +44,36 @@ def test_alg1_dedupes_identical_signatures():
 
 
 @pytest.mark.parametrize("G", [1, 2, 3, 8])
-def test_shard_plan_is_a_balanced_partition_of_partitions(c1, G):
+@pytest.mark.parametrize("routed", [False, True])
+def test_shard_plan_contiguous_balanced_ranges(c1, G, routed):
+    """tm_shard_plan: contiguous ranges of the partition table, deterministic, each
+    shard's work within one partition's work of the fair share W/G (the midpoint rule)."""
     sig = o2.encode(c1.db)
     masks, sizes, _ = tm.partition_host(sig, 300)
-    own = tm.shard_plan(masks, sizes, G)
+    r = None
+    if routed:   # weights from a routed query sample: Alg. 2 by brute force (the oracle's)
+        qs = o2.encode(c1.queries)
+        r = np.array([int(np.sum(np.all((m[None, :] & ~qs) == 0, axis=1))) for m in masks], np.uint64)
+        w = sizes.astype(float) * r
+    else:
+        w = sizes * 0.25 ** np.array([sum(bin(int(x)).count("1") for x in m) for m in masks])
+    own = tm.shard_plan(masks, sizes, G, r)
     assert own.shape[0] == masks.shape[0] and own.max() < G
-    assert np.array_equal(own, tm.shard_plan(masks, sizes, G))   # deterministic
-    w = sizes * 0.25 ** np.array([sum(bin(int(x)).count("1") for x in m) for m in masks])
+    assert np.all(np.diff(own.astype(np.int64)) >= 0)                 # contiguous ranges, in order
+    assert np.array_equal(own, tm.shard_plan(masks, sizes, G, r))    # deterministic
     load = np.array([w[own == g].sum() for g in range(G)])
-    assert load.max() - load.min() <= w.max() + 1e-9              # greedy LPT bound
+    assert np.all(np.abs(load - w.sum() / G) <= w.max() + 1e-9)
+
+
+def test_exchange_plan_offsets():
+    """tm_exchange_plan: send offsets = prefix of the rank's row, receive offsets = prefix of its column."""
+    rng = np.random.default_rng(5)
+    for G in (1, 2, 3, 8):
+        c = rng.integers(0, 1000, (G, G)).astype(np.uint64)
+        for r in range(G):
+            so, ro = tm.exchange_plan(c, r)
+            assert np.array_equal(so, np.concatenate([[0], np.cumsum(c[r, :])]))
+            assert np.array_equal(ro, np.concatenate([[0], np.cumsum(c[:, r])]))
 
 
 @pytest.mark.parametrize("Q,G", [(0, 3), (1, 4), (100, 3), (100_000, 8), (7, 7)])
@@ -97,26 +118,38 @@ def _shard_worker(rank, world, port, result):
             # local match of this shard (the oracle stands in for the GPU scan)
             lq, lk = o2.match_brute(sig[idx], ko, ks, qsig, unique)
             pairs = (lq.astype(np.uint64) << np.uint64(32)) | lk.astype(np.uint64)
-            # cut at the owner boundaries, exchange counts, then the pairs
+            # cut at the owner boundaries, all-gather the count matrix, then the library's
+            # exchange plan (tm_exchange_plan) gives the send / receive offsets
             cuts = [tm.owner_range(Q, world, g) for g in range(world)]
-            seg = [pairs[(lq >= lo) & (lq < hi)] for lo, hi in cuts]
-            cnt = torch.tensor([s.size for s in seg], dtype=torch.int64)
+            cnt = torch.tensor([int(np.sum((lq >= lo) & (lq < hi))) for lo, hi in cuts], dtype=torch.int64)
             allc = [torch.zeros(world, dtype=torch.int64) for _ in range(world)]
             dist.all_gather(allc, cnt)
-            # grouped point-to-point send/recv, as ncclSend/ncclRecv in the library
-            recv = [torch.zeros(int(allc[g][rank]), dtype=torch.int64) for g in range(world)]
+            counts = np.stack([a.numpy() for a in allc]).astype(np.uint64)
+            soff, roff = tm.exchange_plan(counts, rank)
+            # grouped point-to-point send/recv, as ncclSend/ncclRecv in the library: the sorted
+            # local pairs are the send buffer (owners are contiguous query ranges)
+            rbuf = torch.zeros(int(roff[-1]), dtype=torch.int64)
+            sbuf = torch.from_numpy(pairs.view(np.int64).copy())
             reqs = []
             for g in range(world):
+                s0, s1 = int(soff[g]), int(soff[g + 1])
+                r0, r1 = int(roff[g]), int(roff[g + 1])
                 if g == rank:
-                    recv[g] = torch.from_numpy(seg[g].view(np.int64).copy())
+                    rbuf[r0:r1] = sbuf[s0:s1]
                     continue
-                if seg[g].size:
-                    reqs.append(dist.isend(torch.from_numpy(seg[g].view(np.int64).copy()), g))
-                if recv[g].numel():
-                    reqs.append(dist.irecv(recv[g], g))
-            for r in reqs:
-                r.wait()
-            got = np.concatenate([recv[g].numpy().view(np.uint64) for g in range(world)])
+                if s1 > s0:
+                    reqs.append(dist.isend(sbuf[s0:s1].clone(), g))
+                if r1 > r0:
+                    tmp = torch.zeros(r1 - r0, dtype=torch.int64)
+                    reqs.append((dist.irecv(tmp, g), tmp, r0, r1))
+            for rq in reqs:
+                if isinstance(rq, tuple):
+                    rq[0].wait()
+                    rbuf[rq[2]:rq[3]] = rq[1]
+                else:
+                    rq.wait()
+            recv = [rbuf]
+            got = np.concatenate([r.numpy().view(np.uint64) for r in recv])
             got = np.sort(got)
             if unique:
                 got = np.unique(got)
