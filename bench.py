@@ -26,7 +26,7 @@ N > 1  : one process per GPU (torchrun), the same batch on every rank, "scaling"
          partitions and the pairs go to query owners over NCCL (tm_match_batch_sharded_device).
          --replicated: every rank holds the whole database and matches its owner range of the
          batch, no exchange (NEXT-1; the library's TM_SHARD_REPLICATED).
-MAX_P  : auto (TM_AUTO_MAX_PARTITION: clamp(N / 10^4, 5K, 200K), R8b) unless
+MAX_P  : auto (TM_AUTO_MAX_PARTITION: clamp(N / 3*10^4, 5K, 200K), R8b) unless
          --max-partition N (--max-partition 200000 = the paper's value).
 --impl reference : the oracle (oracle/o2.c, the paper's CPU method) on the
          host cores, on a bounded sample of the same workload per step.
@@ -131,7 +131,7 @@ def load_workload(name: str, rank: int = 0):
         mp = getattr(load_workload, "max_partition", -1)
         c = dict(tmgen.CRAFTED[name], max_partition=0xFFFFFFFE if mp == -1 else (mp or 200_000), total_tags=0,
                  oracle_max_partition=200_000)
-        c["resolved_max_partition"] = min(200_000, max(5_000, c["n_sets"] // 10_000))
+        c["resolved_max_partition"] = min(200_000, max(5_000, c["n_sets"] // 30_000))
         wl = tmgen.config(name, max_partition=c["max_partition"],
                           query_seed=c["seed"] + (1 << 32) + 7919 * rank)
         return wl, c
@@ -140,7 +140,7 @@ def load_workload(name: str, rank: int = 0):
     mp = getattr(load_workload, "max_partition", -1)
     if mp == -1:
         c["max_partition"] = 0xFFFFFFFE   # TM_AUTO_MAX_PARTITION
-        c["resolved_max_partition"] = min(200_000, max(5_000, c["n_sets"] // 10_000))  # the library's rule
+        c["resolved_max_partition"] = min(200_000, max(5_000, c["n_sets"] // 30_000))  # the library's rule
     elif mp:
         c["max_partition"] = mp
     wl = tmgen.generate(c["n_sets"], c["n_queries"], c["seed"], total_tags=c["total_tags"],
@@ -231,7 +231,7 @@ def config_block(c, args, wl, sharded=False):
             "query_tags": (f"{c['set_tags']}-tag DB sets, {c['query_tags']}-tag queries (PAPER.md:391-399)"
                            if "set_tags" in c else
                            "base set + 2..4 extra" if not c["total_tags"] else f"total {c['total_tags']}"),
-            "max_partition": (f"auto: clamp(N/1e4, 5000, 200000) = {c['resolved_max_partition']}"
+            "max_partition": (f"auto: clamp(N/3e4, 5000, 200000) = {c['resolved_max_partition']}"
                               if c["max_partition"] == 0xFFFFFFFE else c["max_partition"]),
             "mode": "match-unique" if args.unique else "match",
             "tile_filter": ["alg4-prefix", "tile-and", "none"][args.tile_filter],

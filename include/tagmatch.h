@@ -57,10 +57,10 @@ extern "C" {
 /* max_partition value meaning "no partitioning": one partition with the empty
  * mask, routed to every query (reading R8; BASELINE config C1). */
 #define TM_NO_PARTITIONING 0xFFFFFFFFu
-/* max_partition value meaning "choose MAX_P from the database size": clamp(n_sets / 10^4,
+/* max_partition value meaning "choose MAX_P from the database size": clamp(n_sets / 30,000,
  * 5,000, 200,000) (reading R8b: the paper's optimum of ~200K
  * comes from its CPU pipeline's per-partition cost; with the bit-sliced GPU router the
- * measured optimum is ~10^4 partitions: C2 best at 5K, C3 at 10K). */
+ * measured optimum is much smaller: C2 (1M sets) and C3 (100M) at 5K, C4 (300M) at 10K). */
 #define TM_AUTO_MAX_PARTITION 0xFFFFFFFEu
 
 typedef struct tm_db tm_db; /* opaque, owned by the library */
@@ -227,6 +227,30 @@ uint32_t tm_abi_version(void);
 /* Identifier of the library build: a hash of its CUDA/C++ sources, fixed at compile time
  * (lets measurement scripts tie a profile to the exact kernels it was taken on). */
 const char *tm_build_id(void);
+
+/* ------------------------------------------- add-set / remove-set / consolidate --- */
+/*
+ * The paper's interface (Table 2): add-set(set, key) and remove-set(set, key)
+ * "are not immediately effective and instead are staged in a temporary index and become
+ * effective only after a call to the consolidate function", which builds the partition and
+ * tagset tables (Algorithm 1).  tm_create makes an empty, mutable database
+ * (matches see the last consolidated state: initially empty); tm_build's handles are not
+ * mutable (TM_ESTATE).  A set is given as n_tags tag strings bytes[tag_off[t] .. tag_off[t+1])
+ * (tag_off[0] = 0); repeated tags do not count, order does not matter.  The database is a
+ * multiset of (set, key) entries: add-set adds one instance; remove-set removes one instance
+ * of an identical entry if there is one (else nothing; reading R20).  Staged
+ * operations are applied in call order by tm_consolidate, which then rebuilds the GPU tables
+ * (the same encode / sort / Alg. 1 / layout as tm_build; on failure the handle keeps its
+ * tables and the operations stay staged).  The library keeps the entries on the host.
+ */
+tm_status tm_create(const tm_config *cfg, tm_db **out);
+tm_status tm_add_set(tm_db *db, const uint8_t *bytes, const uint64_t *tag_off, uint64_t n_tags, uint32_t key);
+tm_status tm_remove_set(tm_db *db, const uint8_t *bytes, const uint64_t *tag_off, uint64_t n_tags, uint32_t key);
+/* add-set for every (set i, key) of a batch (key_off / keys as tm_build) */
+tm_status tm_add_sets(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys);
+tm_status tm_consolidate(tm_db *db);
+/* staged operations and live entries (instances) of a mutable handle */
+tm_status tm_pending(const tm_db *db, uint64_t *n_staged, uint64_t *n_live);
 
 /* ---------------------------------------------------------- test hooks --- */
 

@@ -259,7 +259,6 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
         sp.wsel = db->wsel.as<uint8_t>();
         sp.range_rows = range_rows;
         sp.one = 1;
-        sp.pmask = db->masks.as<uint64_t>();
         // variant: TM_SCAN_VARIANT if set; else a call whose partition batches are all small
         // (Q <= kSmallBatch) takes the streaming path only, in the streaming-only kernels (small
         // shared memory: 8 CTAs/SM) -- up to four queries checked directly (variant 6), 5-8
@@ -436,8 +435,8 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
     if (K > 0 && !keys) fail(TM_EINVAL, "keys is NULL");
     db->n_sets = N;
     db->n_entries = K;
-    if (db->cfg.max_partition == TM_AUTO_MAX_PARTITION)  // reading R8b: ~10^4 partitions
-        db->cfg.max_partition = (uint32_t)std::min<uint64_t>(200000, std::max<uint64_t>(5000, N / 10000));
+    if (db->cfg.max_partition == TM_AUTO_MAX_PARTITION)  // reading R8b: MAX_P = N / 3*10^4 (measured)
+        db->cfg.max_partition = (uint32_t)std::min<uint64_t>(200000, std::max<uint64_t>(5000, N / 30000));
 
     // S0a: encode every set on the GPU
     DevBuf d_bytes, d_voff, d_tidx, d_soff, d_vsig, d_planes, d_sorted, d_idx, d_idx2, d_key, d_key2;
@@ -613,6 +612,7 @@ tm_db *new_db(const tm_config *cfg) {
 
 void destroy_db(tm_db *db) {
     if (!db) return;
+    store_destroy(db);
     for (tm_db *sub : db->subs) destroy_db(sub);
     db->subs.clear();
     int prev = -1;
@@ -750,6 +750,36 @@ tm_tagsets upload_queries(tm_db *db, const tm_tagsets *q, cudaStream_t s) {
         dq.tag_idx = nullptr;
     }
     return dq;
+}
+// consolidate() of a mutable handle: a fresh database is built from the live entries and swapped
+// into the handle (the caller's pointer stays valid); the old tables are freed.
+void rebuild(tm_db *db, const tm_tagsets *sets, const uint32_t *keys, const tm_config *cfg) {
+    tm_db *fresh = nullptr;
+    if (cfg->n_gpus > 1) {
+        fresh = new_db(cfg);
+        try {
+            group_build(fresh, sets, nullptr, keys, cfg);
+        } catch (...) {
+            destroy_db(fresh);
+            throw;
+        }
+    } else {
+        fresh = build_db(sets, nullptr, keys, cfg);
+    }
+    Store *st = db->store;
+    std::vector<int32_t> devs = std::move(db->store_devices);
+    void *comm = db->nccl_comm;
+    const int nr = db->nranks, rk = db->rank;
+    db->store = nullptr;
+    db->nccl_comm = nullptr;
+    std::swap(*db, *fresh);
+    db->store = st;
+    db->store_devices = std::move(devs);
+    db->nccl_comm = comm;
+    db->nranks = nr;
+    db->rank = rk;
+    fresh->nccl_comm = nullptr;
+    destroy_db(fresh);
 }
 }  // namespace tmb
 

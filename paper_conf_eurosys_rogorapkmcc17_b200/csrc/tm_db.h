@@ -13,6 +13,8 @@
 
 namespace tmb {
 
+struct Store;  // add-set / remove-set staging of a mutable handle (tm_store.cpp)
+
 struct CudaFail {
     cudaError_t e;
     const char *what;
@@ -151,6 +153,9 @@ struct tm_db {
     uint64_t merged_n = 0;
     // in-process multi-GPU database (tm_group.cu): sub-databases, one per device
     std::vector<tm_db *> subs;
+    // mutable handle (tm_create; tm_store.cpp): the entry multiset + staged operations
+    Store *store = nullptr;
+    std::vector<int32_t> store_devices;
     void *nccl_comm = nullptr;
     int nranks = 1, rank = 0;
     DevBuf xcounts, xall, xrecv, xalt, mq, mk;
@@ -172,7 +177,7 @@ void check_tagsets_device(const tm_tagsets *t);
 void check_tagsets_host(const tm_tagsets *t, const char *what);
 int bits_for(uint64_t n);
 // partition -> shard plan of the handle's config (tm_shard.cu): contiguous ranges of ~equal
-// estimated work; all zeros for one shard or a replicated database
+// estimated work; one shard: all 0; replicated: all = this handle's shard (it keeps everything)
 std::vector<uint32_t> plan_shards(tm_db *db, const std::vector<Partition> &parts);
 std::vector<uint32_t> plan_ranges(const std::vector<double> &w, uint32_t n_shards);
 std::vector<double> model_weights(const std::vector<Partition> &parts);
@@ -197,6 +202,9 @@ void group_build(tm_db *top, const tm_tagsets *sets, const uint64_t *key_off, co
 void group_match(tm_db *top, const tm_tagsets *q, int unique, tm_pairs *pout, tm_csr *cout);
 void group_stats(const tm_db *top, tm_stats_t *out);
 tm_db *build_db(const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys, const tm_config *cfg);
+// consolidate(): rebuild the handle's tables in place from sets / keys (one key per set)
+void rebuild(tm_db *db, const tm_tagsets *sets, const uint32_t *keys, const tm_config *cfg);
+void store_destroy(tm_db *db);
 void destroy_db(tm_db *db);
 void shard_destroy(tm_db *db);
 // exact subset post-check (tm_exact.cu)

@@ -28,10 +28,10 @@ constexpr int kScanWarps = 4;      // warps per CTA
 constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch); 640 fits 7 CTAs/SM of shared memory and measured 1.3% faster than 512 (profiles/r1v34_ab.txt)
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
-constexpr int kScanVariants = 15;    // k_scan variants (TM_SCAN_VARIANT)
-constexpr int kTune[] = {5, 0};  // variants the handle times on its first calls (first = default); 2 never won
+constexpr int kScanVariants = 14;    // k_scan variants (TM_SCAN_VARIANT)
+constexpr int kTune[] = {8, 5};  // variants the handle times on its first calls (first = default); 0-4 never won
 constexpr int kTuneN = 2;
-constexpr int kTuneDense[] = {10, 9};  // tables without a pre-filter (tile_filter = 2): the dense scan
+constexpr int kTuneDense[] = {9, 13};  // tables without a pre-filter (tile_filter = 2): the dense scan
 constexpr int kTuneMinQ = 4096;     // smaller calls are not tuned (default variant kTune[0])
 
 struct DevCounters {            // zeroed at the start of every match call
@@ -67,7 +67,6 @@ struct ScanParams {
     const uint8_t *wsel;              // [rows] pre-check word per row (variant 5)
     uint32_t range_rows;              // rows per work item (multiple of 256)
     uint32_t one;                     // 1 (a run-time operand, so the FMA-pipe accumulate stays an IMAD)
-    const uint64_t *pmask;            // [P][3] partition masks (bits every routed query contains)
 };
 
 // ------------------------------------------------------------ launchers --

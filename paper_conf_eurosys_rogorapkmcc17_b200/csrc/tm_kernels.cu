@@ -546,12 +546,10 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // MINB: resident CTAs per SM the register allocator must allow (__launch_bounds__); shared memory
 // caps residency at 8 CTAs, which ptxas cannot see (the scan's shared memory is dynamic).
 // STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
-// OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>); bit 3 = lazy row
-// loads (a tile's sets are loaded only when level B found a survivor; AND-mask tables).
+// OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>).
 template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     constexpr bool kImad = (OPT & 1) != 0;
-    constexpr bool kLazy = (OPT & 8) != 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -821,15 +819,8 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                 const uint32_t row = row0 + lane;
                 const uint32_t nvalid = min(32u, real_end - row0);
                 const bool valid = (uint32_t)lane < nvalid;
-                // rows are padded to whole tiles: every lane may load.  kLazy (AND-mask tables): the
-                // rows are loaded only once level B has found a survivor (most visited tiles have none)
-                const bool lazy = kLazy && WORD1 && p.filter != 0;
-                uint64_t s0 = ~0ULL, s1 = ~0ULL, s2 = ~0ULL;
-                if (!lazy) {
-                    s0 = __ldg(p.w0 + row);
-                    s1 = __ldg(p.w1 + row);
-                    s2 = __ldg(p.w2 + row);
-                }
+                // rows are padded to whole tiles: every lane may load
+                const uint64_t s0 = __ldg(p.w0 + row), s1 = __ldg(p.w1 + row), s2 = __ldg(p.w2 + row);
                 uint64_t g0 = 0, g1 = 0, g2 = 0;
                 if (p.filter == 0) {
                     tile_prefix(shfl64(s0, 0), shfl64(s1, 0), shfl64(s2, 0), shfl64(s0, nvalid - 1),
@@ -839,35 +830,21 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     g1 = sm.tmask[warp][1][t - t_first];
                     g2 = sm.tmask[warp][2][t - t_first];
                 }
+                // 32-bit halves of the lane's set (invalid lanes: all ones, never pass)
+                const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
+                const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
+                const uint32_t a2l = valid ? (uint32_t)s2 : ~0u, a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
                 if constexpr (WORD1) {
-                    // 32-bit halves of the lane's set (invalid lanes: all ones, never pass), its two
-                    // pre-check words and their planes: set up by row_setup() (at once, or lazily)
-                    uint32_t a0l, a0h, a1l, a1h, a2l, a2h, aw, aw2, my_plane, my_plane2;
+                    const uint32_t wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
+                    const uint32_t wl = wsel & 15u, wl2 = wsel >> 4;
+                    // branch-free word select: block wl >> 1, half wl & 1 (invalid lanes: all ones)
+                    const uint32_t aw = pick_word(s0, s1, s2, wl, valid);
+                    const uint32_t aw2 = pick_word(s0, s1, s2, wl2, valid);
+                    st_tests += na;
                     const uint32_t *swp = sm.sw[warp][0];
                     const uint32_t sw_base = (uint32_t)__cvta_generic_to_shared(swp);
-                    auto row_setup = [&]() {
-                        if (lazy) {
-                            s0 = __ldg(p.w0 + row);
-                            s1 = __ldg(p.w1 + row);
-                            s2 = __ldg(p.w2 + row);
-                        }
-                        a0l = valid ? (uint32_t)s0 : ~0u;
-                        a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
-                        a1l = valid ? (uint32_t)s1 : ~0u;
-                        a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
-                        a2l = valid ? (uint32_t)s2 : ~0u;
-                        a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
-                        const uint32_t wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
-                        const uint32_t wl = wsel & 15u, wl2 = wsel >> 4;
-                        // branch-free word select: block wl >> 1, half wl & 1 (invalid lanes: all ones)
-                        aw = pick_word(s0, s1, s2, wl, valid);
-                        aw2 = pick_word(s0, s1, s2, wl2, valid);
-                        my_plane = sw_base + wl * (uint32_t)(kSubWStride * 4);
-                        my_plane2 = sw_base + wl2 * (uint32_t)(kSubWStride * 4);
-                    };
-                    bool have_rows = !lazy;
-                    if (!lazy) row_setup();
-                    st_tests += na;
+                    const uint32_t my_plane = sw_base + wl * (uint32_t)(kSubWStride * 4);
+                    const uint32_t my_plane2 = sw_base + wl2 * (uint32_t)(kSubWStride * 4);
                     for (uint32_t j = 0; j < na;) {
                         // ---- level B: level-A survivors that contain the tile's mask -> word planes,
                         // 32 at a time until the buffer cannot take another 32 (full pre-check groups)
@@ -904,10 +881,6 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                         }
                         st_checks += nb * nvalid;
                         __syncwarp();
-                        if (nb && !have_rows) {  // warp-uniform
-                            row_setup();
-                            have_rows = true;
-                        }
                         for (uint32_t k0 = 0; k0 < nb; k0 += 32) {
                             const uint32_t cnt = min(32u, nb - k0);
                             // ---- pre-check: the lane's word against 32 survivors, pass bits in acc
@@ -955,10 +928,6 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     }
                     continue;
                 }
-                // 32-bit halves of the lane's set (invalid lanes: all ones, never pass)
-                const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
-                const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
-                const uint32_t a2l = valid ? (uint32_t)s2 : ~0u, a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
                 for (uint32_t pb = 0; pb < na; pb += kPiece) {
                     const uint32_t pe = min(na, pb + kPiece);
                     // ---- level B: level-A survivors that contain the tile's mask
@@ -1159,10 +1128,10 @@ __device__ __forceinline__ void bulk_g2s(void *dst, const void *src, uint32_t by
                  : "memory");
 }
 
-// OPT: bit 0 = FMA-pipe pre-check accumulate; bit 2 (direct loads only) = register prefetch of
-// the warp's next unit while the current one is checked (software pipelining of the HBM reads).
+// OPT: bit 0 = FMA-pipe pre-check accumulate; bit 2 (direct loads only) = four rows per lane
+// (128-row units, both row pairs' loads issued before the checks: twice the bytes in flight).
 template <bool BULK, int OPT = 0>
-__global__ void __launch_bounds__(kScanWarps * 32, (BULK || (OPT & 4)) ? 6 : 7) k_dense(const ScanParams p) {
+__global__ void __launch_bounds__(kScanWarps * 32, BULK ? 6 : 7) k_dense(const ScanParams p) {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<BULK, DenseSmemBulk, DenseSmemBase>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -1227,7 +1196,10 @@ __global__ void __launch_bounds__(kScanWarps * 32, (BULK || (OPT & 4)) ? 6 : 7) 
             sm.dp[5][i] = (uint32_t)(a2 >> 32);
         }
         __syncthreads();
-        const uint32_t nunit = (rhi - rlo + kDenseRows - 1) / kDenseRows;
+        // rows per unit: 64 (two per lane), or 128 with kRows4 (four per lane, all loads issued first)
+        constexpr bool kRows4 = !BULK && (OPT & 4) != 0;
+        constexpr uint32_t kUnitRows = kRows4 ? 2 * kDenseRows : kDenseRows;
+        const uint32_t nunit = (rhi - rlo + kUnitRows - 1) / kUnitRows;
         auto take = [&]() {
             uint32_t u = 0;
             if (lane == 0) u = atomicAdd(&sm.unit_ctr, 1u);
@@ -1248,6 +1220,71 @@ __global__ void __launch_bounds__(kScanWarps * 32, (BULK || (OPT & 4)) ? 6 : 7) 
                 }
             }
         };
+        // direct loads of rows (r, r + 1) of a lane (all-ones past the range)
+        auto load_pair = [&](uint32_t r, ulonglong2 &x0, ulonglong2 &x1, ulonglong2 &x2, uint32_t &xw) {
+            x0 = x1 = x2 = make_ulonglong2(~0ULL, ~0ULL);
+            xw = 0x1010u;
+            if (r < rhi) {
+                x0 = ldg_stream2(p.w0 + r);
+                x1 = ldg_stream2(p.w1 + r);
+                x2 = ldg_stream2(p.w2 + r);
+                xw = __ldg(reinterpret_cast<const unsigned short *>(p.wsel + r));
+            }
+        };
+        // the two-word pre-check of rows (u0 + 2 lane, + 1) against the batch, full checks, emission
+        auto check_pair = [&](const ulonglong2 v0, const ulonglong2 v1, const ulonglong2 v2, const uint32_t wab,
+                              const uint32_t u0) {
+                const uint32_t ra = u0 + 2 * (uint32_t)lane, rb = ra + 1;
+                const uint64_t a0 = v0.x, a1 = v1.x, a2 = v2.x, b0 = v0.y, b1 = v1.y, b2 = v2.y;
+                const bool va = ra < vend, vb = rb < vend;
+                const uint32_t wa = wab & 0xffu, wb = wab >> 8;
+                const uint32_t xa = pick_word(a0, a1, a2, wa & 15u, va), ya = pick_word(a0, a1, a2, wa >> 4, va);
+                const uint32_t xb = pick_word(b0, b1, b2, wb & 15u, vb), yb = pick_word(b0, b1, b2, wb >> 4, vb);
+                const uint32_t pxa = dp_base + (wa & 15u) * kPl, pya = dp_base + (wa >> 4) * kPl;
+                const uint32_t pxb = dp_base + (wb & 15u) * kPl, pyb = dp_base + (wb >> 4) * kPl;
+                for (uint32_t k0 = 0; k0 < nq; k0 += 32) {
+                    uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0, d0 = 0, d1 = 0, d2 = 0, d3 = 0;
+                    const uint32_t o = k0 * 4;
+    #define TM_DPRE(B, g)                                                                                        \
+        precheck4x2<B, kImad>(c0, c1, c2, c3, xa, lds128(pxa + o + 16 * (g)), ya, lds128(pya + o + 16 * (g)), p.one); \
+        precheck4x2<B, kImad>(d0, d1, d2, d3, xb, lds128(pxb + o + 16 * (g)), yb, lds128(pyb + o + 16 * (g)), p.one)
+                    const uint32_t left = nq - k0;
+                    TM_DPRE(1u << 0, 0);
+                    if (left > 4) { TM_DPRE(1u << 4, 1); }
+                    if (left > 8) { TM_DPRE(1u << 8, 2); }
+                    if (left > 12) { TM_DPRE(1u << 12, 3); }
+                    if (left > 16) { TM_DPRE(1u << 16, 4); }
+                    if (left > 20) { TM_DPRE(1u << 20, 5); }
+                    if (left > 24) { TM_DPRE(1u << 24, 6); }
+                    if (left > 28) { TM_DPRE(1u << 28, 7); }
+    #undef TM_DPRE
+                    const uint32_t qmask = left >= 32 ? ~0u : ((1u << left) - 1u);
+                    uint32_t acc_a = va ? ((c0 | c1) | (c2 | c3)) & qmask : 0u;
+                    uint32_t acc_b = vb ? ((d0 | d1) | (d2 | d3)) & qmask : 0u;
+                    // Alg. 3 on the pairs that passed: all six words, then emit (keys fused, S7)
+                    while (__any_sync(0xffffffffu, (acc_a | acc_b) != 0)) {
+                        bool m = false;
+                        uint32_t j = 0, row = ra;
+                        if (acc_a | acc_b) {
+                            const bool isb = acc_a == 0;
+                            uint32_t &acc = isb ? acc_b : acc_a;
+                            j = k0 + (uint32_t)(__ffs(acc) - 1);
+                            acc &= acc - 1;
+                            row = isb ? rb : ra;
+                            const uint64_t s0 = isb ? b0 : a0, s1 = isb ? b1 : a1, s2 = isb ? b2 : a2;
+                            m = (((uint32_t)s0 & ~sm.dp[0][j]) | ((uint32_t)(s0 >> 32) & ~sm.dp[1][j]) |
+                                 ((uint32_t)s1 & ~sm.dp[2][j]) | ((uint32_t)(s1 >> 32) & ~sm.dp[3][j]) |
+                                 ((uint32_t)s2 & ~sm.dp[4][j]) | ((uint32_t)(s2 >> 32) & ~sm.dp[5][j])) == 0;
+                        }
+                        const uint32_t bm = __ballot_sync(0xffffffffu, m);
+                        if (bm) {
+                            st_matched += __popc(bm);
+                            emit_keys(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane, sm.pend[warp], npend);
+                        }
+                    }
+                }
+            st_checks += nq * (vend > u0 ? min((uint32_t)kDenseRows, vend - u0) : 0u);
+        };
         // BULK: the warp's reserved units in issue order (stage of ring0 = si, ring1 = si + 1, ...);
         // rotated by value so no array is indexed dynamically (no local memory)
         static_assert(kDenseStages == 3, "the ring below is written for three stages");
@@ -1261,41 +1298,18 @@ __global__ void __launch_bounds__(kScanWarps * 32, (BULK || (OPT & 4)) ? 6 : 7) 
             if (ring2 < nunit) issue(2, ring2);
         }
         uint32_t si = 0;
-        constexpr bool kPf = !BULK && (OPT & 4) != 0;
-        // direct loads of unit u's two rows per lane (all-ones past the range)
-        auto load_unit = [&](uint32_t u, ulonglong2 &x0, ulonglong2 &x1, ulonglong2 &x2, uint32_t &xw) {
-            const uint32_t r = rlo + u * kDenseRows + 2 * (uint32_t)lane;
-            x0 = x1 = x2 = make_ulonglong2(~0ULL, ~0ULL);
-            xw = 0x1010u;
-            if (u < nunit && r < rhi) {
-                x0 = ldg_stream2(p.w0 + r);
-                x1 = ldg_stream2(p.w1 + r);
-                x2 = ldg_stream2(p.w2 + r);
-                xw = __ldg(reinterpret_cast<const unsigned short *>(p.wsel + r));
-            }
-        };
-        uint32_t pu = 0;
-        ulonglong2 pv0, pv1, pv2;
-        uint32_t pwab = 0;
-        if constexpr (kPf) {
-            pu = take();
-            load_unit(pu, pv0, pv1, pv2, pwab);
-        }
         for (;;) {
-            uint32_t u;
-            ulonglong2 v0, v1, v2;
-            uint32_t wab;
             if constexpr (BULK) {
-                u = ring0;
+                const uint32_t u = ring0;
                 if (u >= nunit) break;  // later reservations are larger: nothing is in flight
                 while (!mbar_try_wait(&sm.bar[warp][si], (par >> si) & 1u)) {
                 }
                 par ^= 1u << si;
                 const uint64_t *st = sm.stage[warp][si];
-                v0 = *reinterpret_cast<const ulonglong2 *>(st + 2 * lane);
-                v1 = *reinterpret_cast<const ulonglong2 *>(st + kDenseRows + 2 * lane);
-                v2 = *reinterpret_cast<const ulonglong2 *>(st + 2 * kDenseRows + 2 * lane);
-                wab = *reinterpret_cast<const unsigned short *>(&sm.wstage[warp][si][2 * lane]);
+                ulonglong2 v0 = *reinterpret_cast<const ulonglong2 *>(st + 2 * lane);
+                ulonglong2 v1 = *reinterpret_cast<const ulonglong2 *>(st + kDenseRows + 2 * lane);
+                ulonglong2 v2 = *reinterpret_cast<const ulonglong2 *>(st + 2 * kDenseRows + 2 * lane);
+                uint32_t wab = *reinterpret_cast<const unsigned short *>(&sm.wstage[warp][si][2 * lane]);
                 if (rlo + u * kDenseRows + 2 * (uint32_t)lane >= rhi) {  // past a 32-row unit: stale stage bytes
                     v0 = v1 = v2 = make_ulonglong2(~0ULL, ~0ULL);
                     wab = 0x1010u;
@@ -1307,71 +1321,25 @@ __global__ void __launch_bounds__(kScanWarps * 32, (BULK || (OPT & 4)) ? 6 : 7) 
                 ring1 = ring2;
                 ring2 = nu;
                 si = si == kDenseStages - 1 ? 0 : si + 1;
-            } else if constexpr (kPf) {
-                u = pu;
+                check_pair(v0, v1, v2, wab, rlo + u * kDenseRows);
+            } else if constexpr (kRows4) {
+                const uint32_t u = take();
                 if (u >= nunit) break;
-                v0 = pv0;
-                v1 = pv1;
-                v2 = pv2;
-                wab = pwab;
-                pu = take();  // the next unit's loads fly while this one is checked
-                load_unit(pu, pv0, pv1, pv2, pwab);
+                const uint32_t u0 = rlo + u * kUnitRows;
+                ulonglong2 v0, v1, v2, y0, y1, y2;
+                uint32_t wab, wcd;
+                load_pair(u0 + 2 * (uint32_t)lane, v0, v1, v2, wab);  // 96 B per lane in flight
+                load_pair(u0 + kDenseRows + 2 * (uint32_t)lane, y0, y1, y2, wcd);
+                check_pair(v0, v1, v2, wab, u0);
+                check_pair(y0, y1, y2, wcd, u0 + kDenseRows);
             } else {
-                u = take();
+                const uint32_t u = take();
                 if (u >= nunit) break;
-                load_unit(u, v0, v1, v2, wab);
+                ulonglong2 v0, v1, v2;
+                uint32_t wab;
+                load_pair(rlo + u * kDenseRows + 2 * (uint32_t)lane, v0, v1, v2, wab);
+                check_pair(v0, v1, v2, wab, rlo + u * kDenseRows);
             }
-            const uint32_t u0 = rlo + u * kDenseRows;
-            const uint32_t ra = u0 + 2 * (uint32_t)lane, rb = ra + 1;
-            const uint64_t a0 = v0.x, a1 = v1.x, a2 = v2.x, b0 = v0.y, b1 = v1.y, b2 = v2.y;
-            const bool va = ra < vend, vb = rb < vend;
-            const uint32_t wa = wab & 0xffu, wb = wab >> 8;
-            const uint32_t xa = pick_word(a0, a1, a2, wa & 15u, va), ya = pick_word(a0, a1, a2, wa >> 4, va);
-            const uint32_t xb = pick_word(b0, b1, b2, wb & 15u, vb), yb = pick_word(b0, b1, b2, wb >> 4, vb);
-            const uint32_t pxa = dp_base + (wa & 15u) * kPl, pya = dp_base + (wa >> 4) * kPl;
-            const uint32_t pxb = dp_base + (wb & 15u) * kPl, pyb = dp_base + (wb >> 4) * kPl;
-            for (uint32_t k0 = 0; k0 < nq; k0 += 32) {
-                uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0, d0 = 0, d1 = 0, d2 = 0, d3 = 0;
-                const uint32_t o = k0 * 4;
-#define TM_DPRE(B, g)                                                                                        \
-    precheck4x2<B, kImad>(c0, c1, c2, c3, xa, lds128(pxa + o + 16 * (g)), ya, lds128(pya + o + 16 * (g)), p.one); \
-    precheck4x2<B, kImad>(d0, d1, d2, d3, xb, lds128(pxb + o + 16 * (g)), yb, lds128(pyb + o + 16 * (g)), p.one)
-                const uint32_t left = nq - k0;
-                TM_DPRE(1u << 0, 0);
-                if (left > 4) { TM_DPRE(1u << 4, 1); }
-                if (left > 8) { TM_DPRE(1u << 8, 2); }
-                if (left > 12) { TM_DPRE(1u << 12, 3); }
-                if (left > 16) { TM_DPRE(1u << 16, 4); }
-                if (left > 20) { TM_DPRE(1u << 20, 5); }
-                if (left > 24) { TM_DPRE(1u << 24, 6); }
-                if (left > 28) { TM_DPRE(1u << 28, 7); }
-#undef TM_DPRE
-                const uint32_t qmask = left >= 32 ? ~0u : ((1u << left) - 1u);
-                uint32_t acc_a = va ? ((c0 | c1) | (c2 | c3)) & qmask : 0u;
-                uint32_t acc_b = vb ? ((d0 | d1) | (d2 | d3)) & qmask : 0u;
-                // Alg. 3 on the pairs that passed: all six words, then emit (keys fused, S7)
-                while (__any_sync(0xffffffffu, (acc_a | acc_b) != 0)) {
-                    bool m = false;
-                    uint32_t j = 0, row = ra;
-                    if (acc_a | acc_b) {
-                        const bool isb = acc_a == 0;
-                        uint32_t &acc = isb ? acc_b : acc_a;
-                        j = k0 + (uint32_t)(__ffs(acc) - 1);
-                        acc &= acc - 1;
-                        row = isb ? rb : ra;
-                        const uint64_t s0 = isb ? b0 : a0, s1 = isb ? b1 : a1, s2 = isb ? b2 : a2;
-                        m = (((uint32_t)s0 & ~sm.dp[0][j]) | ((uint32_t)(s0 >> 32) & ~sm.dp[1][j]) |
-                             ((uint32_t)s1 & ~sm.dp[2][j]) | ((uint32_t)(s1 >> 32) & ~sm.dp[3][j]) |
-                             ((uint32_t)s2 & ~sm.dp[4][j]) | ((uint32_t)(s2 >> 32) & ~sm.dp[5][j])) == 0;
-                    }
-                    const uint32_t bm = __ballot_sync(0xffffffffu, m);
-                    if (bm) {
-                        st_matched += __popc(bm);
-                        emit_keys(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane, sm.pend[warp], npend);
-                    }
-                }
-            }
-            st_checks += nq * (vend > u0 ? min((uint32_t)kDenseRows, vend - u0) : 0u);
         }
         __syncthreads();
     }
@@ -1536,8 +1504,7 @@ ScanFn scan_fn(int variant) {
         case 10: return k_dense<true, 1>;   // unfiltered dense scan, bulk-copy (TMA) staged rows
         case 11: return k_dense<false, 0>;
         case 12: return k_dense<true, 0>;
-        case 13: return k_dense<false, 5>;  // 9 + register prefetch of the next unit
-        case 14: return k_scan<4, false, false, true, 7, false, 9>;  // 8 + lazy row loads
+        case 13: return k_dense<false, 5>;  // 9 with four rows per lane
         default: return k_scan<4, false>;
     }
 }

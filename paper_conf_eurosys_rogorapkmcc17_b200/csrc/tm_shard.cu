@@ -217,7 +217,9 @@ std::vector<uint64_t> sample_routes(tm_db *db, const std::vector<Partition> &par
 
 std::vector<uint32_t> plan_shards(tm_db *db, const std::vector<Partition> &parts) {
     const uint32_t G = std::max(1u, db->cfg.n_shards);
-    if (G <= 1 || db->cfg.shard_mode == TM_SHARD_REPLICATED) return std::vector<uint32_t>(parts.size(), 0);
+    if (G <= 1) return std::vector<uint32_t>(parts.size(), 0);
+    // replicated: this handle keeps every partition
+    if (db->cfg.shard_mode == TM_SHARD_REPLICATED) return std::vector<uint32_t>(parts.size(), db->cfg.shard);
     const std::vector<uint64_t> routed = sample_routes(db, parts, db->stream);
     std::vector<double> w(parts.size(), 0.0);
     double W = 0;
@@ -293,7 +295,7 @@ tm_status tm_partition_host(const uint64_t *sigs, uint64_t n, uint32_t max_parti
     if ((n && !sigs) || !masks_out || !sizes_out || !n_parts_out || !n_unique_out) fail(TM_EINVAL, "NULL argument");
     if (max_partition == 0) max_partition = TM_DEFAULT_MAX_PARTITION;
     if (max_partition == TM_AUTO_MAX_PARTITION)  // reading R8b, as tm_build
-        max_partition = (uint32_t)std::min<uint64_t>(200000, std::max<uint64_t>(5000, n / 10000));
+        max_partition = (uint32_t)std::min<uint64_t>(200000, std::max<uint64_t>(5000, n / 30000));
     std::vector<Sig> v(n);
     for (uint64_t i = 0; i < n; ++i) v[i] = Sig{{sigs[3 * i], sigs[3 * i + 1], sigs[3 * i + 2]}};
     auto lt = [](const Sig &a, const Sig &b) {

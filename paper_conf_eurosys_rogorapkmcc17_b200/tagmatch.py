@@ -99,7 +99,8 @@ EXPORTS = ["tm_build", "tm_match_batch", "tm_match_batch_csr", "tm_match_batch_d
            "tm_owner_range", "tm_shard_plan", "tm_exchange_plan", "tm_group_size", "tm_group_member", "tm_partition_host", "tm_last_result", "tm_shard_counts",
            "tm_shard_merge", "tm_nccl_unique_id", "tm_comm_init", "tm_match_batch_sharded_device",
            "tm_stream_open", "tm_stream_submit", "tm_stream_poll", "tm_stream_result_free", "tm_stream_flush",
-           "tm_stream_replay", "tm_stream_close"]
+           "tm_stream_replay", "tm_stream_close", "tm_create", "tm_add_set", "tm_remove_set", "tm_add_sets",
+           "tm_consolidate", "tm_pending"]
 
 _lib = None
 
@@ -158,6 +159,14 @@ def load(path: str = LIB_PATH):
                        ("tm_stream_poll", [vp, i32, P(tm_stream_result)]),
                        ("tm_stream_flush", [vp]),
                        ("tm_stream_replay", [vp, P(tm_tagsets), vp])]:
+        getattr(L, name).restype = ctypes.c_int
+        getattr(L, name).argtypes = args
+    for name, args in [("tm_create", [P(tm_config), P(vp)]),
+                       ("tm_add_set", [vp, vp, vp, u64, u32]),
+                       ("tm_remove_set", [vp, vp, vp, u64, u32]),
+                       ("tm_add_sets", [vp, P(tm_tagsets), vp, vp]),
+                       ("tm_consolidate", [vp]),
+                       ("tm_pending", [vp, vp, vp])]:
         getattr(L, name).restype = ctypes.c_int
         getattr(L, name).argtypes = args
     L.tm_stream_result_free.argtypes = [P(tm_stream_result)]
@@ -242,6 +251,54 @@ class Database:
                           ctypes.byref(cfg), ctypes.byref(h)))
         self.h = h
         del self._sets, ids, smp  # inputs are not retained by the library
+
+    @classmethod
+    def create(cls, max_partition=0, device=-1, tile_filter=0, row_order=0, exact=0, n_gpus=0, shard_mode=0,
+               device_ids=None):
+        """tm_create: an empty mutable database (add_set / remove_set, then consolidate; Table 2)."""
+        self = cls.__new__(cls)
+        cfg = make_config(max_partition, device, 1, 0, tile_filter, row_order, exact, n_gpus, shard_mode)
+        ids = None
+        if device_ids is not None:
+            ids = np.ascontiguousarray(device_ids, dtype=np.int32)
+            cfg.device_ids = ctypes.c_void_p(ids.ctypes.data)
+        h = ctypes.c_void_p()
+        _check(load().tm_create(ctypes.byref(cfg), ctypes.byref(h)))
+        self.h = h
+        return self
+
+    @staticmethod
+    def _tags(tags):
+        b = b"".join(tags)
+        off = np.zeros(len(tags) + 1, np.uint64)
+        if tags:
+            off[1:] = np.cumsum([len(t) for t in tags])
+        buf = np.frombuffer(b, np.uint8) if b else np.zeros(1, np.uint8)
+        return buf, off
+
+    def add_set(self, tags: list[bytes], key: int):
+        buf, off = self._tags(tags)
+        _check(load().tm_add_set(self.h, _ptr(buf), _ptr(off), len(tags), key))
+
+    def remove_set(self, tags: list[bytes], key: int):
+        buf, off = self._tags(tags)
+        _check(load().tm_remove_set(self.h, _ptr(buf), _ptr(off), len(tags), key))
+
+    def add_sets(self, sets, key_off=None, keys=None):
+        s = sets if isinstance(sets, HostTagSets) else HostTagSets.of(sets)
+        ko = None if key_off is None else np.ascontiguousarray(key_off, dtype=np.uint64)
+        ks = np.ascontiguousarray(keys if keys is not None else np.zeros(0), dtype=np.uint32)
+        _check(load().tm_add_sets(self.h, ctypes.byref(s.c), _ptr(ko) if ko is not None else None,
+                                  _ptr(ks) if ks.size else None))
+
+    def consolidate(self):
+        _check(load().tm_consolidate(self.h))
+
+    def pending(self) -> tuple[int, int]:
+        """(staged operations, live entry instances) of a mutable handle."""
+        a, b = ctypes.c_uint64(), ctypes.c_uint64()
+        _check(load().tm_pending(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return a.value, b.value
 
     def match_batch(self, queries, unique: bool) -> tuple[np.ndarray, np.ndarray]:
         """tm_match_batch: host queries -> sorted (query, key) arrays (copies out of pinned memory)."""
