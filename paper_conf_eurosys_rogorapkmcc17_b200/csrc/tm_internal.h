@@ -31,7 +31,7 @@ constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 2
 constexpr int kScanVariants = 14;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {8, 5};  // variants the handle times on its first calls (first = default); 0-4 never won
 constexpr int kTuneN = 2;
-constexpr int kTuneDense[] = {9, 13};  // tables without a pre-filter (tile_filter = 2): the dense scan
+constexpr int kTuneDense[] = {13, 9};  // tables without a pre-filter (tile_filter = 2): the dense scan
 constexpr int kTuneMinQ = 4096;     // smaller calls are not tuned (default variant kTune[0])
 
 struct DevCounters {            // zeroed at the start of every match call

@@ -21,12 +21,20 @@
 
 namespace tmb {
 
+struct VecHash {
+    size_t operator()(const std::vector<uint32_t> &v) const {
+        uint64_t h = 0x9e3779b97f4a7c15ULL ^ v.size();
+        for (uint32_t x : v) h = (h ^ x) * 0x100000001b3ULL;
+        return (size_t)(h ^ (h >> 29));
+    }
+};
+
 struct Store {
     std::unordered_map<std::string, uint32_t> vocab_id;  // tag string -> id
     std::vector<std::string> vocab;                       // id -> tag string
-    std::map<std::vector<uint32_t>, uint32_t> set_id;     // canonical set (sorted distinct ids) -> set id
+    std::unordered_map<std::vector<uint32_t>, uint32_t, VecHash> set_id;  // canonical set -> set id
     std::vector<const std::vector<uint32_t> *> sets;      // set id -> canonical set (owned by set_id)
-    std::map<std::pair<uint32_t, uint32_t>, uint64_t> live;  // (set id, key) -> multiplicity
+    std::unordered_map<uint64_t, uint64_t> live;          // (set id << 32 | key) -> multiplicity
     struct Op {
         bool add;
         uint32_t set;
@@ -90,12 +98,15 @@ void live_input(const Store &st, std::vector<uint8_t> &vb, std::vector<uint64_t>
         vo.push_back(vb.size());
     }
     soff.assign(1, 0);
-    for (const auto &e : st.live) {
-        const std::vector<uint32_t> &ids = *st.sets[e.first.first];
+    // entries in (set id, key) order: a deterministic table for a given multiset
+    std::vector<std::pair<uint64_t, uint64_t>> ent(st.live.begin(), st.live.end());
+    std::sort(ent.begin(), ent.end());
+    for (const auto &e : ent) {
+        const std::vector<uint32_t> &ids = *st.sets[e.first >> 32];
         for (uint64_t m = 0; m < e.second; ++m) {
             tidx.insert(tidx.end(), ids.begin(), ids.end());
             soff.push_back(tidx.size());
-            keys.push_back(e.first.second);
+            keys.push_back((uint32_t)e.first);
         }
     }
 }
@@ -194,7 +205,7 @@ tm_status tm_consolidate(tm_db *db) {
     // apply the temporary index in call order to a copy (the handle is unchanged on failure)
     auto live = st.live;
     for (const tmb::Store::Op &op : st.staged) {
-        const auto k = std::make_pair(op.set, op.key);
+        const uint64_t k = (uint64_t)op.set << 32 | op.key;
         if (op.add) {
             ++live[k];
         } else {

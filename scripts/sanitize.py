@@ -29,7 +29,7 @@ def check(db, q, db_sig, wl, unique, what):
 
 
 def main():
-    variants = (sys.argv[1] if len(sys.argv) > 1 else "0,1,2,3,4,5,6,7,8,9,10,11,12").split(",")
+    variants = (sys.argv[1] if len(sys.argv) > 1 else "0,1,2,3,4,5,6,7,8,9,10,11,12,13").split(",")
     big = int(sys.argv[2]) if len(sys.argv) > 2 else 100_000
     cases = [("C1", tmgen.config("C1"), [(tmb.TM_NO_PARTITIONING, 2), (500, 1), (500, 0)]),
              (f"{big}", tmgen.generate(big, 2000, seed=11, max_partition=5000), [(5000, 1)])]
@@ -45,6 +45,19 @@ def main():
                     small = wl.queries.subset(np.arange(5))
                     check(db, small, db_sig, wl, False, f"{name} maxp={mp} filter={filt} var={v} Q=5")
     os.environ.pop("TM_SCAN_VARIANT", None)
+    # in-process multi-GPU handles (peer-copy exchange, owner merge) and a mutable handle
+    wl = tmgen.generate(big, 2000, seed=12, max_partition=5000)
+    db_sig = o2.encode(wl.db)
+    for mode in (0, 1):
+        with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=5000, tile_filter=1, row_order=1, n_gpus=2,
+                          device_ids=[0, 0], shard_mode=mode) as db:
+            for unique in (False, True):
+                check(db, wl.queries, db_sig, wl, unique, f"group mode={mode} u={unique}")
+    db = tmb.Database.create(max_partition=5000, tile_filter=1, row_order=1)
+    db.add_sets(wl.db, wl.key_off, wl.keys)
+    db.consolidate()
+    check(db, wl.queries, db_sig, wl, False, "mutable: add_sets + consolidate")
+    db.close()
     print("sanitize run complete")
 
 
