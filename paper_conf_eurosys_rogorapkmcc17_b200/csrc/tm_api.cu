@@ -150,6 +150,7 @@ void *cub_tmp(tm_db *db, size_t bytes) {
 // Every query of the batch is encoded; queries [qlo, qlo + qn) are matched (the share of one GPU
 // of a replicated multi-GPU database; default: all), with their batch-global indices.
 uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, uint64_t qlo, uint64_t qn) {
+    NvtxRange nv_call("tm: match (S1-S8)");
     tm_stats_t &st = db->st;
     const uint64_t Qall = q->n_sets;
     if (qlo > Qall) qlo = Qall;
@@ -165,7 +166,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
     db->last_qn = Qm;
     if (Qm == 0 || P == 0) return 0;
     const uint64_t Q = Qall;                       // encoded (and the sort width)
-    const uint64_t NB = route_blocks(Qm);          // route blocks of 512 queries
+    const uint64_t NB = route_blocks(Qm);          // route blocks of 384 queries
     const uint64_t n_words = (uint64_t)P * NB;    // (partition, route block) counts
     uint32_t launches = 0, cub_calls = 0;
 
@@ -173,8 +174,9 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
     DevCounters *ctr = db->ctr.as<DevCounters>();
     if (!db->wsel_ok) {  // pre-check word per row (scan variant 5), once per database
         db->wsel.ensure(std::max<uint64_t>(db->n_rows, 1));
+        db->wwords.ensure(std::max<uint64_t>(db->n_rows, 1) * 8);
         TMCK(launch_word_select(db->planes.as<uint64_t>(), db->tand.as<uint64_t>(), db->n_rows,
-                                db->wsel.as<uint8_t>(), s));
+                                db->wsel.as<uint8_t>(), db->wwords.as<uint2>(), s));
         db->wsel_ok = true;
     }
     TMCK(cudaEventRecord(db->ev[0], s));
@@ -257,6 +259,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
         sp.ctr = ctr;
         sp.filter = db->cfg.tile_filter;
         sp.wsel = db->wsel.as<uint8_t>();
+        sp.wwords = db->wwords.as<uint2>();
         sp.range_rows = range_rows;
         sp.one = 1;
         // variant: TM_SCAN_VARIANT if set; else a call whose partition batches are all small
@@ -410,6 +413,7 @@ tm_status translate(const CudaFail &f) {
 }
 
 void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys) {
+    NvtxRange nv_build("tm: build / consolidate");
     auto t0 = std::chrono::steady_clock::now();
     const bool trace = getenv("TM_TRACE_BUILD") != nullptr;
     auto mark = [&](const char *what) {
@@ -623,7 +627,7 @@ void destroy_db(tm_db *db) {
         shard_destroy(db);
     } catch (...) {
     }
-    for (DevBuf *b : {&db->planes, &db->tand, &db->wsel, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
+    for (DevBuf *b : {&db->planes, &db->tand, &db->wsel, &db->wwords, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
                       &db->in_voff, &db->in_tidx, &db->in_soff, &db->vsig, &db->qplanes, &db->bm, &db->word_off,
                       &db->qidx, &db->qoff, &db->item_cnt, &db->item_off, &db->out, &db->out_alt, &db->res_q,
                       &db->res_k, &db->res_off, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,

@@ -2,6 +2,7 @@
 #pragma once
 
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <functional>
@@ -95,6 +96,15 @@ struct DeviceGuard {
 
 extern thread_local std::string g_err;
 
+// NVTX range for the duration of a scope (stage names in nsys / ncu timelines; free when no
+// tool is attached).
+struct NvtxRange {
+    explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange &) = delete;
+    NvtxRange &operator=(const NvtxRange &) = delete;
+};
+
 }  // namespace tmb
 
 using namespace tmb;
@@ -129,6 +139,7 @@ struct tm_db {
     DevBuf planes;   // 3 x rows u64
     DevBuf tand;     // 3 x (rows / 32) u64: AND of each tile's real rows
     DevBuf wsel;     // rows u8: pre-check word per row (scan variant 5), made on first use
+    DevBuf wwords;   // rows x uint2: those two words (scan variant 14)
     bool wsel_ok = false;
     DevBuf key_off;  // rows + 1 u32
     DevBuf keys;     // K u32

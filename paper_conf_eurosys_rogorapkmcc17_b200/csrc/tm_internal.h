@@ -28,7 +28,7 @@ constexpr int kScanWarps = 4;      // warps per CTA
 constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch); 640 fits 7 CTAs/SM of shared memory and measured 1.3% faster than 512 (profiles/r1v34_ab.txt)
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
-constexpr int kScanVariants = 14;    // k_scan variants (TM_SCAN_VARIANT)
+constexpr int kScanVariants = 15;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {8, 5};  // variants the handle times on its first calls (first = default); 0-4 never won
 constexpr int kTuneN = 2;
 constexpr int kTuneDense[] = {13, 9};  // tables without a pre-filter (tile_filter = 2): the dense scan
@@ -65,6 +65,7 @@ struct ScanParams {
     DevCounters *ctr;
     uint32_t filter;                  // 0 prefix, 1 AND, 2 none
     const uint8_t *wsel;              // [rows] pre-check word per row (variant 5)
+    const uint2 *wwords;              // [rows] the two pre-check words themselves (variant 14)
     uint32_t range_rows;              // rows per work item (multiple of 256)
     uint32_t one;                     // 1 (a run-time operand, so the FMA-pipe accumulate stays an IMAD)
 };
@@ -90,7 +91,7 @@ cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int varia
 int scan_grid(int device, int variant);
 int scan_variant_env();  // -1 = auto-tune
 cudaError_t launch_word_select(const uint64_t *planes, const uint64_t *tand, uint64_t rows, uint8_t *wsel,
-                               cudaStream_t s);
+                               uint2 *wwords, cudaStream_t s);
 cudaError_t launch_split(const uint64_t *pairs, uint64_t n, uint32_t *q, uint32_t *k, cudaStream_t s);
 // q_off[i] = base + (first pair of query qlo + i), i < nq; q_off[nq] = base + n
 cudaError_t launch_query_offsets(const uint64_t *pairs, uint64_t n, uint64_t qlo, uint64_t nq, uint64_t base,

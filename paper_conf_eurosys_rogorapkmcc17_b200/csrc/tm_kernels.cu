@@ -110,15 +110,20 @@ __global__ void k_encode_sets(const uint64_t *__restrict__ vsig, const uint32_t 
 //   Z[pos][i] = ballot over the 32 queries of word i of "bit pos of q is 0"   (pos = 64 w + j)
 // in shared memory; then lane l takes partition p = g + l and ORs Z[pos] over the one-bits pos
 // of its mask (a mask has ~2-5 bits): ~Z-OR is the 32-query routing word of (p, word i), for
-// all kRouteWB words at once (four LDS.128 per mask bit).  Per (partition, 32 queries) that is
+// all kRouteWB words at once (three LDS.128 per mask bit).  Per (partition, 32 queries) that is
 // a few instructions per LANE instead of a 6-op test per (partition, query): routing cost stays
 // small when MAX_P is small and partitions are many.
 // Two passes over the same function: count (per (partition, route block) counts, scanned into
 // the partition-major CSR offsets) and scatter (ascending query ids per partition).  Scratch:
-// 12 B per (partition, 512 queries) instead of a dense P x Q bitmap.
-constexpr int kRouteWB = 16;                 // query words per route block (one warp)
-constexpr int kRouteBlockQ = 32 * kRouteWB;  // 512 queries
-constexpr int kRouteWarps = 4;               // warps per CTA (48 KB of Z)
+// 12 B per (partition, 384 queries) instead of a dense P x Q bitmap.
+// Bank conflicts: lane l reads the Z row of its own mask bit, so the 8 lanes of an LDS.128 phase
+// hit data-dependent rows.  With 16-word rows (64 B) every row started on one of two bank quads
+// of a 128-B window (8 lanes on 2 quads: ~5-way conflicts, the router was LSU-bound: 10 ms at
+// 40K partitions); 12-word rows (48 B) put consecutive rows on different quads (pos x 3 mod 8),
+// so random rows spread over all 8.
+constexpr int kRouteWB = 12;                 // query words per route block (one warp)
+constexpr int kRouteBlockQ = 32 * kRouteWB;  // 384 queries
+constexpr int kRouteWarps = 4;               // warps per CTA (36 KB of Z)
 
 __device__ __forceinline__ void route_build_z(uint32_t *__restrict__ z, const uint64_t *__restrict__ q0,
                                               const uint64_t *__restrict__ q1, const uint64_t *__restrict__ q2,
@@ -546,10 +551,12 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // MINB: resident CTAs per SM the register allocator must allow (__launch_bounds__); shared memory
 // caps residency at 8 CTAs, which ptxas cannot see (the scan's shared memory is dynamic).
 // STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
-// OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>).
+// OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>); bit 4 = lean tile
+// set-up (the two pre-check words read from the build-time wwords plane, no per-lane selects).
 template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     constexpr bool kImad = (OPT & 1) != 0;
+    constexpr bool kLean = WORD1 && !STREAM && (OPT & 16) != 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -830,16 +837,27 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     g1 = sm.tmask[warp][1][t - t_first];
                     g2 = sm.tmask[warp][2][t - t_first];
                 }
-                // 32-bit halves of the lane's set (invalid lanes: all ones, never pass)
-                const uint32_t a0l = valid ? (uint32_t)s0 : ~0u, a0h = valid ? (uint32_t)(s0 >> 32) : ~0u;
-                const uint32_t a1l = valid ? (uint32_t)s1 : ~0u, a1h = valid ? (uint32_t)(s1 >> 32) : ~0u;
-                const uint32_t a2l = valid ? (uint32_t)s2 : ~0u, a2h = valid ? (uint32_t)(s2 >> 32) : ~0u;
+                // 32-bit halves of the lane's set (invalid lanes: all ones, never pass; the lean form
+                // relies on the pre-check mask of invalid lanes being cleared instead)
+                const uint32_t a0l = (kLean || valid) ? (uint32_t)s0 : ~0u, a0h = (kLean || valid) ? (uint32_t)(s0 >> 32) : ~0u;
+                const uint32_t a1l = (kLean || valid) ? (uint32_t)s1 : ~0u, a1h = (kLean || valid) ? (uint32_t)(s1 >> 32) : ~0u;
+                const uint32_t a2l = (kLean || valid) ? (uint32_t)s2 : ~0u, a2h = (kLean || valid) ? (uint32_t)(s2 >> 32) : ~0u;
                 if constexpr (WORD1) {
-                    const uint32_t wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
+                    uint32_t wsel, aw, aw2;
+                    if constexpr (kLean) {
+                        // the row's two pre-check words, precomputed at build (rows are padded to whole
+                        // tiles, so every lane may load; invalid lanes' acc is cleared below)
+                        wsel = (uint32_t)__ldg(p.wsel + row);
+                        const uint2 ww = __ldg(p.wwords + row);
+                        aw = ww.x;
+                        aw2 = ww.y;
+                    } else {
+                        wsel = valid ? (uint32_t)__ldg(p.wsel + row) : 0x10u;
+                        // branch-free word select: block wl >> 1, half wl & 1 (invalid lanes: all ones)
+                        aw = pick_word(s0, s1, s2, wsel & 15u, valid);
+                        aw2 = pick_word(s0, s1, s2, wsel >> 4, valid);
+                    }
                     const uint32_t wl = wsel & 15u, wl2 = wsel >> 4;
-                    // branch-free word select: block wl >> 1, half wl & 1 (invalid lanes: all ones)
-                    const uint32_t aw = pick_word(s0, s1, s2, wl, valid);
-                    const uint32_t aw2 = pick_word(s0, s1, s2, wl2, valid);
                     st_tests += na;
                     const uint32_t *swp = sm.sw[warp][0];
                     const uint32_t sw_base = (uint32_t)__cvta_generic_to_shared(swp);
@@ -1414,7 +1432,7 @@ __global__ void k_iota(uint32_t *v, uint64_t n) {
 __global__ void k_word_select(const uint64_t *__restrict__ w0, const uint64_t *__restrict__ w1,
                               const uint64_t *__restrict__ w2, const uint64_t *__restrict__ t0,
                               const uint64_t *__restrict__ t1, const uint64_t *__restrict__ t2, uint64_t rows,
-                              uint8_t *__restrict__ wsel) {
+                              uint8_t *__restrict__ wsel, uint2 *__restrict__ wwords) {
     uint64_t r = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (r >= rows) return;
     const uint64_t t = r / kTile;
@@ -1434,6 +1452,9 @@ __global__ void k_word_select(const uint64_t *__restrict__ w0, const uint64_t *_
         }
     }
     wsel[r] = (uint8_t)(best | (second << 4));
+    // the two words themselves (the lean scan reads them instead of selecting them per tile)
+    const uint64_t v[3] = {w0[r], w1[r], w2[r]};
+    wwords[r] = make_uint2((uint32_t)(v[best >> 1] >> (32 * (best & 1))), (uint32_t)(v[second >> 1] >> (32 * (second & 1))));
 }
 
 struct WidenAt {
@@ -1470,7 +1491,7 @@ cudaError_t launch_route(int pass, const uint64_t *masks, uint32_t n_parts, cons
                          uint32_t *qidx, unsigned long long cap, cudaStream_t s, uint32_t qbase) {
     const uint64_t nb = route_blocks(n_q);
     if (!nb || !n_parts) return cudaSuccess;
-    const size_t smem = (size_t)kRouteWarps * 192 * kRouteWB * 4;  // 48 KB: within the default dynamic limit
+    const size_t smem = (size_t)kRouteWarps * 192 * kRouteWB * 4;  // 36 KB: within the default dynamic limit
     static_assert((size_t)kRouteWarps * 192 * kRouteWB * 4 <= 48 * 1024, "route Z needs the opt-in attribute");
     auto f = pass == 0 ? k_route<0> : k_route<1>;
     f<<<grid_for(nb, kRouteWarps), kRouteWarps * 32, smem, s>>>(masks, n_parts, q0, q1, q2, n_q, nb, counts, off, qidx,
@@ -1505,6 +1526,7 @@ ScanFn scan_fn(int variant) {
         case 11: return k_dense<false, 0>;
         case 12: return k_dense<true, 0>;
         case 13: return k_dense<false, 5>;  // 9 with four rows per lane
+        case 14: return k_scan<4, false, false, true, 7, false, 17>;  // 8 + lean tile set-up
         default: return k_scan<4, false>;
     }
 }
@@ -1557,11 +1579,11 @@ cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int varia
 }
 
 cudaError_t launch_word_select(const uint64_t *planes, const uint64_t *tand, uint64_t rows, uint8_t *wsel,
-                               cudaStream_t s) {
+                               uint2 *wwords, cudaStream_t s) {
     if (!rows) return cudaSuccess;
     const uint64_t nt = rows / kTile;
     k_word_select<<<grid_for(rows, 256), 256, 0, s>>>(planes, planes + rows, planes + 2 * rows, tand, tand + nt,
-                                                      tand + 2 * nt, rows, wsel);
+                                                      tand + 2 * nt, rows, wsel, wwords);
     return cudaGetLastError();
 }
 

@@ -210,7 +210,8 @@ def test_c2_full_parity(c2, c2_oracle, layout):
     assert np.unique(got[0]).size == wl.queries.n_sets
 
 
-@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9", "10", "11", "12", "13"])
+@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9", "10", "11", "12", "13",
+                                     "14"])
 def test_c2_every_scan_variant(c2, c2_oracle, variant, monkeypatch):
     """Every scan-kernel variant (TM_SCAN_VARIANT) gives the oracle's
     pairs at C2, in the layout bench.py times (balanced splits + AND masks)."""
