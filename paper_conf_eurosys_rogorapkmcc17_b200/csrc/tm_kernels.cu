@@ -156,7 +156,7 @@ __device__ __forceinline__ void route_build_z(uint32_t *__restrict__ z, const ui
 // PASS 0: counts[p * NB + blk] = routed queries of partition p in route block blk.
 // PASS 1: scatter the routed query ids of (p, blk) at off[p * NB + blk] (ascending query order).
 template <int PASS>
-__global__ void __launch_bounds__(kRouteWarps * 32) k_route(const uint64_t *__restrict__ masks, uint32_t n_parts,
+__global__ void __launch_bounds__(kRouteWarps * 32, 6) k_route(const uint64_t *__restrict__ masks, uint32_t n_parts,
                                                             const uint64_t *__restrict__ q0,
                                                             const uint64_t *__restrict__ q1,
                                                             const uint64_t *__restrict__ q2, uint64_t n_q,
@@ -174,14 +174,30 @@ __global__ void __launch_bounds__(kRouteWarps * 32) k_route(const uint64_t *__re
     __syncwarp();
     // valid-query mask of each word of the block (warp-uniform)
     const uint64_t nvq = n_q - qb;  // > 0
-    for (uint32_t g = 0; g < n_parts; g += 32) {
-        const uint32_t p = g + lane;
-        uint64_t m[3] = {0, 0, 0};
+    // masks of the lane's partition in the next group are loaded one group ahead (their L2 latency
+    // would otherwise serialise with every group's short bit loop)
+    auto load_mask = [&](uint32_t p, uint64_t (&m)[3]) {
+        m[0] = m[1] = m[2] = 0;
         if (p < n_parts) {
             m[0] = __ldg(masks + 3 * (uint64_t)p);
             m[1] = __ldg(masks + 3 * (uint64_t)p + 1);
             m[2] = __ldg(masks + 3 * (uint64_t)p + 2);
         }
+    };
+    // PASS 1: the lane's CSR offset, likewise one group ahead
+    auto load_off = [&](uint32_t p) -> unsigned long long {
+        if constexpr (PASS == 1) return p < n_parts ? __ldg(off + (uint64_t)p * n_blocks + blk) : 0ULL;
+        return 0ULL;
+    };
+    uint64_t mn[3];
+    load_mask(lane, mn);
+    unsigned long long on = load_off(lane);
+    for (uint32_t g = 0; g < n_parts; g += 32) {
+        const uint32_t p = g + lane;
+        uint64_t m[3] = {mn[0], mn[1], mn[2]};
+        const unsigned long long o_here = on;
+        load_mask(g + 32 + lane, mn);
+        on = load_off(g + 32 + lane);
         uint32_t acc[kRouteWB];
 #pragma unroll
         for (int i = 0; i < kRouteWB; ++i) acc[i] = 0;
@@ -213,7 +229,7 @@ __global__ void __launch_bounds__(kRouteWarps * 32) k_route(const uint64_t *__re
             }
             counts[(uint64_t)p * n_blocks + blk] = c;
         } else {
-            unsigned long long o = off[(uint64_t)p * n_blocks + blk];
+            unsigned long long o = o_here;
 #pragma unroll
             for (int i = 0; i < kRouteWB; ++i) {
                 const uint64_t lo = 32ULL * i;
@@ -1238,26 +1254,40 @@ __global__ void __launch_bounds__(kScanWarps * 32, BULK ? 6 : 7) k_dense(const S
                 }
             }
         };
+        // kLeanD (direct loads): the rows' pre-check words come from the build-time wwords plane
+        constexpr bool kLeanD = !BULK && (OPT & 16) != 0;
         // direct loads of rows (r, r + 1) of a lane (all-ones past the range)
-        auto load_pair = [&](uint32_t r, ulonglong2 &x0, ulonglong2 &x1, ulonglong2 &x2, uint32_t &xw) {
+        auto load_pair = [&](uint32_t r, ulonglong2 &x0, ulonglong2 &x1, ulonglong2 &x2, uint32_t &xw, uint4 &ww) {
             x0 = x1 = x2 = make_ulonglong2(~0ULL, ~0ULL);
             xw = 0x1010u;
+            ww = make_uint4(~0u, ~0u, ~0u, ~0u);
             if (r < rhi) {
                 x0 = ldg_stream2(p.w0 + r);
                 x1 = ldg_stream2(p.w1 + r);
                 x2 = ldg_stream2(p.w2 + r);
                 xw = __ldg(reinterpret_cast<const unsigned short *>(p.wsel + r));
+                if constexpr (kLeanD) ww = __ldg(reinterpret_cast<const uint4 *>(p.wwords + r));
             }
         };
         // the two-word pre-check of rows (u0 + 2 lane, + 1) against the batch, full checks, emission
         auto check_pair = [&](const ulonglong2 v0, const ulonglong2 v1, const ulonglong2 v2, const uint32_t wab,
-                              const uint32_t u0) {
+                              const uint32_t u0, const uint4 ww) {
                 const uint32_t ra = u0 + 2 * (uint32_t)lane, rb = ra + 1;
                 const uint64_t a0 = v0.x, a1 = v1.x, a2 = v2.x, b0 = v0.y, b1 = v1.y, b2 = v2.y;
                 const bool va = ra < vend, vb = rb < vend;
                 const uint32_t wa = wab & 0xffu, wb = wab >> 8;
-                const uint32_t xa = pick_word(a0, a1, a2, wa & 15u, va), ya = pick_word(a0, a1, a2, wa >> 4, va);
-                const uint32_t xb = pick_word(b0, b1, b2, wb & 15u, vb), yb = pick_word(b0, b1, b2, wb >> 4, vb);
+                uint32_t xa, ya, xb, yb;
+                if constexpr (kLeanD) {  // invalid rows: their pass masks are cleared below
+                    xa = ww.x;
+                    ya = ww.y;
+                    xb = ww.z;
+                    yb = ww.w;
+                } else {
+                    xa = pick_word(a0, a1, a2, wa & 15u, va);
+                    ya = pick_word(a0, a1, a2, wa >> 4, va);
+                    xb = pick_word(b0, b1, b2, wb & 15u, vb);
+                    yb = pick_word(b0, b1, b2, wb >> 4, vb);
+                }
                 const uint32_t pxa = dp_base + (wa & 15u) * kPl, pya = dp_base + (wa >> 4) * kPl;
                 const uint32_t pxb = dp_base + (wb & 15u) * kPl, pyb = dp_base + (wb >> 4) * kPl;
                 for (uint32_t k0 = 0; k0 < nq; k0 += 32) {
@@ -1339,24 +1369,26 @@ __global__ void __launch_bounds__(kScanWarps * 32, BULK ? 6 : 7) k_dense(const S
                 ring1 = ring2;
                 ring2 = nu;
                 si = si == kDenseStages - 1 ? 0 : si + 1;
-                check_pair(v0, v1, v2, wab, rlo + u * kDenseRows);
+                check_pair(v0, v1, v2, wab, rlo + u * kDenseRows, make_uint4(0u, 0u, 0u, 0u));
             } else if constexpr (kRows4) {
                 const uint32_t u = take();
                 if (u >= nunit) break;
                 const uint32_t u0 = rlo + u * kUnitRows;
                 ulonglong2 v0, v1, v2, y0, y1, y2;
                 uint32_t wab, wcd;
-                load_pair(u0 + 2 * (uint32_t)lane, v0, v1, v2, wab);  // 96 B per lane in flight
-                load_pair(u0 + kDenseRows + 2 * (uint32_t)lane, y0, y1, y2, wcd);
-                check_pair(v0, v1, v2, wab, u0);
-                check_pair(y0, y1, y2, wcd, u0 + kDenseRows);
+                uint4 wwa, wwc;
+                load_pair(u0 + 2 * (uint32_t)lane, v0, v1, v2, wab, wwa);  // 96 B per lane in flight
+                load_pair(u0 + kDenseRows + 2 * (uint32_t)lane, y0, y1, y2, wcd, wwc);
+                check_pair(v0, v1, v2, wab, u0, wwa);
+                check_pair(y0, y1, y2, wcd, u0 + kDenseRows, wwc);
             } else {
                 const uint32_t u = take();
                 if (u >= nunit) break;
                 ulonglong2 v0, v1, v2;
                 uint32_t wab;
-                load_pair(rlo + u * kDenseRows + 2 * (uint32_t)lane, v0, v1, v2, wab);
-                check_pair(v0, v1, v2, wab, rlo + u * kDenseRows);
+                uint4 ww;
+                load_pair(rlo + u * kDenseRows + 2 * (uint32_t)lane, v0, v1, v2, wab, ww);
+                check_pair(v0, v1, v2, wab, rlo + u * kDenseRows, ww);
             }
         }
         __syncthreads();
@@ -1527,13 +1559,14 @@ ScanFn scan_fn(int variant) {
         case 12: return k_dense<true, 0>;
         case 13: return k_dense<false, 5>;  // 9 with four rows per lane
         case 14: return k_scan<4, false, false, true, 7, false, 17>;  // 8 + lean tile set-up
+        case 15: return k_dense<false, 21>;  // 13 + the build-time pre-check words (no selects)
         default: return k_scan<4, false>;
     }
 }
 }  // namespace
 
 size_t scan_smem(int variant) {
-    if (variant == 9 || variant == 11 || variant == 13) return sizeof(DenseSmemBase);
+    if (variant == 9 || variant == 11 || variant == 13 || variant == 15) return sizeof(DenseSmemBase);
 
     if (variant == 10 || variant == 12) return sizeof(DenseSmemBulk);
     return (variant == 6 || variant == 7) ? sizeof(StreamSmem) : sizeof(ScanSmem);
