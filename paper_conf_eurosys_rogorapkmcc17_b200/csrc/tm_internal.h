@@ -29,7 +29,7 @@ constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
 constexpr int kScanVariants = 16;    // k_scan variants (TM_SCAN_VARIANT)
-constexpr int kTune[] = {8, 5};  // variants the handle times on its first calls (first = default); 0-4 never won
+constexpr int kTune[] = {14, 8};  // variants the handle times on its first calls (first = default)
 constexpr int kTuneN = 2;
 constexpr int kTuneDense[] = {13, 9};  // tables without a pre-filter (tile_filter = 2): the dense scan
 constexpr int kTuneMinQ = 4096;     // smaller calls are not tuned (default variant kTune[0])

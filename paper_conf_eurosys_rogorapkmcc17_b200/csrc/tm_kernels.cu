@@ -548,15 +548,8 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // check "amounts to a simple operation on each Bloom-filter block").
 // Filters: 0 = Alg. 4 common prefix of first/last row; 1 = AND of the rows
 // (precomputed per tile at build); 2 = none.
-// Survivor layout: FULL3 = false: one 16-B entry (blocks 0, 1) per survivor, up to
-// kSubB per pass, block 2 checked on a hit; FULL3 = true: two 16-B entries
-// (blocks 0, 1 | block 2, slot) per survivor, up to kSubB / 2 per pass, all
-// three blocks checked in the main loop.  U = survivors per loop iteration.
-// UNION2 (with FULL3 = false): survivors are first tested in pairs against the
-// OR of the pair's blocks 0-1 (a necessary condition: s within a implies s
-// within a|b), and individually only when some lane passes the pair test --
-// about 1 pair in 9 on the Twitter-like workload, so the check loop issues
-// ~40% fewer LOP3.
+// Without WORD1 (variant 0): level-B survivors are 16-B entries (blocks 0, 1), tested four per
+// iteration with one LDS.128 each, block 2 on a hit.
 // WORD1: per-lane word pre-check.  Every row carries a build-time choice of two of its six
 // 32-bit words (those with the most one-bits outside its tile's AND mask, k_word_select);
 // each lane tests its set's two words against those words of 4 survivors per LDS.128 pair
@@ -569,7 +562,7 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
 // OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>); bit 4 = lean tile
 // set-up (the two pre-check words read from the build-time wwords plane, no per-lane selects).
-template <int U, bool FULL3, bool UNION2 = false, bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
+template <bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     constexpr bool kImad = (OPT & 1) != 0;
     constexpr bool kLean = WORD1 && !STREAM && (OPT & 16) != 0;
@@ -590,9 +583,6 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
     uint4 *sbuf = sm.sbuf[warp];
     uint16_t *sbi = sm.sbi[warp];
     const uint32_t sb_addr = (uint32_t)__cvta_generic_to_shared(sbuf);
-    // level-B survivors per pass (UNION2: entries [0, 80), pair unions at [80, 120))
-    constexpr uint32_t kPiece = FULL3 ? kSubB / 2 : (UNION2 ? 80 : kSubB);
-    constexpr uint32_t kUnionBase = 80;
 
     for (;;) {
         if (lane == 0 && (st_tests | st_checks | st_matched)) {  // shared atomics: no global contention
@@ -962,8 +952,8 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     }
                     continue;
                 }
-                for (uint32_t pb = 0; pb < na; pb += kPiece) {
-                    const uint32_t pe = min(na, pb + kPiece);
+                for (uint32_t pb = 0; pb < na; pb += kSubB) {
+                    const uint32_t pe = min(na, pb + kSubB);
                     // ---- level B: level-A survivors that contain the tile's mask
                     uint32_t nb = 0;
                     for (uint32_t j = pb; j < pe; j += 32) {
@@ -981,105 +971,33 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                         const uint32_t b = __ballot_sync(0xffffffffu, ok);
                         if (ok) {
                             const uint32_t k = nb + __popc(b & lt_mask);
-                            if (FULL3) {
-                                sbuf[2 * k] = make_uint4((uint32_t)a0, (uint32_t)(a0 >> 32), (uint32_t)a1,
-                                                         (uint32_t)(a1 >> 32));
-                                sbuf[2 * k + 1] = make_uint4((uint32_t)a2, (uint32_t)(a2 >> 32), i, 0u);
-                            } else {
-                                sbuf[k] = make_uint4((uint32_t)a0, (uint32_t)(a0 >> 32), (uint32_t)a1,
-                                                     (uint32_t)(a1 >> 32));
-                                sbi[k] = (uint16_t)i;
-                            }
+                            sbuf[k] = make_uint4((uint32_t)a0, (uint32_t)(a0 >> 32), (uint32_t)a1, (uint32_t)(a1 >> 32));
+                            sbi[k] = (uint16_t)i;
                         }
                         nb += __popc(b);
                     }
                     st_tests += pe - pb;
                     st_checks += nb * nvalid;
-                    // pad to a multiple of U with zeros (masked by k < nb below)
-                    constexpr uint32_t kPad = UNION2 ? 8 : U;
-                    if ((uint32_t)lane < ((kPad - (nb % kPad)) % kPad)) {
-                        if (FULL3) {
-                            sbuf[2 * (nb + lane)] = make_uint4(0, 0, 0, 0);
-                            sbuf[2 * (nb + lane) + 1] = make_uint4(0, 0, 0, 0);
-                        } else {
-                            sbuf[nb + lane] = make_uint4(0, 0, 0, 0);
-                            sbi[nb + lane] = 0;
-                        }
+                    // pad to a multiple of 4 with zeros (masked by k < nb below)
+                    if ((uint32_t)lane < ((4 - (nb % 4)) % 4)) {
+                        sbuf[nb + lane] = make_uint4(0, 0, 0, 0);
+                        sbi[nb + lane] = 0;
                     }
                     __syncwarp();
-                    if (UNION2) {
-                        // ---- Alg. 3 with pair unions: 4 pairs (8 survivors) per iteration
-                        const uint32_t npair = (nb + 7) / 8 * 4;
-                        for (uint32_t i = lane; i < npair; i += 32) {
-                            const uint4 x = sbuf[2 * i], y = sbuf[2 * i + 1];
-                            sbuf[kUnionBase + i] = make_uint4(x.x | y.x, x.y | y.y, x.z | y.z, x.w | y.w);
+                    // ---- Alg. 3: 4 survivors per iteration against the warp's 32 sets, blocks 0-1
+                    // first (one LDS.128 each), block 2 only when some lane passed
+                    for (uint32_t k = 0; k < nb; k += 4) {
+                        bool h[4];
+#pragma unroll
+                        for (int j = 0; j < 4; ++j) {
+                            const uint4 v = lds128(sb_addr + (k + j) * 16);
+                            h[j] = ((a0l & ~v.x) | (a0h & ~v.y) | (a1l & ~v.z) | (a1h & ~v.w)) == 0;
                         }
-                        __syncwarp();
-                        for (uint32_t k = 0; k < nb; k += 8) {
-                            const uint32_t ua = sb_addr + (kUnionBase + k / 2) * 16;
-                            const uint4 u0 = lds128(ua), u1 = lds128(ua + 16), u2 = lds128(ua + 32),
-                                        u3 = lds128(ua + 48);
-                            bool hu[4];
-                            hu[0] = ((a0l & ~u0.x) | (a0h & ~u0.y) | (a1l & ~u0.z) | (a1h & ~u0.w)) == 0;
-                            hu[1] = ((a0l & ~u1.x) | (a0h & ~u1.y) | (a1l & ~u1.z) | (a1h & ~u1.w)) == 0;
-                            hu[2] = ((a0l & ~u2.x) | (a0h & ~u2.y) | (a1l & ~u2.z) | (a1h & ~u2.w)) == 0;
-                            hu[3] = ((a0l & ~u3.x) | (a0h & ~u3.y) | (a1l & ~u3.z) | (a1h & ~u3.w)) == 0;
-                            if (__any_sync(0xffffffffu, hu[0] | hu[1] | hu[2] | hu[3])) {
+                        if (__any_sync(0xffffffffu, (h[0] | h[1]) | (h[2] | h[3]))) {
 #pragma unroll
-                                for (int j = 0; j < 4; ++j) {
-                                    if (!__any_sync(0xffffffffu, hu[j])) continue;
-#pragma unroll
-                                    for (int t = 0; t < 2; ++t) {
-                                        const uint32_t e = k + 2 * j + t;
-                                        if (e >= nb) continue;
-                                        const uint4 v = lds128(sb_addr + e * 16);
-                                        const bool h = ((a0l & ~v.x) | (a0h & ~v.y) | (a1l & ~v.z) | (a1h & ~v.w)) == 0;
-                                        if (__any_sync(0xffffffffu, h))
-                                            check_block2(h, sbi[e], s2, row, sm, p, lane, st_matched, npend);
-                                    }
-                                }
-                            }
-                        }
-                        __syncwarp();
-                        continue;
-                    }
-                    // ---- Alg. 3: U survivors per iteration against the warp's 32 sets
-                    for (uint32_t k = 0; k < nb; k += U) {
-                        bool h[U];
-                        uint32_t slot[U];
-#pragma unroll
-                        for (int j = 0; j < U; ++j) {
-                            if (FULL3) {
-                                const uint32_t a = sb_addr + (k + j) * 32;
-                                const uint4 v = lds128(a), w = lds128(a + 16);
-                                h[j] = ((a0l & ~v.x) | (a0h & ~v.y) | (a1l & ~v.z) | (a1h & ~v.w) | (a2l & ~w.x) |
-                                        (a2h & ~w.y)) == 0;
-                                slot[j] = w.z;
-                            } else {
-                                const uint4 v = lds128(sb_addr + (k + j) * 16);
-                                h[j] = ((a0l & ~v.x) | (a0h & ~v.y) | (a1l & ~v.z) | (a1h & ~v.w)) == 0;
-                                slot[j] = 0;
-                            }
-                        }
-                        bool any = false;
-#pragma unroll
-                        for (int j = 0; j < U; ++j) any |= h[j];
-                        if (__any_sync(0xffffffffu, any)) {
-#pragma unroll
-                            for (int j = 0; j < U; ++j) {
-                                if (k + j < nb && __any_sync(0xffffffffu, h[j])) {
-                                    if (FULL3) {
-                                        const bool m = h[j] && valid;
-                                        const uint32_t bm = __ballot_sync(0xffffffffu, m);
-                                        if (bm) {
-                                            st_matched += __popc(bm);
-                                            emit_keys(m, bm, row, __ldg(sm.qid + slot[j]), p, lane, sm.pend[warp], npend);
-                                        }
-                                    } else {
-                                        check_block2(h[j], sbi[k + j], s2, row, sm, p, lane, st_matched, npend);
-                                    }
-                                }
-                            }
+                            for (int j = 0; j < 4; ++j)
+                                if (k + j < nb && __any_sync(0xffffffffu, h[j]))
+                                    check_block2(h[j], sbi[k + j], s2, row, sm, p, lane, st_matched, npend);
                         }
                     }
                     __syncwarp();
@@ -1542,25 +1460,24 @@ cudaError_t launch_items(const unsigned long long *word_off, uint64_t qw, const 
 namespace {
 using ScanFn = void (*)(const ScanParams);
 ScanFn scan_fn(int variant) {
+    // variants 1-4 of round 1 (8 survivors per iteration, all three blocks in the main loop, pair
+    // unions) never won a tuning class and were removed in round 2; their numbers stay unused
     switch (variant) {
-        case 1: return k_scan<8, false>;
-        case 2: return k_scan<4, true>;
-        case 3: return k_scan<8, true>;
-        case 4: return k_scan<4, false, true>;
+        case 0: return k_scan<false>;  // no word pre-check: 4 survivors per iteration, blocks 0-1 first
         // 72 registers and 7 CTAs/SM, no spills: 2.00 ms at C2 vs 2.10 ms with 64 registers and
         // 8 CTAs (spills) and 2.05 ms with 76 registers and 6 CTAs (profiles/r1v29_minb.txt)
-        case 5: return k_scan<4, false, false, true, 7>;
-        case 6: return k_scan<4, false, false, false, 8, true>;  // streaming only, direct check
-        case 7: return k_scan<4, false, false, true, 8, true>;   // streaming only, word pre-check
-        case 8: return k_scan<4, false, false, true, 7, false, 1>;  // 5 + pre-check accumulate on the FMA pipe
+        case 5: return k_scan<true, 7>;
+        case 6: return k_scan<false, 8, true>;   // streaming only, direct check
+        case 7: return k_scan<true, 8, true>;    // streaming only, word pre-check
+        case 8: return k_scan<true, 7, false, 1>;  // 5 + pre-check accumulate on the FMA pipe
         case 9: return k_dense<false, 1>;   // unfiltered dense scan, direct loads, FMA-pipe accumulate
         case 10: return k_dense<true, 1>;   // unfiltered dense scan, bulk-copy (TMA) staged rows
         case 11: return k_dense<false, 0>;
         case 12: return k_dense<true, 0>;
         case 13: return k_dense<false, 5>;  // 9 with four rows per lane
-        case 14: return k_scan<4, false, false, true, 7, false, 17>;  // 8 + lean tile set-up
+        case 14: return k_scan<true, 7, false, 17>;  // 8 + lean tile set-up (the default)
         case 15: return k_dense<false, 21>;  // 13 + the build-time pre-check words (no selects)
-        default: return k_scan<4, false>;
+        default: return nullptr;
     }
 }
 }  // namespace
@@ -1573,15 +1490,17 @@ size_t scan_smem(int variant) {
 }
 
 int scan_variant_env() {
-    // TM_SCAN_VARIANT forces a scan-kernel variant: 0 = 4 survivors per
-    // iteration, blocks 0-1 first; 1 = 8, blocks 0-1; 2 = 4, all three blocks; 3 = 8, all three;
-    // 4 = pair unions first; 5 = per-lane word pre-check (WORD1); 6 / 7 = streaming-only kernels
-    // (direct check / word pre-check; calls of <= kSmallBatch queries, else mapped to 0 / 5 by the
-    // caller).  Unset (-1): the handle tunes on its first calls.
+    // TM_SCAN_VARIANT forces a scan-kernel variant: 0 = no word pre-check;
+    // 5 = per-lane two-word pre-check (WORD1); 8 = 5 + FMA-pipe accumulate; 14 = 8 + lean tile
+    // set-up (default); 6 / 7 = streaming-only kernels (direct check / word pre-check; calls of
+    // <= kSmallBatch queries, else mapped to 0 / 5 by the caller); 9-13, 15 = the dense
+    // (unfiltered) scan (9 two rows per lane, 13 four, 10 / 12 bulk-copy staged, 11 / 12 without
+    // the FMA accumulate, 15 = 13 with build-time pre-check words).  Unset or unknown (-1): the
+    // handle tunes on its first calls.
     const char *e = getenv("TM_SCAN_VARIANT");
     if (!e) return -1;
     const int v = atoi(e);
-    return (v >= 0 && v < kScanVariants) ? v : -1;
+    return (v >= 0 && v < kScanVariants && scan_fn(v)) ? v : -1;
 }
 
 uint32_t range_rows_env(uint64_t n_rows) {
@@ -1599,6 +1518,7 @@ int scan_grid(int device, int variant) {
     int sms = 0, per = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
     ScanFn f = scan_fn(variant);
+    if (!f) return 0;  // unused variant number
     cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem(variant));
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, kScanWarps * 32, scan_smem(variant));
     if (per < 1) per = 1;

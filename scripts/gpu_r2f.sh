@@ -10,5 +10,5 @@ timeout 900 python scripts/build_time.py 1000000,5000000 > gpurun_out/${TAG}_bui
 for T in memcheck racecheck synccheck; do
   N=100000; [ $T != memcheck ] && N=20000
   timeout 1500 /usr/local/cuda/bin/compute-sanitizer --tool $T --error-exitcode 99 python scripts/sanitize.py \
-    0,1,2,3,4,5,6,7,8,9,10,11,12,13 $N > gpurun_out/${TAG}_sanitize_${T}.log 2>&1; echo "sanitize $T rc=$?"; tail -2 gpurun_out/${TAG}_sanitize_${T}.log
+    0,5,6,7,8,9,10,11,12,13,14,15 $N > gpurun_out/${TAG}_sanitize_${T}.log 2>&1; echo "sanitize $T rc=$?"; tail -2 gpurun_out/${TAG}_sanitize_${T}.log
 done

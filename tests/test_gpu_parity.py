@@ -210,7 +210,7 @@ def test_c2_full_parity(c2, c2_oracle, layout):
     assert np.unique(got[0]).size == wl.queries.n_sets
 
 
-@pytest.mark.parametrize("variant", ["0", "1", "2", "3", "4", "5", "6", "7", "8", "9", "10", "11", "12", "13",
+@pytest.mark.parametrize("variant", ["0", "5", "6", "7", "8", "9", "10", "11", "12", "13",
                                      "14", "15"])
 def test_c2_every_scan_variant(c2, c2_oracle, variant, monkeypatch):
     """Every scan-kernel variant (TM_SCAN_VARIANT) gives the oracle's
@@ -396,7 +396,7 @@ def test_variant_tuning_flag(c1, c2, c2_oracle, monkeypatch):
         assert flags[0] == 1 and 0 in flags, flags
         settled = flags.index(0)
         assert all(f == 0 for f in flags[settled:]) and len(set(variants[settled + 1:])) == 1, (flags, variants)
-        assert {8, 5} <= set(variants[:settled + 1]), variants   # kTune (tm_internal.h)
+        assert {14, 8} <= set(variants[:settled + 1]), variants   # kTune (tm_internal.h)
         db.match_batch(c2.queries.subset(np.arange(3)), False)    # streaming-only call
         assert db.stats()["tuning"] == 0
     monkeypatch.setenv("TM_SCAN_VARIANT", "5")
