@@ -262,6 +262,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
         sp.wwords = db->wwords.as<uint2>();
         sp.range_rows = range_rows;
         sp.one = 1;
+        sp.unit_target = unit_target_env();
         // variant: TM_SCAN_VARIANT if set; else a call whose partition batches are all small
         // (Q <= kSmallBatch) takes the streaming path only, in the streaming-only kernels (small
         // shared memory: 8 CTAs/SM) -- up to four queries checked directly (variant 6), 5-8

@@ -66,6 +66,7 @@ struct ScanParams {
     uint32_t filter;                  // 0 prefix, 1 AND, 2 none
     const uint8_t *wsel;              // [rows] pre-check word per row (variant 5)
     const uint2 *wwords;              // [rows] the two pre-check words themselves (variant 14)
+    uint32_t unit_target;             // filtered path: split items of fewer blocks to this many units
     uint32_t range_rows;              // rows per work item (multiple of 256)
     uint32_t one;                     // 1 (a run-time operand, so the FMA-pipe accumulate stays an IMAD)
 };
@@ -87,6 +88,7 @@ cudaError_t launch_items(const unsigned long long *word_off, uint64_t qw, const 
                          const uint32_t *part_n, uint32_t n_parts, unsigned long long *qoff,
                          unsigned long long *item_cnt, DevCounters *ctr, uint32_t range_rows, cudaStream_t s);
 uint32_t range_rows_env(uint64_t n_rows);  // TM_RANGE_ROWS (multiple of 256), else by table size
+uint32_t unit_target_env();                // TM_UNIT_TARGET, else kScanWarps
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant);
 int scan_grid(int device, int variant);
 int scan_variant_env();  // -1 = auto-tune

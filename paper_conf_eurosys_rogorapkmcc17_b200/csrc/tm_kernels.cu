@@ -758,7 +758,11 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
         const uint32_t nblock = (ntile + kBlockTiles - 1) / kBlockTiles;
         // unit = (256-row block, query sub-range), taken dynamically through unit_ctr;
         // few blocks: split the batch so every warp has work
-        const uint32_t nsplit = nblock >= (uint32_t)kScanWarps ? 1u : (uint32_t)kScanWarps / max(nblock, 1u);
+        // (a small item -- few blocks -- is split over query sub-ranges until it has p.unit_target
+        // units, so its warps finish together at the item barrier)
+        const uint32_t nsplit = nblock >= p.unit_target
+                                    ? 1u
+                                    : min((p.unit_target + max(nblock, 1u) - 1) / max(nblock, 1u), (nq + 31) / 32);
         const uint32_t subsz = ((nq + nsplit - 1) / nsplit + 31) & ~31u;
         const uint32_t units = nblock * nsplit;
         for (;;) {
@@ -1512,6 +1516,12 @@ uint32_t range_rows_env(uint64_t n_rows) {
     const long v = atol(e);
     // at most 2^20 rows: one item then decides < 2^32 pairs (the kernel's 32-bit per-item statistics)
     return (v >= 256 && v <= (1L << 20) && v % 256 == 0) ? (uint32_t)v : def;
+}
+
+uint32_t unit_target_env() {
+    const char *e = getenv("TM_UNIT_TARGET");
+    const long v = e ? atol(e) : 0;
+    return (v >= 1 && v <= 64) ? (uint32_t)v : (uint32_t)kScanWarps;
 }
 
 int scan_grid(int device, int variant) {

@@ -31,7 +31,8 @@ def main():
     gen_s = time.time() - t0
     t0 = time.time()
     # the layout bench.py times: balanced splits inside partitions + tile AND masks (DESIGN R17/R18)
-    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=200_000, tile_filter=1, row_order=1)
+    mp = int(os.environ.get("C5_MAX_PARTITION", str(tmb.TM_AUTO_MAX_PARTITION)))  # bench.py's default
+    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=mp, tile_filter=1, row_order=1)
     build_s = time.time() - t0
     db_sig = o2.encode(wl.db)
     flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
@@ -76,6 +77,7 @@ def main():
                               "pair_checks": st["pair_checks"], "routed_per_query": st["routed"] / q.n_sets,
                               "sample_parity": ok, "n_sets": n_sets, "n_queries": q.n_sets,
                               "scan_variant": st["scan_variant"], "layout": "tile-and + balanced-splits",
+                              "max_partition": db.stats()["max_partition"],
                               "gen_s": gen_s, "build_s": build_s}), flush=True)
     db.close()
 
