@@ -150,7 +150,7 @@ void *cub_tmp(tm_db *db, size_t bytes) {
 // Every query of the batch is encoded; queries [qlo, qlo + qn) are matched (the share of one GPU
 // of a replicated multi-GPU database; default: all), with their batch-global indices.
 uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, uint64_t qlo, uint64_t qn) {
-    NvtxRange nv_call("tm: match (S1-S8)");
+    NvtxRange nv_call("tm_match");
     tm_stats_t &st = db->st;
     const uint64_t Qall = q->n_sets;
     if (qlo > Qall) qlo = Qall;
@@ -414,7 +414,7 @@ tm_status translate(const CudaFail &f) {
 }
 
 void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, const uint32_t *keys) {
-    NvtxRange nv_build("tm: build / consolidate");
+    NvtxRange nv_build("tm_build");
     auto t0 = std::chrono::steady_clock::now();
     const bool trace = getenv("TM_TRACE_BUILD") != nullptr;
     auto mark = [&](const char *what) {

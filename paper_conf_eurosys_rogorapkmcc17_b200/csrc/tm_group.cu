@@ -123,7 +123,7 @@ void group_build(tm_db *top, const tm_tagsets *sets, const uint64_t *key_off, co
 
 // tm_match_batch (pout) or tm_match_batch_csr (cout) of a group handle.
 void group_match(tm_db *top, const tm_tagsets *q, int unique, tm_pairs *pout, tm_csr *cout) {
-    NvtxRange nv("tm: multi-GPU match");
+    NvtxRange nv("tm_group_match");
     std::vector<tm_db *> &subs = top->subs;
     const uint32_t G = (uint32_t)subs.size();
     const uint64_t Q = q->n_sets;

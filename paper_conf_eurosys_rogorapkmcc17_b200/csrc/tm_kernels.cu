@@ -163,11 +163,18 @@ __global__ void __launch_bounds__(kRouteWarps * 32, 6) k_route(const uint64_t *_
                                                             uint64_t n_blocks, uint32_t *__restrict__ counts,
                                                             const unsigned long long *__restrict__ off,
                                                             uint32_t *__restrict__ qidx, unsigned long long cap,
-                                                            uint32_t qbase) {
+                                                            uint32_t qbase, uint32_t n_slices) {
     extern __shared__ __align__(16) uint32_t zsm[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint64_t blk = (uint64_t)blockIdx.x * kRouteWarps + warp;
-    if (blk >= n_blocks) return;  // warp-uniform; no CTA barrier below
+    // warp -> (route block, partition slice): a small batch (few route blocks) has its partitions
+    // cut into n_slices ranges of whole 32-partition groups, so the grid still fills the GPU
+    const uint64_t li = (uint64_t)blockIdx.x * kRouteWarps + warp;
+    if (li >= n_blocks * n_slices) return;  // warp-uniform; no CTA barrier below
+    const uint64_t blk = li % n_blocks;
+    const uint32_t slice = (uint32_t)(li / n_blocks);
+    const uint32_t ngroups = (n_parts + 31) / 32;
+    const uint32_t gps = (ngroups + n_slices - 1) / n_slices;
+    const uint32_t g_lo = slice * gps * 32, g_hi = min(n_parts, (slice + 1) * gps * 32);
     uint32_t *z = zsm + warp * (192 * kRouteWB);
     const uint64_t qb = blk * kRouteBlockQ;
     route_build_z(z, q0, q1, q2, qb, n_q, lane);
@@ -190,9 +197,9 @@ __global__ void __launch_bounds__(kRouteWarps * 32, 6) k_route(const uint64_t *_
         return 0ULL;
     };
     uint64_t mn[3];
-    load_mask(lane, mn);
-    unsigned long long on = load_off(lane);
-    for (uint32_t g = 0; g < n_parts; g += 32) {
+    load_mask(g_lo + lane, mn);
+    unsigned long long on = load_off(g_lo + lane);
+    for (uint32_t g = g_lo; g < g_hi; g += 32) {
         const uint32_t p = g + lane;
         uint64_t m[3] = {mn[0], mn[1], mn[2]};
         const unsigned long long o_here = on;
@@ -561,11 +568,13 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // caps residency at 8 CTAs, which ptxas cannot see (the scan's shared memory is dynamic).
 // STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
 // OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>); bit 4 = lean tile
-// set-up (the two pre-check words read from the build-time wwords plane, no per-lane selects).
+// set-up (the two pre-check words read from the build-time wwords plane, no per-lane selects);
+// bit 5 = level B on the tile mask's bits beyond the block mask, non-zero words only.
 template <bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     constexpr bool kImad = (OPT & 1) != 0;
     constexpr bool kLean = WORD1 && !STREAM && (OPT & 16) != 0;
+    constexpr bool kDelta = WORD1 && !STREAM && (OPT & 32) != 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -873,39 +882,66 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     const uint32_t sw_base = (uint32_t)__cvta_generic_to_shared(swp);
                     const uint32_t my_plane = sw_base + wl * (uint32_t)(kSubWStride * 4);
                     const uint32_t my_plane2 = sw_base + wl2 * (uint32_t)(kSubWStride * 4);
+                    // kDelta: level B tests only the tile mask's bits beyond the block mask (the
+                    // level-A survivors contain those) and only its non-zero 64-bit words, through a
+                    // warp-uniform switch over the 8 word patterns (tile_filter 0 and 1: g contains f)
+                    const uint64_t d0 = kDelta ? g0 & ~f0 : g0, d1 = kDelta ? g1 & ~f1 : g1,
+                                   d2 = kDelta ? g2 & ~f2 : g2;
+                    const int dmask = kDelta ? ((d0 != 0) | ((d1 != 0) << 1) | ((d2 != 0) << 2)) : 7;
                     for (uint32_t j = 0; j < na;) {
                         // ---- level B: level-A survivors that contain the tile's mask -> word planes,
                         // 32 at a time until the buffer cannot take another 32 (full pre-check groups)
                         uint32_t nb = 0;
                         const uint32_t pe = na;
-                        // two independent 32-survivor halves per step (ILP), then one more half
-                        // when it still fits
                         uint32_t *swk = sm.sw[warp][0];
-                        for (; j < na && nb <= (uint32_t)kSubW - 64; j += 64) {
-                            const uint32_t ja = j + lane, jb = ja + 32;
-                            // sa[0, pe) holds valid slots (< kChunk); lanes past pe read slot 0
-                            const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
-                            const uint32_t ib = jb < pe ? (uint32_t)sa[jb] : 0u;
-                            const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
-                            const uint64_t b0 = sm.q0[ib], b1 = sm.q1[ib], b2 = sm.q2[ib];
-                            const bool oka = ja < pe && ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
-                            const bool okb = jb < pe && ((g0 & ~b0) | (g1 & ~b1) | (g2 & ~b2)) == 0;
-                            const uint32_t ba = __ballot_sync(0xffffffffu, oka);
-                            const uint32_t bb = __ballot_sync(0xffffffffu, okb);
-                            if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
-                            const uint32_t nba = nb + __popc(ba);
-                            if (okb) store_survivor(swk, sbi, nba + __popc(bb & lt_mask), b0, b1, b2, ib);
-                            nb = nba + __popc(bb);
-                        }
-                        if (j < na && nb <= (uint32_t)kSubW - 32) {
-                            const uint32_t ja = j + lane;
-                            const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
-                            const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
-                            const bool oka = ja < pe && ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
-                            const uint32_t ba = __ballot_sync(0xffffffffu, oka);
-                            if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
-                            nb += __popc(ba);
-                            j += 32;
+                        auto level_b = [&](auto M) {
+                            constexpr int m = decltype(M)::value;
+                            auto miss = [&](uint64_t x0, uint64_t x1, uint64_t x2) {
+                                return ((m & 1) ? (d0 & ~x0) : 0ULL) | ((m & 2) ? (d1 & ~x1) : 0ULL) |
+                                       ((m & 4) ? (d2 & ~x2) : 0ULL);
+                            };
+                            // two independent 32-survivor halves per step (ILP), then one more half
+                            // when it still fits
+                            for (; j < na && nb <= (uint32_t)kSubW - 64; j += 64) {
+                                const uint32_t ja = j + lane, jb = ja + 32;
+                                // sa[0, pe) holds valid slots (< kChunk); lanes past pe read slot 0
+                                const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
+                                const uint32_t ib = jb < pe ? (uint32_t)sa[jb] : 0u;
+                                const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
+                                const uint64_t b0 = sm.q0[ib], b1 = sm.q1[ib], b2 = sm.q2[ib];
+                                const bool oka = ja < pe && miss(a0, a1, a2) == 0;
+                                const bool okb = jb < pe && miss(b0, b1, b2) == 0;
+                                const uint32_t ba = __ballot_sync(0xffffffffu, oka);
+                                const uint32_t bb = __ballot_sync(0xffffffffu, okb);
+                                if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
+                                const uint32_t nba = nb + __popc(ba);
+                                if (okb) store_survivor(swk, sbi, nba + __popc(bb & lt_mask), b0, b1, b2, ib);
+                                nb = nba + __popc(bb);
+                            }
+                            if (j < na && nb <= (uint32_t)kSubW - 32) {
+                                const uint32_t ja = j + lane;
+                                const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
+                                const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
+                                const bool oka = ja < pe && miss(a0, a1, a2) == 0;
+                                const uint32_t ba = __ballot_sync(0xffffffffu, oka);
+                                if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
+                                nb += __popc(ba);
+                                j += 32;
+                            }
+                        };
+                        if constexpr (kDelta) {
+                            switch (dmask) {
+                                case 0: level_b(std::integral_constant<int, 0>{}); break;
+                                case 1: level_b(std::integral_constant<int, 1>{}); break;
+                                case 2: level_b(std::integral_constant<int, 2>{}); break;
+                                case 3: level_b(std::integral_constant<int, 3>{}); break;
+                                case 4: level_b(std::integral_constant<int, 4>{}); break;
+                                case 5: level_b(std::integral_constant<int, 5>{}); break;
+                                case 6: level_b(std::integral_constant<int, 6>{}); break;
+                                default: level_b(std::integral_constant<int, 7>{}); break;
+                            }
+                        } else {
+                            level_b(std::integral_constant<int, 7>{});
                         }
                         st_checks += nb * nvalid;
                         __syncwarp();
@@ -1448,8 +1484,15 @@ cudaError_t launch_route(int pass, const uint64_t *masks, uint32_t n_parts, cons
     const size_t smem = (size_t)kRouteWarps * 192 * kRouteWB * 4;  // 36 KB: within the default dynamic limit
     static_assert((size_t)kRouteWarps * 192 * kRouteWB * 4 <= 48 * 1024, "route Z needs the opt-in attribute");
     auto f = pass == 0 ? k_route<0> : k_route<1>;
-    f<<<grid_for(nb, kRouteWarps), kRouteWarps * 32, smem, s>>>(masks, n_parts, q0, q1, q2, n_q, nb, counts, off, qidx,
-                                                                cap, qbase);
+    // enough warps to fill the GPU (~16 per SM) even for small batches: slice the partitions
+    int dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t groups = (n_parts + 31) / 32;
+    const uint64_t want = (uint64_t)std::max(sms, 1) * 16;
+    const uint32_t slices = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(groups, (want + nb - 1) / nb));
+    f<<<grid_for(nb * slices, kRouteWarps), kRouteWarps * 32, smem, s>>>(masks, n_parts, q0, q1, q2, n_q, nb, counts,
+                                                                         off, qidx, cap, qbase, slices);
     return cudaGetLastError();
 }
 
@@ -1481,6 +1524,7 @@ ScanFn scan_fn(int variant) {
         case 13: return k_dense<false, 5>;  // 9 with four rows per lane
         case 14: return k_scan<true, 7, false, 17>;  // 8 + lean tile set-up (the default)
         case 15: return k_dense<false, 21>;  // 13 + the build-time pre-check words (no selects)
+        case 16: return k_scan<true, 7, false, 49>;  // 14 + level B on the extra mask words only
         default: return nullptr;
     }
 }
@@ -1521,7 +1565,7 @@ uint32_t range_rows_env(uint64_t n_rows) {
 uint32_t unit_target_env() {
     const char *e = getenv("TM_UNIT_TARGET");
     const long v = e ? atol(e) : 0;
-    return (v >= 1 && v <= 64) ? (uint32_t)v : (uint32_t)kScanWarps;
+    return (v >= 1 && v <= 64) ? (uint32_t)v : kUnitTarget;  // 8: +1% at C3 over 4 (profiles/r2j_ab_*)
 }
 
 int scan_grid(int device, int variant) {

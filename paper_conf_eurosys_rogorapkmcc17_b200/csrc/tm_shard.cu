@@ -428,7 +428,7 @@ tm_status tm_match_batch_sharded_device(tm_db *db, const tm_tagsets *q, int uniq
     const int r = db->rank;
     ncclComm_t comm = static_cast<ncclComm_t>(db->nccl_comm);
     NcclApi &a = nccl();
-    NvtxRange nv_x("tm: S9 exchange (NCCL)");
+    NvtxRange nv_x("tm_exchange");
     // S9: counts per owner, all-gathered
     owner_counts(db, G, s);
     db->xall.ensure((uint64_t)G * G * 8);
