@@ -568,13 +568,11 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // caps residency at 8 CTAs, which ptxas cannot see (the scan's shared memory is dynamic).
 // STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
 // OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>); bit 4 = lean tile
-// set-up (the two pre-check words read from the build-time wwords plane, no per-lane selects);
-// bit 5 = level B on the tile mask's bits beyond the block mask, non-zero words only.
+// set-up (the two pre-check words read from the build-time wwords plane, no per-lane selects).
 template <bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     constexpr bool kImad = (OPT & 1) != 0;
     constexpr bool kLean = WORD1 && !STREAM && (OPT & 16) != 0;
-    constexpr bool kDelta = WORD1 && !STREAM && (OPT & 32) != 0;
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -882,66 +880,39 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                     const uint32_t sw_base = (uint32_t)__cvta_generic_to_shared(swp);
                     const uint32_t my_plane = sw_base + wl * (uint32_t)(kSubWStride * 4);
                     const uint32_t my_plane2 = sw_base + wl2 * (uint32_t)(kSubWStride * 4);
-                    // kDelta: level B tests only the tile mask's bits beyond the block mask (the
-                    // level-A survivors contain those) and only its non-zero 64-bit words, through a
-                    // warp-uniform switch over the 8 word patterns (tile_filter 0 and 1: g contains f)
-                    const uint64_t d0 = kDelta ? g0 & ~f0 : g0, d1 = kDelta ? g1 & ~f1 : g1,
-                                   d2 = kDelta ? g2 & ~f2 : g2;
-                    const int dmask = kDelta ? ((d0 != 0) | ((d1 != 0) << 1) | ((d2 != 0) << 2)) : 7;
                     for (uint32_t j = 0; j < na;) {
                         // ---- level B: level-A survivors that contain the tile's mask -> word planes,
                         // 32 at a time until the buffer cannot take another 32 (full pre-check groups)
                         uint32_t nb = 0;
                         const uint32_t pe = na;
+                        // two independent 32-survivor halves per step (ILP), then one more half
+                        // when it still fits
                         uint32_t *swk = sm.sw[warp][0];
-                        auto level_b = [&](auto M) {
-                            constexpr int m = decltype(M)::value;
-                            auto miss = [&](uint64_t x0, uint64_t x1, uint64_t x2) {
-                                return ((m & 1) ? (d0 & ~x0) : 0ULL) | ((m & 2) ? (d1 & ~x1) : 0ULL) |
-                                       ((m & 4) ? (d2 & ~x2) : 0ULL);
-                            };
-                            // two independent 32-survivor halves per step (ILP), then one more half
-                            // when it still fits
-                            for (; j < na && nb <= (uint32_t)kSubW - 64; j += 64) {
-                                const uint32_t ja = j + lane, jb = ja + 32;
-                                // sa[0, pe) holds valid slots (< kChunk); lanes past pe read slot 0
-                                const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
-                                const uint32_t ib = jb < pe ? (uint32_t)sa[jb] : 0u;
-                                const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
-                                const uint64_t b0 = sm.q0[ib], b1 = sm.q1[ib], b2 = sm.q2[ib];
-                                const bool oka = ja < pe && miss(a0, a1, a2) == 0;
-                                const bool okb = jb < pe && miss(b0, b1, b2) == 0;
-                                const uint32_t ba = __ballot_sync(0xffffffffu, oka);
-                                const uint32_t bb = __ballot_sync(0xffffffffu, okb);
-                                if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
-                                const uint32_t nba = nb + __popc(ba);
-                                if (okb) store_survivor(swk, sbi, nba + __popc(bb & lt_mask), b0, b1, b2, ib);
-                                nb = nba + __popc(bb);
-                            }
-                            if (j < na && nb <= (uint32_t)kSubW - 32) {
-                                const uint32_t ja = j + lane;
-                                const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
-                                const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
-                                const bool oka = ja < pe && miss(a0, a1, a2) == 0;
-                                const uint32_t ba = __ballot_sync(0xffffffffu, oka);
-                                if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
-                                nb += __popc(ba);
-                                j += 32;
-                            }
-                        };
-                        if constexpr (kDelta) {
-                            switch (dmask) {
-                                case 0: level_b(std::integral_constant<int, 0>{}); break;
-                                case 1: level_b(std::integral_constant<int, 1>{}); break;
-                                case 2: level_b(std::integral_constant<int, 2>{}); break;
-                                case 3: level_b(std::integral_constant<int, 3>{}); break;
-                                case 4: level_b(std::integral_constant<int, 4>{}); break;
-                                case 5: level_b(std::integral_constant<int, 5>{}); break;
-                                case 6: level_b(std::integral_constant<int, 6>{}); break;
-                                default: level_b(std::integral_constant<int, 7>{}); break;
-                            }
-                        } else {
-                            level_b(std::integral_constant<int, 7>{});
+                        for (; j < na && nb <= (uint32_t)kSubW - 64; j += 64) {
+                            const uint32_t ja = j + lane, jb = ja + 32;
+                            // sa[0, pe) holds valid slots (< kChunk); lanes past pe read slot 0
+                            const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
+                            const uint32_t ib = jb < pe ? (uint32_t)sa[jb] : 0u;
+                            const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
+                            const uint64_t b0 = sm.q0[ib], b1 = sm.q1[ib], b2 = sm.q2[ib];
+                            const bool oka = ja < pe && ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
+                            const bool okb = jb < pe && ((g0 & ~b0) | (g1 & ~b1) | (g2 & ~b2)) == 0;
+                            const uint32_t ba = __ballot_sync(0xffffffffu, oka);
+                            const uint32_t bb = __ballot_sync(0xffffffffu, okb);
+                            if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
+                            const uint32_t nba = nb + __popc(ba);
+                            if (okb) store_survivor(swk, sbi, nba + __popc(bb & lt_mask), b0, b1, b2, ib);
+                            nb = nba + __popc(bb);
+                        }
+                        if (j < na && nb <= (uint32_t)kSubW - 32) {
+                            const uint32_t ja = j + lane;
+                            const uint32_t ia = ja < pe ? (uint32_t)sa[ja] : 0u;
+                            const uint64_t a0 = sm.q0[ia], a1 = sm.q1[ia], a2 = sm.q2[ia];
+                            const bool oka = ja < pe && ((g0 & ~a0) | (g1 & ~a1) | (g2 & ~a2)) == 0;
+                            const uint32_t ba = __ballot_sync(0xffffffffu, oka);
+                            if (oka) store_survivor(swk, sbi, nb + __popc(ba & lt_mask), a0, a1, a2, ia);
+                            nb += __popc(ba);
+                            j += 32;
                         }
                         st_checks += nb * nvalid;
                         __syncwarp();
@@ -1524,7 +1495,6 @@ ScanFn scan_fn(int variant) {
         case 13: return k_dense<false, 5>;  // 9 with four rows per lane
         case 14: return k_scan<true, 7, false, 17>;  // 8 + lean tile set-up (the default)
         case 15: return k_dense<false, 21>;  // 13 + the build-time pre-check words (no selects)
-        case 16: return k_scan<true, 7, false, 49>;  // 14 + level B on the extra mask words only
         default: return nullptr;
     }
 }
