@@ -28,9 +28,10 @@ def main():
     timeouts = [int(x) for x in (sys.argv[4] if len(sys.argv) > 4 else "500,1000,2000,5000").split(",")]
     max_batch = int(sys.argv[5]) if len(sys.argv) > 5 else 1 << 20
     c = dict(tmgen.CONFIGS[cfg])
-    wl = tmgen.generate(c["n_sets"], max(nq, c["n_queries"]), c["seed"], max_partition=c["max_partition"])
+    mp = int(os.environ.get("STREAM_MAX_PARTITION", str(tmb.TM_AUTO_MAX_PARTITION)))  # bench.py's default
+    wl = tmgen.generate(c["n_sets"], max(nq, c["n_queries"]), c["seed"])
     q = wl.queries.subset(np.arange(nq))
-    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=c["max_partition"], tile_filter=1, row_order=1)
+    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=mp, tile_filter=1, row_order=1)
     db.match_batch(q, True)          # warm-up: grow every device / pinned buffer once
     for b in (1, 8, 100, 1000, 3000, 10000):   # and load the kernels small batches use (CUB
         db.match_batch(q.subset(np.arange(min(b, nq))), True)  # single-tile sorts; lazy loading)
