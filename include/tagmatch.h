@@ -370,9 +370,13 @@ tm_status tm_shard_merge(tm_db *db, const uint64_t *pairs, uint64_t n, uint64_t 
 
 /* In-process multi-GPU databases (tm_config.n_gpus > 1).  tm_build builds one sub-database per
  * device (in parallel, one host thread each); tm_match_batch / tm_match_batch_csr run the batch
- * on all of them and return one result, sorted by (query, key) as always; the exchange of a
- * partitioned database is peer-to-peer copies between the GPUs (cudaMemcpyPeerAsync over
- * NVLink; peer access is enabled at build), the per-owner merge runs on the owner's GPU.
+ * on all of them and return one result, sorted by (query, key) as always.  The exchange of a
+ * partitioned database is fused into the scan: each GPU's scan kernel stores every (query, key)
+ * pair straight into the query owner's receive region for that GPU (peer memory over NVLink;
+ * peer access is enabled at build), and each owner compacts and merges its regions on its GPU.
+ * Without peer access between some pair of GPUs, for more than 8 GPUs, in exact mode, or with
+ * TM_NO_FUSED_EXCHANGE=1 in the environment, each GPU merges locally and the owners pull their
+ * pieces with peer copies (cudaMemcpyPeerAsync).
  * tm_stats sums the counters and takes the maximum of the times over the GPUs.  Calls taking
  * device pointers (tm_match_batch_device, the shard hooks) return TM_ESTATE on such a handle.
  * tm_group_size: number of sub-databases (1 for a single-GPU handle); tm_group_member: the

@@ -164,6 +164,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
     db->last_Q = Qall;
     db->last_qlo = qlo;
     db->last_qn = Qm;
+    for (uint64_t &c : db->fx.counts) c = 0;  // fused exchange: nothing sent yet
     if (Qm == 0 || P == 0) return 0;
     const uint64_t Q = Qall;                       // encoded (and the sort width)
     const uint64_t NB = route_blocks(Qm);          // route blocks of 384 queries
@@ -263,6 +264,19 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
         sp.range_rows = range_rows;
         sp.one = 1;
         sp.unit_target = unit_target_env();
+        // fused exchange (in-process multi-GPU group, tm_group.cu): emit to the owners' regions
+        sp.n_owners = db->fx.G > 1 ? db->fx.G : 0;
+        sp.xcap = db->fx.xcap;
+        sp.xcnt = nullptr;
+        for (int g = 0; g < kMaxOwners; ++g) {
+            sp.xstart[g] = db->fx.xstart[g];
+            sp.xout[g] = db->fx.xout[g];
+        }
+        if (sp.n_owners) {
+            db->xfcnt.ensure(kMaxOwners * 8);
+            sp.xcnt = db->xfcnt.as<unsigned long long>();
+            TMCK(cudaMemsetAsync(sp.xcnt, 0, kMaxOwners * 8, s));
+        }
         // variant: TM_SCAN_VARIANT if set; else a call whose partition batches are all small
         // (Q <= kSmallBatch) takes the streaming path only, in the streaming-only kernels (small
         // shared memory: 8 CTAs/SM) -- up to four queries checked directly (variant 6), 5-8
@@ -298,6 +312,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
         st.scan_launches++;
         TMCK(cudaEventRecord(db->ev[3], s));
         TMCK(cudaMemcpyAsync(db->h_ctr, ctr, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
+        if (sp.n_owners) TMCK(cudaMemcpyAsync(db->h_fx, sp.xcnt, kMaxOwners * 8, cudaMemcpyDeviceToHost, s));
         TMCK(cudaStreamSynchronize(s));
         const DevCounters c = *db->h_ctr;
         if (c.input_err)
@@ -326,6 +341,16 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
         st.emitted_pairs = c.n_out;
         st.work_items = c.n_items;
         break;
+    }
+    if (db->fx.G > 1) {  // fused exchange: the pairs are in the owners' regions; they merge them
+        st.emitted_pairs = 0;
+        for (uint32_t g = 0; g < db->fx.G; ++g) {
+            db->fx.counts[g] = db->h_fx[g];
+            st.emitted_pairs += db->h_fx[g];
+        }
+        TMCK(cudaEventRecord(db->ev[4], s));
+        st.kernel_launches = launches;
+        return 0;
     }
     uint64_t n = st.emitted_pairs;
     if (db->cfg.exact) {  // S7': exact subset check of the (query, set) candidates, then keys
@@ -628,7 +653,7 @@ void destroy_db(tm_db *db) {
         shard_destroy(db);
     } catch (...) {
     }
-    for (DevBuf *b : {&db->planes, &db->tand, &db->wsel, &db->wwords, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
+    for (DevBuf *b : {&db->xfcnt, &db->xfin, &db->planes, &db->tand, &db->wsel, &db->wwords, &db->key_off, &db->keys, &db->masks, &db->part_row, &db->part_n, &db->in_bytes,
                       &db->in_voff, &db->in_tidx, &db->in_soff, &db->vsig, &db->qplanes, &db->bm, &db->word_off,
                       &db->qidx, &db->qoff, &db->item_cnt, &db->item_off, &db->out, &db->out_alt, &db->res_q,
                       &db->res_k, &db->res_off, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,
@@ -640,6 +665,7 @@ void destroy_db(tm_db *db) {
         if (e) cudaEventDestroy(e);
     if (db->h_ctr) cudaFreeHost(db->h_ctr);
     if (db->h_nuniq) cudaFreeHost(db->h_nuniq);
+    if (db->h_fx) cudaFreeHost(db->h_fx);
     if (db->stream) cudaStreamDestroy(db->stream);
     if (prev >= 0) cudaSetDevice(prev);
     delete db;
@@ -712,6 +738,7 @@ tm_db *build_db(const tm_tagsets *sets, const uint64_t *key_off, const uint32_t 
         for (auto &e : db->ev) TMCK(cudaEventCreate(&e));
         TMCK(cudaMallocHost((void **)&db->h_ctr, sizeof(DevCounters)));
         TMCK(cudaMallocHost((void **)&db->h_nuniq, 8));
+        TMCK(cudaMallocHost((void **)&db->h_fx, kMaxOwners * 8));
         db->scan_grid = 0;
         build_impl(db, sets, key_off, keys);
         // load every scan-kernel variant now (lazy module loading would otherwise put ~10-30 ms into

@@ -164,6 +164,18 @@ struct tm_db {
     uint64_t merged_n = 0;
     // in-process multi-GPU database (tm_group.cu): sub-databases, one per device
     std::vector<tm_db *> subs;
+    bool fused_ok = false;  // group: every pair of its GPUs has peer access (the fused exchange)
+    uint64_t fx_cap = 0;    // group: receive-region capacity of the last call (pairs)
+    // a sub-database's fused-exchange target for the current call (G = 0: none)
+    struct {
+        uint32_t G = 0;
+        uint32_t xstart[kMaxOwners] = {};
+        uint64_t *xout[kMaxOwners] = {};
+        unsigned long long xcap = 0;
+        uint64_t counts[kMaxOwners] = {};  // pairs this GPU wrote to each owner in the last call
+    } fx;
+    DevBuf xfcnt, xfin;  // fused exchange: counters per owner; an owner's compacted receive buffer
+    unsigned long long *h_fx = nullptr;  // pinned copy of xfcnt
     // mutable handle (tm_create; tm_store.cpp): the entry multiset + staged operations
     Store *store = nullptr;
     std::vector<int32_t> store_devices;

@@ -54,13 +54,17 @@ void on_each(const std::vector<tm_db *> &subs, F f) {
         if (err[g].failed) fail(err[g].s, "GPU " + std::to_string(g) + ": " + err[g].msg);
 }
 
-void enable_peers(const std::vector<int> &dev) {
+// Enables peer access between every pair of distinct devices; returns whether every pair has it
+// (the fused exchange stores into peer memory from the scan kernel).
+bool enable_peers(const std::vector<int> &dev) {
+    bool all = true;
     for (int a : dev)
         for (int b : dev) {
             if (a == b) continue;
             int ok = 0;
             if (cudaDeviceCanAccessPeer(&ok, a, b) != cudaSuccess || !ok) {
                 cudaGetLastError();
+                all = false;
                 continue;  // cudaMemcpyPeerAsync still works (staged by the driver)
             }
             DeviceGuard g(a);
@@ -68,6 +72,7 @@ void enable_peers(const std::vector<int> &dev) {
             if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) throw CudaFail{e, "cudaDeviceEnablePeerAccess", __LINE__};
             cudaGetLastError();
         }
+    return all;
 }
 
 }  // namespace
@@ -89,7 +94,11 @@ void group_build(tm_db *top, const tm_tagsets *sets, const uint64_t *key_off, co
         if (dev[g] < 0 || dev[g] >= visible) fail(TM_EINVAL, "device_ids[" + std::to_string(g) + "] is not a visible device");
         check_device(dev[g]);
     }
-    enable_peers(dev);
+    // the fused exchange needs peer stores between every pair of GPUs, at most kMaxOwners of them,
+    // and the Bloom result (exact mode post-checks candidates on the GPU that found them);
+    // TM_NO_FUSED_EXCHANGE=1 selects the pull exchange (peer copies after a local merge)
+    top->fused_ok = enable_peers(dev) && G <= (uint32_t)kMaxOwners && !cfg->exact &&
+                    !getenv("TM_NO_FUSED_EXCHANGE");
     top->device = dev[0];
     top->cfg.device_ids = nullptr;
     top->cfg.plan_sample = nullptr;
@@ -134,9 +143,80 @@ void group_match(tm_db *top, const tm_tagsets *q, int unique, tm_pairs *pout, tm
         hi[g] = owner_start(Q, G, g + 1);
     }
     const auto t0 = std::chrono::steady_clock::now();
+    std::vector<uint64_t> counts((size_t)G * G, 0);
+    std::vector<const uint64_t *> res(G, nullptr);  // owner g's sorted (q<<32|key) pairs
+    std::vector<uint64_t> n(G, 0);
+    std::vector<uint64_t> sent(G, 0), recvd(G, 0);
+    std::chrono::steady_clock::time_point t1, t2;
+    if (!repl && top->fused_ok && G > 1) {
+        // ---- fused exchange: every GPU's scan stores each pair straight into its query owner's
+        // receive region for that GPU (peer memory over NVLink); no local sort, no copy step
+        uint64_t xcap = top->fx_cap ? top->fx_cap : std::max<uint64_t>(1 << 16, 8 * Q / G + 1024);
+        if (const char *e = getenv("TM_FUSED_XCAP"))  // tests: start small to exercise the retry
+            if (!top->fx_cap && atoll(e) > 0) xcap = (uint64_t)atoll(e);
+        for (int attempt = 0;; ++attempt) {
+            for (uint32_t d = 0; d < G; ++d) {
+                DeviceGuard dg(subs[d]->device);
+                subs[d]->xrecv.ensure((uint64_t)G * xcap * 8);
+            }
+            for (uint32_t g = 0; g < G; ++g) {
+                auto &fx = subs[g]->fx;
+                fx.G = G;
+                fx.xcap = xcap;
+                for (uint32_t d = 0; d < G; ++d) {
+                    fx.xstart[d] = (uint32_t)lo[d];
+                    fx.xout[d] = subs[d]->xrecv.as<uint64_t>() + (uint64_t)g * xcap;
+                }
+            }
+            try {
+                on_each(subs, [&](size_t g) {
+                    tm_db *db = subs[g];
+                    const tm_tagsets dq = upload_queries(db, q, db->stream);
+                    match_core(db, &dq, unique, db->stream);
+                    finish_timing(db, db->stream);
+                    for (uint32_t d = 0; d < G; ++d) counts[(size_t)g * G + d] = db->fx.counts[d];
+                });
+            } catch (...) {
+                for (tm_db *db : subs) db->fx.G = 0;
+                throw;
+            }
+            uint64_t mx = 0;
+            for (uint64_t c : counts) mx = std::max(mx, c);
+            if (mx <= xcap) break;
+            if (attempt >= 4) {
+                for (tm_db *db : subs) db->fx.G = 0;
+                fail(TM_ESTATE, "fused exchange: capacity retry did not converge");
+            }
+            xcap = mx + mx / 4;  // a region overflowed (the stores past xcap were dropped): again
+        }
+        for (tm_db *db : subs) db->fx.G = 0;
+        top->fx_cap = xcap;
+        t1 = std::chrono::steady_clock::now();
+        // each owner compacts its G regions and merges them (sort / de-duplicate)
+        on_each(subs, [&](size_t d) {
+            tm_db *db = subs[d];
+            cudaStream_t s = db->stream;
+            uint64_t total = 0;
+            for (uint32_t g = 0; g < G; ++g) total += counts[(size_t)g * G + d];
+            db->xfin.ensure(std::max<uint64_t>(total, 1) * 8);
+            uint64_t o = 0;
+            for (uint32_t g = 0; g < G; ++g) {
+                const uint64_t c = counts[(size_t)g * G + d];
+                if (c)
+                    TMCK(cudaMemcpyAsync(db->xfin.as<uint64_t>() + o, db->xrecv.as<uint64_t>() + (uint64_t)g * xcap,
+                                         c * 8, cudaMemcpyDeviceToDevice, s));
+                if (g != d) recvd[d] += c * 8;
+                o += c;
+            }
+            n[d] = merge_pairs(db, db->xfin.as<uint64_t>(), total, Q, unique, s);
+            res[d] = db->merged;
+            for (uint32_t dd = 0; dd < G; ++dd)
+                if (dd != d) sent[d] += 8 * counts[(size_t)d * G + dd];
+        });
+        t2 = std::chrono::steady_clock::now();
+    } else {
     // phase 1: every GPU runs S1-S8 (partitioned: the whole batch against its partitions;
     // replicated: its owner range against the whole table)
-    std::vector<uint64_t> counts((size_t)G * G, 0);
     on_each(subs, [&](size_t g) {
         tm_db *db = subs[g];
         const tm_tagsets dq = upload_queries(db, q, db->stream);
@@ -152,11 +232,8 @@ void group_match(tm_db *top, const tm_tagsets *q, int unique, tm_pairs *pout, tm
             TMCK(cudaStreamSynchronize(db->stream));
         }
     });
-    const auto t1 = std::chrono::steady_clock::now();
+    t1 = std::chrono::steady_clock::now();
     // phase 2 (partitioned): each owner pulls its pieces from every GPU and merges them
-    std::vector<const uint64_t *> res(G, nullptr);  // owner g's sorted (q<<32|key) pairs
-    std::vector<uint64_t> n(G, 0);
-    std::vector<uint64_t> sent(G, 0), recvd(G, 0);
     if (repl) {
         for (uint32_t g = 0; g < G; ++g) {
             res[g] = subs[g]->last_sorted;
@@ -182,7 +259,8 @@ void group_match(tm_db *top, const tm_tagsets *q, int unique, tm_pairs *pout, tm
             sent[d] = 8 * (soff[d][G] - (soff[d][d + 1] - soff[d][d]));
         });
     }
-    const auto t2 = std::chrono::steady_clock::now();
+    t2 = std::chrono::steady_clock::now();
+    }
     std::vector<uint64_t> base(G + 1, 0);
     for (uint32_t g = 0; g < G; ++g) base[g + 1] = base[g] + n[g];
     const uint64_t N = base[G];

@@ -23,6 +23,7 @@ constexpr int kTile = 32;  // rows per warp tile (= one warp, Alg. 4 "thread blo
 // Scan-kernel geometry.
 constexpr int kScanWarps = 4;      // warps per CTA
 constexpr uint32_t kUnitTarget = 8; // filtered path: items of fewer blocks are split to this many units
+constexpr int kMaxOwners = 8;       // fused exchange: GPUs of an in-process group the scan can emit to
 #ifndef TM_CHUNK
 #define TM_CHUNK 640
 #endif
@@ -70,6 +71,13 @@ struct ScanParams {
     uint32_t unit_target;             // filtered path: split items of fewer blocks to this many units
     uint32_t range_rows;              // rows per work item (multiple of 256)
     uint32_t one;                     // 1 (a run-time operand, so the FMA-pipe accumulate stays an IMAD)
+    // fused exchange (n_owners > 1): pairs of query q go to xout[owner(q)] (owner(q) = last g with
+    // xstart[g] <= q), reserved on the local counter xcnt[owner], at most xcap pairs per region
+    uint32_t n_owners;
+    uint32_t xstart[kMaxOwners];
+    uint64_t *xout[kMaxOwners];
+    unsigned long long *xcnt;
+    unsigned long long xcap;
 };
 
 // ------------------------------------------------------------ launchers --

@@ -459,11 +459,55 @@ __device__ __forceinline__ void tile_prefix(uint64_t f0, uint64_t f1, uint64_t f
 // Emit the (query, key) pairs of the lanes whose set matched: the key lookup and a
 // warp-aggregated output reservation (replacing the per-pair atomic of PAPER.md:158).  bm = the
 // warp's ballot of m (warp-uniform call); m lanes write their set's keys.
+// Fused exchange (in-process multi-GPU database, tm_group.cu): the lanes' keys go straight to the
+// query owner's receive region for this GPU (a peer pointer over NVLink) instead of the local output;
+// one warp-aggregated reservation per owner present in the warp, on this GPU's counter of that
+// owner (no remote atomics).  nk = the lane's key count, kb = its first key, qg = its query.
+__device__ __forceinline__ uint32_t owner_of(uint32_t qg, const ScanParams &p) {
+    uint32_t d = 0;
+#pragma unroll
+    for (int g = 1; g < kMaxOwners; ++g)
+        if ((uint32_t)g < p.n_owners && qg >= p.xstart[g]) d = (uint32_t)g;
+    return d;
+}
+
+__device__ __forceinline__ void emit_fused(uint32_t nk, uint32_t kb, uint32_t qg, const ScanParams &p, int lane) {
+    const uint32_t d = nk ? owner_of(qg, p) : 0u;
+    uint32_t todo = __ballot_sync(0xffffffffu, nk > 0);
+    while (todo) {
+        const int leader = __ffs(todo) - 1;
+        const uint32_t dd = __shfl_sync(0xffffffffu, d, leader);
+        const bool mine = nk > 0 && d == dd;
+        todo &= ~__ballot_sync(0xffffffffu, mine);
+        uint32_t v = mine ? nk : 0u, incl = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += t;
+        }
+        const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+        unsigned long long base = 0;
+        if (lane == leader) base = atomicAdd(p.xcnt + dd, (unsigned long long)total);
+        base = __shfl_sync(0xffffffffu, base, leader);
+        if (mine) {
+            unsigned long long o = base + (incl - v);
+            uint64_t *dst = p.xout[dd];
+            const uint64_t hi = (uint64_t)qg << 32;
+            for (uint32_t j = 0; j < nk; ++j, ++o)
+                if (o < p.xcap) dst[o] = hi | (uint64_t)__ldg(p.keys + kb + j);
+        }
+    }
+}
+
 __device__ __forceinline__ void emit_direct(bool m, uint32_t row, uint32_t qg, const ScanParams &p, int lane) {
     uint32_t kb = 0, nk = 0;
     if (m) {
         kb = __ldg(p.key_off + row);
         nk = __ldg(p.key_off + row + 1) - kb;
+    }
+    if (p.n_owners > 1) {
+        emit_fused(nk, kb, qg, p, lane);
+        return;
     }
     uint32_t incl = nk;
 #pragma unroll
@@ -492,6 +536,12 @@ __device__ __forceinline__ void flush_pend(uint2 *pend, uint32_t &npend, const S
     if (m) {
         kb = __ldg(p.key_off + e.x);
         nk = __ldg(p.key_off + e.x + 1) - kb;
+    }
+    if (p.n_owners > 1) {
+        emit_fused(nk, kb, e.y, p, lane);
+        npend = 0;
+        __syncwarp();
+        return;
     }
     uint32_t incl = nk;
 #pragma unroll

@@ -44,7 +44,14 @@ def _csr_to_pairs(off, key):
 @pytest.mark.parametrize("G", [2, 3])
 @pytest.mark.parametrize("mode", [tm.TM_SHARD_PARTITIONED, tm.TM_SHARD_REPLICATED])
 @pytest.mark.parametrize("tile_filter,row_order", [(1, 1), (0, 0)])
-def test_in_process_group_equals_oracle(wl, want, G, mode, tile_filter, row_order):
+@pytest.mark.parametrize("fused", [True, False])
+def test_in_process_group_equals_oracle(wl, want, G, mode, tile_filter, row_order, fused, monkeypatch):
+    """Partitioned groups exchange through the fused scan emission (pairs stored into the owners'
+    receive regions) or, with TM_NO_FUSED_EXCHANGE, through local merges + peer pulls."""
+    if fused:
+        monkeypatch.delenv("TM_NO_FUSED_EXCHANGE", raising=False)
+    else:
+        monkeypatch.setenv("TM_NO_FUSED_EXCHANGE", "1")
     with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=tile_filter,
                       row_order=row_order, n_gpus=G, shard_mode=mode, device_ids=[0] * G) as db:
         assert db.group_size() == G
@@ -66,8 +73,12 @@ def test_in_process_group_equals_oracle(wl, want, G, mode, tile_filter, row_orde
                 assert st["xchg_send_bytes"] == 0
 
 
-def test_group_edge_batches(wl, want):
-    """Empty batch, one query, fewer queries than GPUs (empty owner ranges)."""
+@pytest.mark.parametrize("variant", ["", "13", "0", "6"])
+def test_group_edge_batches(wl, want, variant, monkeypatch):
+    """Empty batch, one query, fewer queries than GPUs (empty owner ranges), through the fused
+    exchange of every emission path (filtered default, dense, no pre-check, streaming)."""
+    if variant:
+        monkeypatch.setenv("TM_SCAN_VARIANT", variant)
     with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=1, row_order=1,
                       n_gpus=3, device_ids=[0, 0, 0]) as db:
         for n in (0, 1, 2, 5):
@@ -77,6 +88,16 @@ def test_group_edge_batches(wl, want):
             _eq(db.match_batch(q, False), (wq, wk), f"n={n}")
             off, key = db.match_batch_csr(q, False)
             assert off.size == n + 1 and off[-1] == wq.size
+
+
+def test_fused_exchange_region_overflow_retry(wl, want, monkeypatch):
+    """Receive regions far too small for the first call: the scan's stores past the capacity are
+    dropped, the counters report the overflow, the call re-runs with regions that fit."""
+    monkeypatch.setenv("TM_FUSED_XCAP", "16")
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=1, row_order=1,
+                      n_gpus=3, device_ids=[0, 0, 0]) as db:
+        for unique in (False, True):
+            _eq(db.match_batch(wl.queries, unique), want[unique], f"overflow retry u={unique}")
 
 
 def test_group_rejects_device_pointer_calls(wl):

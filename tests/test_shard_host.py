@@ -176,3 +176,14 @@ def test_exchange_protocol_two_ranks_gloo():
     result = mgr.dict()
     mp.spawn(_shard_worker, args=(2, port, result), nprocs=2, join=True)
     assert dict(result) == {0: (True, True, True), 1: (True, True, True)}
+
+
+def test_auto_max_partition_rule(c1):
+    """TM_AUTO_MAX_PARTITION (R8b) resolves to clamp(n / 30,000, 5,000, 200,000): on the
+    host hook the table equals the one built with that MAX_P given explicitly."""
+    sig = o2.encode(c1.db)
+    auto = tm.partition_host(sig, tm.TM_AUTO_MAX_PARTITION)
+    want = min(200_000, max(5_000, sig.shape[0] // 30_000))
+    explicit = tm.partition_host(sig, want)
+    for a, b in zip(auto, explicit):
+        assert np.array_equal(a, b)
