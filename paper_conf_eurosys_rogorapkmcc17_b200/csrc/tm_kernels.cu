@@ -499,13 +499,14 @@ __device__ __forceinline__ void emit_fused(uint32_t nk, uint32_t kb, uint32_t qg
     }
 }
 
+template <bool FUSED>
 __device__ __forceinline__ void emit_direct(bool m, uint32_t row, uint32_t qg, const ScanParams &p, int lane) {
     uint32_t kb = 0, nk = 0;
     if (m) {
         kb = __ldg(p.key_off + row);
         nk = __ldg(p.key_off + row + 1) - kb;
     }
-    if (p.n_owners > 1) {
+    if constexpr (FUSED) {
         emit_fused(nk, kb, qg, p, lane);
         return;
     }
@@ -526,6 +527,7 @@ __device__ __forceinline__ void emit_direct(bool m, uint32_t row, uint32_t qg, c
 }
 
 // Emit the warp's staged matches (lanes 0..npend-1 take one each); warp-uniform call.
+template <bool FUSED>
 __device__ __forceinline__ void flush_pend(uint2 *pend, uint32_t &npend, const ScanParams &p, int lane) {
     if (!npend) return;
     __syncwarp();
@@ -537,7 +539,7 @@ __device__ __forceinline__ void flush_pend(uint2 *pend, uint32_t &npend, const S
         kb = __ldg(p.key_off + e.x);
         nk = __ldg(p.key_off + e.x + 1) - kb;
     }
-    if (p.n_owners > 1) {
+    if constexpr (FUSED) {
         emit_fused(nk, kb, e.y, p, lane);
         npend = 0;
         __syncwarp();
@@ -563,12 +565,13 @@ __device__ __forceinline__ void flush_pend(uint2 *pend, uint32_t &npend, const S
 
 // Stage the matches of one warp step (bm = ballot of m, nonzero, warp-uniform); a step with more
 // matches than the stage holds is emitted directly.
+template <bool FUSED>
 __device__ __forceinline__ void emit_keys(bool m, uint32_t bm, uint32_t row, uint32_t qg, const ScanParams &p,
                                           int lane, uint2 *pend, uint32_t &npend) {
     const uint32_t c = __popc(bm);
-    if (npend + c > kPend) flush_pend(pend, npend, p, lane);
+    if (npend + c > kPend) flush_pend<FUSED>(pend, npend, p, lane);
     if (c > kPend) {
-        emit_direct(m, row, qg, p, lane);
+        emit_direct<FUSED>(m, row, qg, p, lane);
         return;
     }
     if (m) pend[npend + __popc(bm & ((1u << lane) - 1u))] = make_uint2(row, qg);
@@ -576,6 +579,7 @@ __device__ __forceinline__ void emit_keys(bool m, uint32_t bm, uint32_t row, uin
 }
 
 // Block 2 of one survivor whose blocks 0-1 passed in some lane, then emit.
+template <bool FUSED>
 __device__ __forceinline__ void check_block2(bool hit01, uint32_t slot, uint64_t s2, uint32_t row,
                                              ScanSmem &sm, const ScanParams &p, int lane,
                                              uint32_t &matched, uint32_t &npend) {
@@ -583,7 +587,7 @@ __device__ __forceinline__ void check_block2(bool hit01, uint32_t slot, uint64_t
     const uint32_t b = __ballot_sync(0xffffffffu, m);
     if (b) {
         matched += __popc(b);
-        emit_keys(m, b, row, __ldg(sm.qid + slot), p, lane, sm.pend[threadIdx.x >> 5], npend);
+        emit_keys<FUSED>(m, b, row, __ldg(sm.qid + slot), p, lane, sm.pend[threadIdx.x >> 5], npend);
     }
 }
 
@@ -623,6 +627,7 @@ template <bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     constexpr bool kImad = (OPT & 1) != 0;
     constexpr bool kLean = WORD1 && !STREAM && (OPT & 16) != 0;
+    constexpr bool kFused = (OPT & 64) != 0;  // emission into the owners' regions (in-process group)
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -761,7 +766,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                         const uint32_t bm = __ballot_sync(0xffffffffu, m);
                         if (bm) {
                             st_matched += __popc(bm);
-                            emit_keys(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane, sm.pend[warp], npend);
+                            emit_keys<kFused>(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane, sm.pend[warp], npend);
                         }
                     }
                     const uint32_t u0 = rlo + u * 64;
@@ -799,7 +804,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                             const uint32_t bq = __ballot_sync(0xffffffffu, hh[e]);
                             if (bq) {
                                 st_matched += __popc(bq);
-                                emit_keys(hh[e], bq, rr4[e], qg, p, lane, sm.pend[warp], npend);
+                                emit_keys<kFused>(hh[e], bq, rr4[e], qg, p, lane, sm.pend[warp], npend);
                             }
                         }
                     }
@@ -1005,7 +1010,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                                 const uint32_t bm = __ballot_sync(0xffffffffu, m);
                                 if (bm) {
                                     st_matched += __popc(bm);
-                                    emit_keys(m, bm, row, m ? __ldg(sm.qid + sbi[e]) : 0u, p, lane, sm.pend[warp], npend);
+                                    emit_keys<kFused>(m, bm, row, m ? __ldg(sm.qid + sbi[e]) : 0u, p, lane, sm.pend[warp], npend);
                                 }
                             }
                         }
@@ -1058,7 +1063,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
 #pragma unroll
                             for (int j = 0; j < 4; ++j)
                                 if (k + j < nb && __any_sync(0xffffffffu, h[j]))
-                                    check_block2(h[j], sbi[k + j], s2, row, sm, p, lane, st_matched, npend);
+                                    check_block2<kFused>(h[j], sbi[k + j], s2, row, sm, p, lane, st_matched, npend);
                         }
                     }
                     __syncwarp();
@@ -1069,7 +1074,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
         __syncthreads();
     }
     // the loop ends for all warps together (after the barrier that read the last item)
-    flush_pend(sm.pend[warp], npend, p, lane);
+    flush_pend<kFused>(sm.pend[warp], npend, p, lane);
     if (lane == 0 && (st_tests | st_checks | st_matched)) {
         atomicAdd(&sm.cnt[0], (unsigned long long)st_tests);
         atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
@@ -1149,6 +1154,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, BULK ? 6 : 7) k_dense(const S
     using Smem = typename std::conditional<BULK, DenseSmemBulk, DenseSmemBase>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
     constexpr bool kImad = (OPT & 1) != 0;
+    constexpr bool kFused = (OPT & 64) != 0;  // emission into the owners' regions (in-process group)
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     uint32_t st_checks = 0, st_matched = 0;
     uint32_t npend = 0;
@@ -1306,7 +1312,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, BULK ? 6 : 7) k_dense(const S
                         const uint32_t bm = __ballot_sync(0xffffffffu, m);
                         if (bm) {
                             st_matched += __popc(bm);
-                            emit_keys(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane, sm.pend[warp], npend);
+                            emit_keys<kFused>(m, bm, row, m ? __ldg(sm.qid + j) : 0u, p, lane, sm.pend[warp], npend);
                         }
                     }
                 }
@@ -1372,7 +1378,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, BULK ? 6 : 7) k_dense(const S
         }
         __syncthreads();
     }
-    flush_pend(sm.pend[warp], npend, p, lane);
+    flush_pend<kFused>(sm.pend[warp], npend, p, lane);
     if (lane == 0 && (st_checks | st_matched)) {
         atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
         atomicAdd(&sm.cnt[2], (unsigned long long)st_matched);
@@ -1527,27 +1533,32 @@ cudaError_t launch_items(const unsigned long long *word_off, uint64_t qw, const 
 
 namespace {
 using ScanFn = void (*)(const ScanParams);
-ScanFn scan_fn(int variant) {
+// FUSED: the same kernel with the fused-exchange emission (OPT bit 6), launched when
+// ScanParams.n_owners > 1 (in-process partitioned groups); the local-output kernels stay untouched
+template <int F>
+ScanFn scan_fn_t(int variant) {
     // variants 1-4 of round 1 (8 survivors per iteration, all three blocks in the main loop, pair
     // unions) never won a tuning class and were removed in round 2; their numbers stay unused
     switch (variant) {
-        case 0: return k_scan<false>;  // no word pre-check: 4 survivors per iteration, blocks 0-1 first
+        case 0: return k_scan<false, 8, false, F>;  // no word pre-check: 4 survivors per iteration, blocks 0-1 first
         // 72 registers and 7 CTAs/SM, no spills: 2.00 ms at C2 vs 2.10 ms with 64 registers and
         // 8 CTAs (spills) and 2.05 ms with 76 registers and 6 CTAs (profiles/r1v29_minb.txt)
-        case 5: return k_scan<true, 7>;
-        case 6: return k_scan<false, 8, true>;   // streaming only, direct check
-        case 7: return k_scan<true, 8, true>;    // streaming only, word pre-check
-        case 8: return k_scan<true, 7, false, 1>;  // 5 + pre-check accumulate on the FMA pipe
-        case 9: return k_dense<false, 1>;   // unfiltered dense scan, direct loads, FMA-pipe accumulate
-        case 10: return k_dense<true, 1>;   // unfiltered dense scan, bulk-copy (TMA) staged rows
-        case 11: return k_dense<false, 0>;
-        case 12: return k_dense<true, 0>;
-        case 13: return k_dense<false, 5>;  // 9 with four rows per lane
-        case 14: return k_scan<true, 7, false, 17>;  // 8 + lean tile set-up (the default)
-        case 15: return k_dense<false, 21>;  // 13 + the build-time pre-check words (no selects)
+        case 5: return k_scan<true, 7, false, F>;
+        case 6: return k_scan<false, 8, true, F>;   // streaming only, direct check
+        case 7: return k_scan<true, 8, true, F>;    // streaming only, word pre-check
+        case 8: return k_scan<true, 7, false, 1 | F>;  // 5 + pre-check accumulate on the FMA pipe
+        case 9: return k_dense<false, 1 | F>;   // unfiltered dense scan, direct loads, FMA-pipe accumulate
+        case 10: return k_dense<true, 1 | F>;   // unfiltered dense scan, bulk-copy (TMA) staged rows
+        case 11: return k_dense<false, 0 | F>;
+        case 12: return k_dense<true, 0 | F>;
+        case 13: return k_dense<false, 5 | F>;  // 9 with four rows per lane
+        case 14: return k_scan<true, 7, false, 17 | F>;  // 8 + lean tile set-up (the default)
+        case 15: return k_dense<false, 21 | F>;  // 13 + the build-time pre-check words (no selects)
         default: return nullptr;
     }
 }
+
+ScanFn scan_fn(int variant, bool fused = false) { return fused ? scan_fn_t<64>(variant) : scan_fn_t<0>(variant); }
 }  // namespace
 
 size_t scan_smem(int variant) {
@@ -1593,6 +1604,7 @@ int scan_grid(int device, int variant) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
     ScanFn f = scan_fn(variant);
     if (!f) return 0;  // unused variant number
+    cudaFuncSetAttribute(scan_fn(variant, true), cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem(variant));
     cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)scan_smem(variant));
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, f, kScanWarps * 32, scan_smem(variant));
     if (per < 1) per = 1;
@@ -1601,7 +1613,7 @@ int scan_grid(int device, int variant) {
 }
 
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant) {
-    scan_fn(variant)<<<grid, kScanWarps * 32, scan_smem(variant), s>>>(p);
+    scan_fn(variant, p.n_owners > 1)<<<grid, kScanWarps * 32, scan_smem(variant), s>>>(p);
     return cudaGetLastError();
 }
 

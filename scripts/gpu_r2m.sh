@@ -1,0 +1,7 @@
+TAG=${1:-r2m}
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
+TM_FULL_SIZE=0 timeout 1200 python -m pytest tests -m gpu -q -x -k "group or store or shard or variant or fuzz or c1" > gpurun_out/${TAG}_pytest.log 2>&1; echo "pytest rc=$?"; tail -3 gpurun_out/${TAG}_pytest.log
+timeout 600 python scripts/ab.py C2 "14" "5000" 7 > gpurun_out/${TAG}_ab_C2.jsonl 2>&1; echo "ab C2 rc=$?"
+timeout 900 python scripts/ab.py C3 "14" "5000" 5 > gpurun_out/${TAG}_ab_C3.jsonl 2>&1; echo "ab C3 rc=$?"
+timeout 900 compute-sanitizer --tool memcheck --error-exitcode 99 python scripts/sanitize.py 14,13,6 20000 > gpurun_out/${TAG}_memcheck.log 2>&1; echo "memcheck rc=$?"; tail -1 gpurun_out/${TAG}_memcheck.log
