@@ -253,116 +253,6 @@ __global__ void __launch_bounds__(kRouteWarps * 32, 6) k_route(const uint64_t *_
     }
 }
 
-// Transposed form (TM_ROUTE=1 selects it): lane = query word.  A warp owns 32
-// query words (1024 queries) and walks the partitions one at a time, all lanes on the same mask:
-// per mask bit one conflict-free LDS.32 (lane l reads Z[pos][l]) and one OR give 32 queries'
-// routing bits in every lane at once, instead of a data-dependent 48-byte row per lane.
-constexpr int kRouteTWarps = 2;              // warps per CTA
-constexpr int kRouteTStride = 33;            // Z row stride (words): conflict-free transposed stores
-constexpr int kRouteTBlockQ = 32 * 32;       // 1024 queries per warp
-
-template <int PASS>
-__global__ void __launch_bounds__(kRouteTWarps * 32) k_route_t(const uint64_t *__restrict__ masks, uint32_t n_parts,
-                                                              const uint64_t *__restrict__ q0,
-                                                              const uint64_t *__restrict__ q1,
-                                                              const uint64_t *__restrict__ q2, uint64_t n_q,
-                                                              uint64_t n_blocks, uint32_t *__restrict__ counts,
-                                                              const unsigned long long *__restrict__ off,
-                                                              uint32_t *__restrict__ qidx, unsigned long long cap,
-                                                              uint32_t qbase, uint32_t n_slices) {
-    extern __shared__ __align__(16) uint32_t zsm[];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint64_t li = (uint64_t)blockIdx.x * kRouteTWarps + warp;
-    if (li >= n_blocks * n_slices) return;  // warp-uniform; no CTA barrier below
-    const uint64_t blk = li % n_blocks;
-    const uint32_t slice = (uint32_t)(li / n_blocks);
-    const uint32_t pps = (n_parts + n_slices - 1) / n_slices;
-    const uint32_t p_lo = slice * pps, p_hi = min(n_parts, p_lo + pps);
-    uint32_t *z = zsm + warp * (192 * kRouteTStride);
-    const uint64_t qb = blk * kRouteTBlockQ;
-    // Z[pos][w] (stride 33): bit t = query qb + 32 w + t lacks position pos
-    for (int w = 0; w < 32; ++w) {
-        const uint64_t q = qb + (uint64_t)w * 32 + lane;
-        uint64_t a[3] = {~0ULL, ~0ULL, ~0ULL};
-        if (q < n_q) {
-            a[0] = __ldg(q0 + q);
-            a[1] = __ldg(q1 + q);
-            a[2] = __ldg(q2 + q);
-        }
-#pragma unroll
-        for (int wd = 0; wd < 3; ++wd) {
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const uint32_t x = (uint32_t)(a[wd] >> (32 * h));
-                uint32_t mine = 0;
-#pragma unroll
-                for (int t = 0; t < 32; ++t) {
-                    const uint32_t b = __ballot_sync(0xffffffffu, ((x >> t) & 1u) == 0u);
-                    if (lane == t) mine = b;
-                }
-                z[(64 * wd + 32 * h + lane) * kRouteTStride + w] = mine;
-            }
-        }
-    }
-    __syncwarp();
-    const uint64_t lo = qb + 32ULL * lane;  // this lane's query word
-    const uint32_t vm = n_q > lo ? (n_q - lo >= 32 ? ~0u : ((1u << (n_q - lo)) - 1u)) : 0u;
-    const uint32_t *zl = z + lane;
-    uint64_t m0 = 0, m1 = 0, m2 = 0;
-    if (p_lo < p_hi) {
-        m0 = __ldg(masks + 3 * (uint64_t)p_lo);
-        m1 = __ldg(masks + 3 * (uint64_t)p_lo + 1);
-        m2 = __ldg(masks + 3 * (uint64_t)p_lo + 2);
-    }
-    for (uint32_t p = p_lo; p < p_hi; ++p) {
-        uint64_t x0 = m0, x1 = m1, x2 = m2;
-        if (p + 1 < p_hi) {  // the next partition's mask, one step ahead
-            m0 = __ldg(masks + 3 * (uint64_t)(p + 1));
-            m1 = __ldg(masks + 3 * (uint64_t)(p + 1) + 1);
-            m2 = __ldg(masks + 3 * (uint64_t)(p + 1) + 2);
-        }
-        uint32_t acc = 0;
-        while (x0) {
-            const int j = __ffsll((long long)x0) - 1;
-            x0 &= x0 - 1;
-            acc |= zl[j * kRouteTStride];
-        }
-        while (x1) {
-            const int j = __ffsll((long long)x1) - 1;
-            x1 &= x1 - 1;
-            acc |= zl[(64 + j) * kRouteTStride];
-        }
-        while (x2) {
-            const int j = __ffsll((long long)x2) - 1;
-            x2 &= x2 - 1;
-            acc |= zl[(128 + j) * kRouteTStride];
-        }
-        const uint32_t r = ~acc & vm;
-        if constexpr (PASS == 0) {
-            const uint32_t c = __reduce_add_sync(0xffffffffu, (uint32_t)__popc(r));
-            if (lane == 0) counts[(uint64_t)p * n_blocks + blk] = c;
-        } else {
-            const uint32_t cnt = __popc(r);
-            uint32_t incl = cnt;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t t = __shfl_up_sync(0xffffffffu, incl, o);
-                if (lane >= o) incl += t;
-            }
-            if (cnt) {
-                unsigned long long o = __ldg(off + (uint64_t)p * n_blocks + blk) + (incl - cnt);
-                uint32_t rr = r;
-                while (rr) {
-                    const int t = __ffs(rr) - 1;
-                    rr &= rr - 1;
-                    if (o < cap) qidx[o] = qbase + (uint32_t)(lo + (uint32_t)t);
-                    ++o;
-                }
-            }
-        }
-    }
-}
-
 // ------------------------------------------------------------------ S3 ---
 constexpr uint32_t kSmallRange = 4096;  // rows per work item of a partition routed to <= kSmallBatch queries
 
@@ -1611,35 +1501,13 @@ cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, co
     return cudaGetLastError();
 }
 
-bool route_transposed() {
-    const char *e = getenv("TM_ROUTE");
-    return e && atoi(e) == 1;
-}
-
-uint64_t route_blocks(uint64_t n_q) {
-    const uint64_t bq = route_transposed() ? kRouteTBlockQ : kRouteBlockQ;
-    return (n_q + bq - 1) / bq;
-}
+uint64_t route_blocks(uint64_t n_q) { return (n_q + kRouteBlockQ - 1) / kRouteBlockQ; }
 
 cudaError_t launch_route(int pass, const uint64_t *masks, uint32_t n_parts, const uint64_t *q0, const uint64_t *q1,
                          const uint64_t *q2, uint64_t n_q, uint32_t *counts, const unsigned long long *off,
                          uint32_t *qidx, unsigned long long cap, cudaStream_t s, uint32_t qbase) {
     const uint64_t nb = route_blocks(n_q);
     if (!nb || !n_parts) return cudaSuccess;
-    if (route_transposed()) {
-        int dev = 0, sms = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        const size_t smem = (size_t)kRouteTWarps * 192 * kRouteTStride * 4;  // 50.7 KB: opt-in
-        auto f = pass == 0 ? k_route_t<0> : k_route_t<1>;
-        cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        if (e != cudaSuccess) return e;
-        const uint64_t want = (uint64_t)std::max(sms, 1) * 8;
-        const uint32_t slices = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>(n_parts, (want + nb - 1) / nb));
-        f<<<grid_for(nb * slices, kRouteTWarps), kRouteTWarps * 32, smem, s>>>(masks, n_parts, q0, q1, q2, n_q, nb,
-                                                                                counts, off, qidx, cap, qbase, slices);
-        return cudaGetLastError();
-    }
     const size_t smem = (size_t)kRouteWarps * 192 * kRouteWB * 4;  // 36 KB: within the default dynamic limit
     static_assert((size_t)kRouteWarps * 192 * kRouteWB * 4 <= 48 * 1024, "route Z needs the opt-in attribute");
     auto f = pass == 0 ? k_route<0> : k_route<1>;
