@@ -387,21 +387,6 @@ __device__ __forceinline__ void store_survivor(uint32_t *sw, uint16_t *sbi, uint
 // IMAD = true: the predicated accumulate is an integer multiply-add (acc += one * bit; the bits of an
 // accumulator are disjoint, so + is |), which runs on the FMA pipe instead of the ALU pipe: the
 // pre-check then puts 2 of its 3 ops per pair on the ALU pipe (scripts/int_peak.cu measures both).
-// One-word form: survivor j passes when (a & ~v_j) == 0 (one LOP3 with a predicate result and the
-// FMA-pipe accumulate per survivor; passes ~6x more pairs to the full check than the two-word form).
-template <int B>
-__device__ __forceinline__ void precheck4x1(uint32_t &c0, uint32_t &c1, uint32_t &c2, uint32_t &c3, uint32_t a,
-                                            uint4 v, uint32_t one) {
-    asm("{\n\t.reg .pred p0, p1, p2, p3;\n\t.reg .b32 t0, t1, t2, t3;\n\t"
-        "not.b32 t0, %5;\n\tnot.b32 t1, %6;\n\tnot.b32 t2, %7;\n\tnot.b32 t3, %8;\n\t"
-        "and.b32 t0, t0, %4;\n\tand.b32 t1, t1, %4;\n\tand.b32 t2, t2, %4;\n\tand.b32 t3, t3, %4;\n\t"
-        "setp.eq.u32 p0, t0, 0;\n\tsetp.eq.u32 p1, t1, 0;\n\tsetp.eq.u32 p2, t2, 0;\n\tsetp.eq.u32 p3, t3, 0;\n\t"
-        "@p0 mad.lo.u32 %0, %13, %9, %0;\n\t@p1 mad.lo.u32 %1, %13, %10, %1;\n\t"
-        "@p2 mad.lo.u32 %2, %13, %11, %2;\n\t@p3 mad.lo.u32 %3, %13, %12, %3;\n\t}"
-        : "+r"(c0), "+r"(c1), "+r"(c2), "+r"(c3)
-        : "r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "n"(B), "n"(B << 1), "n"(B << 2), "n"(B << 3), "r"(one));
-}
-
 template <int B, bool IMAD = false>
 __device__ __forceinline__ void precheck4x2(uint32_t &c0, uint32_t &c1, uint32_t &c2, uint32_t &c3, uint32_t a,
                                             uint4 v, uint32_t b, uint4 u, uint32_t one = 1u) {
@@ -643,7 +628,6 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
     constexpr bool kImad = (OPT & 1) != 0;
     constexpr bool kLean = WORD1 && !STREAM && (OPT & 16) != 0;
     constexpr bool kFused = (OPT & 64) != 0;  // emission into the owners' regions (in-process group)
-    constexpr bool kOneWord = WORD1 && !STREAM && (OPT & 128) != 0;  // one-word pre-check
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -992,9 +976,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                             // ---- pre-check: the lane's word against 32 survivors, pass bits in acc
                             uint32_t c0 = 0, c1 = 0, c2 = 0, c3 = 0;
                             const uint32_t pa = my_plane + k0 * 4, pa2 = my_plane2 + k0 * 4;
-#define TM_PRE(B, o)                                                                                      \
-    if constexpr (kOneWord) precheck4x1<B>(c0, c1, c2, c3, aw, lds128(pa + (o)), p.one);                  \
-    else precheck4x2<B, kImad>(c0, c1, c2, c3, aw, lds128(pa + (o)), aw2, lds128(pa2 + (o)), p.one)
+#define TM_PRE(B, o) precheck4x2<B, kImad>(c0, c1, c2, c3, aw, lds128(pa + (o)), aw2, lds128(pa2 + (o)), p.one)
                             TM_PRE(1u << 0, 0);
                             TM_PRE(1u << 4, 16);
                             if (cnt > 8) {
@@ -1572,7 +1554,6 @@ ScanFn scan_fn_t(int variant) {
         case 13: return k_dense<false, 5 | F>;  // 9 with four rows per lane
         case 14: return k_scan<true, 7, false, 17 | F>;  // 8 + lean tile set-up (the default)
         case 15: return k_dense<false, 21 | F>;  // 13 + the build-time pre-check words (no selects)
-        case 16: return k_scan<true, 7, false, 145 | F>;  // 14 with a one-word pre-check
         default: return nullptr;
     }
 }
