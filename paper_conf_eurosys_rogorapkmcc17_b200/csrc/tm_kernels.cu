@@ -181,30 +181,14 @@ __global__ void __launch_bounds__(kRouteWarps * 32, 6) k_route(const uint64_t *_
     __syncwarp();
     // valid-query mask of each word of the block (warp-uniform)
     const uint64_t nvq = n_q - qb;  // > 0
-    // masks of the lane's partition in the next group are loaded one group ahead (their L2 latency
-    // would otherwise serialise with every group's short bit loop)
-    auto load_mask = [&](uint32_t p, uint64_t (&m)[3]) {
-        m[0] = m[1] = m[2] = 0;
+    for (uint32_t g = g_lo; g < g_hi; g += 32) {
+        const uint32_t p = g + lane;
+        uint64_t m[3] = {0, 0, 0};
         if (p < n_parts) {
             m[0] = __ldg(masks + 3 * (uint64_t)p);
             m[1] = __ldg(masks + 3 * (uint64_t)p + 1);
             m[2] = __ldg(masks + 3 * (uint64_t)p + 2);
         }
-    };
-    // PASS 1: the lane's CSR offset, likewise one group ahead
-    auto load_off = [&](uint32_t p) -> unsigned long long {
-        if constexpr (PASS == 1) return p < n_parts ? __ldg(off + (uint64_t)p * n_blocks + blk) : 0ULL;
-        return 0ULL;
-    };
-    uint64_t mn[3];
-    load_mask(g_lo + lane, mn);
-    unsigned long long on = load_off(g_lo + lane);
-    for (uint32_t g = g_lo; g < g_hi; g += 32) {
-        const uint32_t p = g + lane;
-        uint64_t m[3] = {mn[0], mn[1], mn[2]};
-        const unsigned long long o_here = on;
-        load_mask(g + 32 + lane, mn);
-        on = load_off(g + 32 + lane);
         uint32_t acc[kRouteWB];
 #pragma unroll
         for (int i = 0; i < kRouteWB; ++i) acc[i] = 0;
@@ -236,7 +220,7 @@ __global__ void __launch_bounds__(kRouteWarps * 32, 6) k_route(const uint64_t *_
             }
             counts[(uint64_t)p * n_blocks + blk] = c;
         } else {
-            unsigned long long o = o_here;
+            unsigned long long o = off[(uint64_t)p * n_blocks + blk];
 #pragma unroll
             for (int i = 0; i < kRouteWB; ++i) {
                 const uint64_t lo = 32ULL * i;
