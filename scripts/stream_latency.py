@@ -43,9 +43,12 @@ def main():
             st.replay(q, arrivals)
             st.flush()
             lat, sizes, first_sub, last_done = [], [], None, 0
+            service, wait_disp = [], []
             while (r := st.poll(wait=False)) is not None:
                 lat.append(r["done_ns"] - r["submit_ns"])
                 sizes.append(r["tickets"].size)
+                service.append((r["done_ns"] - r["dispatch_ns"]) / 1e6)          # the GPU call
+                wait_disp.append((r["dispatch_ns"] - r["submit_ns"].min()) / 1e6)  # oldest query's wait
                 first_sub = r["submit_ns"].min() if first_sub is None else min(first_sub, r["submit_ns"].min())
                 last_done = max(last_done, r["done_ns"])
             lat = np.concatenate(lat) / 1e6
@@ -55,6 +58,9 @@ def main():
                               "latency_ms_p50": float(np.percentile(lat, 50)),
                               "latency_ms_p99": float(np.percentile(lat, 99)), "latency_ms_max": float(lat.max()),
                               "batches": int(sizes.size), "mean_batch": float(sizes.mean()),
+                              "service_ms_max": float(max(service)), "service_ms_p50": float(np.median(service)),
+                              "dispatch_wait_ms_max": float(max(wait_disp)),
+                              "slowest_batch": int(sizes[int(np.argmax(service))]),
                               "wall_s": time.time() - t0}), flush=True)
     db.close()
 
