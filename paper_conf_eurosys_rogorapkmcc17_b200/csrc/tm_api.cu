@@ -314,6 +314,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
         TMCK(cudaMemcpyAsync(db->h_ctr, ctr, sizeof(DevCounters), cudaMemcpyDeviceToHost, s));
         if (sp.n_owners) TMCK(cudaMemcpyAsync(db->h_fx, sp.xcnt, kMaxOwners * 8, cudaMemcpyDeviceToHost, s));
         TMCK(cudaStreamSynchronize(s));
+        scan_debug_dump(var);
         const DevCounters c = *db->h_ctr;
         if (c.input_err)
             fail(TM_EINVAL, std::string("queries: malformed CSR found by the encoder (") +

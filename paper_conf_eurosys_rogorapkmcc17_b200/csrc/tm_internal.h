@@ -30,7 +30,7 @@ constexpr int kMaxOwners = 8;       // fused exchange: GPUs of an in-process gro
 constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch); 640 fits 7 CTAs/SM of shared memory and measured 1.3% faster than 512 (profiles/r1v34_ab.txt)
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
-constexpr int kScanVariants = 16;    // k_scan variants (TM_SCAN_VARIANT)
+constexpr int kScanVariants = 17;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {14, 8};  // variants the handle times on its first calls (first = default)
 constexpr int kTuneN = 2;
 constexpr int kTuneDense[] = {13, 9};  // tables without a pre-filter (tile_filter = 2): the dense scan
@@ -99,6 +99,7 @@ cudaError_t launch_items(const unsigned long long *word_off, uint64_t qw, const 
 uint32_t range_rows_env(uint64_t n_rows);  // TM_RANGE_ROWS (multiple of 256), else by table size
 uint32_t unit_target_env();                // TM_UNIT_TARGET, else kUnitTarget
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant);
+void scan_debug_dump(int variant);  // variant 16: pre-check pass statistics to stderr
 int scan_grid(int device, int variant);
 int scan_variant_env();  // -1 = auto-tune
 cudaError_t launch_word_select(const uint64_t *planes, const uint64_t *tand, uint64_t rows, uint8_t *wsel,

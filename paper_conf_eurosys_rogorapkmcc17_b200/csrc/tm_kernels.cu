@@ -607,11 +607,19 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // STREAM: streaming path only (launched for calls of <= kSmallBatch queries), with StreamSmem.
 // OPT: bit 0 = pre-check accumulate on the FMA pipe (precheck4x2<B, true>); bit 4 = lean tile
 // set-up (the two pre-check words read from the build-time wwords plane, no per-lane selects).
+__device__ unsigned long long g_scan_dbg[12];  // OPT & 512: pre-check pass statistics (diagnostic variant)
+
 template <bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
     constexpr bool kImad = (OPT & 1) != 0;
     constexpr bool kLean = WORD1 && !STREAM && (OPT & 16) != 0;
     constexpr bool kFused = (OPT & 64) != 0;  // emission into the owners' regions (in-process group)
+    constexpr bool kDbg = WORD1 && !STREAM && (OPT & 512) != 0;    // pre-check pass statistics (g_scan_dbg)
+    unsigned long long dbg[12];
+    if constexpr (kDbg) {
+#pragma unroll
+        for (int i = 0; i < 12; ++i) dbg[i] = 0;
+    }
     extern __shared__ __align__(16) unsigned char smem_raw[];
     using Smem = typename std::conditional<STREAM, StreamSmem, ScanSmem>::type;
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -979,7 +987,33 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                             uint32_t acc = (c0 | c1) | (c2 | c3);
                             if (cnt < 32) acc &= (1u << cnt) - 1u;
                             if (!valid) acc = 0;
+                            if constexpr (kDbg) {
+                                const uint32_t pc = __popc(acc);
+                                const uint32_t mx = __reduce_max_sync(0xffffffffu, pc);
+                                dbg[0] += __reduce_add_sync(0xffffffffu, pc);
+                                dbg[1] += 1;
+                                dbg[2] += mx;
+                                dbg[3 + (mx == 0 ? 0 : mx == 1 ? 1 : mx == 2 ? 2 : mx <= 4 ? 3 : mx <= 8 ? 4 : mx <= 16 ? 5 : 6)] += 1;
+                                dbg[10] += __reduce_add_sync(0xffffffffu, pc > 8 ? pc : 0u);
+                                dbg[11] += __reduce_add_sync(0xffffffffu, pc ? 1u : 0u);
+                            }
                             // ---- Alg. 3 on the pairs that passed: all six words, then emit
+                            while (__any_sync(0xffffffffu, acc != 0)) {
+                                    const bool has = acc != 0;
+                                    const uint32_t e = k0 + (uint32_t)(__ffs(acc | 0x80000000u) - 1);
+                                    acc &= acc - 1;
+                                    const uint32_t *c = swp + e;
+                                    const bool m = has & (((a0l & ~c[0]) | (a0h & ~c[kSubWStride]) |
+                                                           (a1l & ~c[2 * kSubWStride]) | (a1h & ~c[3 * kSubWStride]) |
+                                                           (a2l & ~c[4 * kSubWStride]) | (a2h & ~c[5 * kSubWStride])) == 0);
+                                    const uint32_t bm = __ballot_sync(0xffffffffu, m);
+                                    if (bm) {
+                                        st_matched += __popc(bm);
+                                        emit_keys<kFused>(m, bm, row, m ? __ldg(sm.qid + sbi[e]) : 0u, p, lane, sm.pend[warp], npend);
+                                    }
+                                }
+                                continue;
+                            }
                             while (__any_sync(0xffffffffu, acc != 0)) {
                                 bool m = false;
                                 uint32_t e = 0;
@@ -1059,6 +1093,10 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
     }
     // the loop ends for all warps together (after the barrier that read the last item)
     flush_pend<kFused>(sm.pend[warp], npend, p, lane);
+    if constexpr (kDbg) {
+        if (lane == 0)
+            for (int i = 0; i < 12; ++i) atomicAdd(&g_scan_dbg[i], dbg[i]);
+    }
     if (lane == 0 && (st_tests | st_checks | st_matched)) {
         atomicAdd(&sm.cnt[0], (unsigned long long)st_tests);
         atomicAdd(&sm.cnt[1], (unsigned long long)st_checks);
@@ -1538,6 +1576,7 @@ ScanFn scan_fn_t(int variant) {
         case 13: return k_dense<false, 5 | F>;  // 9 with four rows per lane
         case 14: return k_scan<true, 7, false, 17 | F>;  // 8 + lean tile set-up (the default)
         case 15: return k_dense<false, 21 | F>;  // 13 + the build-time pre-check words (no selects)
+        case 16: return k_scan<true, 7, false, 17 | 512 | F>;  // 14 + pre-check pass statistics (diagnostic)
         default: return nullptr;
     }
 }
@@ -1558,7 +1597,8 @@ int scan_variant_env() {
     // set-up (default); 6 / 7 = streaming-only kernels (direct check / word pre-check; calls of
     // <= kSmallBatch queries, else mapped to 0 / 5 by the caller); 9-13, 15 = the dense
     // (unfiltered) scan (9 two rows per lane, 13 four, 10 / 12 bulk-copy staged, 11 / 12 without
-    // the FMA accumulate, 15 = 13 with build-time pre-check words).  Unset or unknown (-1): the
+    // the FMA accumulate, 15 = 13 with build-time pre-check words; 16 = 14 printing pre-check pass
+    // statistics, a diagnostic).  Unset or unknown (-1): the
     // handle tunes on its first calls.
     const char *e = getenv("TM_SCAN_VARIANT");
     if (!e) return -1;
@@ -1594,6 +1634,16 @@ int scan_grid(int device, int variant) {
     if (per < 1) per = 1;
     if (sms < 1) sms = 1;
     return sms * per;
+}
+
+void scan_debug_dump(int variant) {
+    // variant 16 (diagnostic): print and reset the pre-check pass statistics of the last scan
+    if (variant != 16) return;
+    unsigned long long h[12] = {}, z[12] = {};
+    if (cudaMemcpyFromSymbol(h, g_scan_dbg, sizeof h) != cudaSuccess) return;
+    cudaMemcpyToSymbol(g_scan_dbg, z, sizeof z);
+    fprintf(stderr, "scan_dbg passes %llu groups %llu iters(sum max) %llu hist[0,1,2,3-4,5-8,9-16,17-32] %llu %llu %llu %llu %llu %llu %llu heavy_passes %llu lanes_with_pass %llu\n",
+            h[0], h[1], h[2], h[3], h[4], h[5], h[6], h[7], h[8], h[9], h[10], h[11]);
 }
 
 cudaError_t launch_scan(const ScanParams &p, int grid, cudaStream_t s, int variant) {

@@ -5,9 +5,9 @@ TAG=${1:-final}
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
 S=$(date +%s); timeout 1500 python -m pytest tests -m gpu -q -s > gpurun_out/${TAG}_pytest.log 2>&1; echo "pytest rc=$? in $(( $(date +%s) - S )) s"; tail -2 gpurun_out/${TAG}_pytest.log
-timeout 1500 compute-sanitizer --tool memcheck --error-exitcode 99 python scripts/sanitize.py 0,5,6,7,8,9,10,11,12,13,14,15 100000 > gpurun_out/${TAG}_sanitize_memcheck.log 2>&1; echo "memcheck rc=$?"; tail -1 gpurun_out/${TAG}_sanitize_memcheck.log
+timeout 1500 compute-sanitizer --tool memcheck --error-exitcode 99 python scripts/sanitize.py 0,5,6,7,8,9,10,11,12,13,14,15,16 100000 > gpurun_out/${TAG}_sanitize_memcheck.log 2>&1; echo "memcheck rc=$?"; tail -1 gpurun_out/${TAG}_sanitize_memcheck.log
 for T in racecheck synccheck; do
-  timeout 1500 compute-sanitizer --tool $T --error-exitcode 99 python scripts/sanitize.py 0,5,6,7,8,9,10,11,12,13,14,15 20000 > gpurun_out/${TAG}_sanitize_${T}.log 2>&1; echo "$T rc=$?"; tail -1 gpurun_out/${TAG}_sanitize_${T}.log
+  timeout 1500 compute-sanitizer --tool $T --error-exitcode 99 python scripts/sanitize.py 0,5,6,7,8,9,10,11,12,13,14,15,16 20000 > gpurun_out/${TAG}_sanitize_${T}.log 2>&1; echo "$T rc=$?"; tail -1 gpurun_out/${TAG}_sanitize_${T}.log
 done
 BID=$(python -c "from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as t; print(t.build_id())")
 for CFG in C3 C4; do

@@ -29,7 +29,7 @@ def check(db, q, db_sig, wl, unique, what):
 
 
 def main():
-    variants = (sys.argv[1] if len(sys.argv) > 1 else "0,5,6,7,8,9,10,11,12,13,14,15").split(",")
+    variants = (sys.argv[1] if len(sys.argv) > 1 else "0,5,6,7,8,9,10,11,12,13,14,15,16").split(",")
     big = int(sys.argv[2]) if len(sys.argv) > 2 else 100_000
     cases = [("C1", tmgen.config("C1"), [(tmb.TM_NO_PARTITIONING, 2), (500, 1), (500, 0)]),
              (f"{big}", tmgen.generate(big, 2000, seed=11, max_partition=5000), [(5000, 1)])]
