@@ -999,22 +999,6 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                             }
                             // ---- Alg. 3 on the pairs that passed: all six words, then emit
                             while (__any_sync(0xffffffffu, acc != 0)) {
-                                    const bool has = acc != 0;
-                                    const uint32_t e = k0 + (uint32_t)(__ffs(acc | 0x80000000u) - 1);
-                                    acc &= acc - 1;
-                                    const uint32_t *c = swp + e;
-                                    const bool m = has & (((a0l & ~c[0]) | (a0h & ~c[kSubWStride]) |
-                                                           (a1l & ~c[2 * kSubWStride]) | (a1h & ~c[3 * kSubWStride]) |
-                                                           (a2l & ~c[4 * kSubWStride]) | (a2h & ~c[5 * kSubWStride])) == 0);
-                                    const uint32_t bm = __ballot_sync(0xffffffffu, m);
-                                    if (bm) {
-                                        st_matched += __popc(bm);
-                                        emit_keys<kFused>(m, bm, row, m ? __ldg(sm.qid + sbi[e]) : 0u, p, lane, sm.pend[warp], npend);
-                                    }
-                                }
-                                continue;
-                            }
-                            while (__any_sync(0xffffffffu, acc != 0)) {
                                 bool m = false;
                                 uint32_t e = 0;
                                 if (acc) {
