@@ -47,7 +47,7 @@
 extern "C" {
 #endif
 
-#define TM_ABI_VERSION 4u
+#define TM_ABI_VERSION 5u  /* 5: tm_tagsets.vocab_hash (pre-hashed vocabulary) */
 /* Bloom filter width and number of hash functions. */
 #define TM_SIG_BITS 192u
 #define TM_SIG_WORDS 3u
@@ -103,6 +103,14 @@ typedef struct {
     uint64_t n_vocab;
     uint64_t n_tags;
     uint64_t n_sets;
+    /* Pre-hashed vocabulary (SURVEY 8(b) "n_tags pre-hashed tags"; 8(d): the throughput protocol
+     * times pre-hashed query tags): NULL, or n_vocab values FNV-1a-64(bytes of string v) (DESIGN.md
+     * reading R1, the hash tm_encode applies to the bytes).  When given, vocab_bytes must be NULL,
+     * n_bytes 0 and vocab_off is ignored (may be NULL); with tag_idx NULL the hashes are the tags.
+     * Accepted by the match calls (tm_match_batch*, tm_match_batch_sharded_device), tm_encode and a
+     * config's plan_sample; calls that keep tag strings (tm_build, tm_add_sets, tm_stream_replay,
+     * exact mode) fail with TM_EINVAL.  Device-resident on tm_match_batch_device. */
+    const uint64_t *vocab_hash;
 } tm_tagsets;
 
 typedef struct {

@@ -69,11 +69,37 @@ void pinned_put(PinnedBlock *b) {
 }
 
 // ------------------------------------------------------------ validation --
+// a pre-hashed vocabulary (tm_tagsets.vocab_hash) comes without strings
+static void check_hashed(const tm_tagsets *t, const std::string &w) {
+    if (t->vocab_bytes || t->n_bytes) fail(TM_EINVAL, w + ": vocab_hash given together with vocab_bytes / n_bytes");
+    if (t->n_vocab > 0xFFFFFFFFull) fail(TM_ERANGE, w + ": more than 2^32-1 vocabulary strings");
+    if (t->n_tags > 0 && t->tag_idx == nullptr && t->n_tags != t->n_vocab)
+        fail(TM_EINVAL, w + ": tag_idx NULL requires n_tags == n_vocab");
+    if (t->n_tags > 0 && t->n_vocab == 0) fail(TM_EINVAL, w + ": tags without a vocabulary");
+}
+
+void require_strings(const tm_tagsets *t, const char *what) {
+    if (t && t->vocab_hash)
+        fail(TM_EINVAL, std::string(what) + ": this call needs tag strings (vocab_hash is accepted by the match calls, "
+                                            "tm_encode and plan_sample only)");
+}
+
 void check_tagsets_host(const tm_tagsets *t, const char *what) {
     const std::string w(what);
     if (!t) fail(TM_EINVAL, w + ": NULL tagsets");
     if (t->n_sets > 0xFFFFFFFFull) fail(TM_ERANGE, w + ": more than 2^32-1 sets");
     if (!t->set_off) fail(TM_EINVAL, w + ": set_off is NULL");
+    if (t->vocab_hash) {
+        check_hashed(t, w);
+        if (t->set_off[0] != 0 || t->set_off[t->n_sets] != t->n_tags)
+            fail(TM_EINVAL, w + ": set_off[0] != 0 or set_off[n_sets] != n_tags");
+        for (uint64_t i = 0; i < t->n_sets; ++i)
+            if (t->set_off[i + 1] < t->set_off[i]) fail(TM_EINVAL, w + ": set_off not non-decreasing");
+        if (t->tag_idx)
+            for (uint64_t i = 0; i < t->n_tags; ++i)
+                if (t->tag_idx[i] >= t->n_vocab) fail(TM_EINVAL, w + ": tag_idx out of range");
+        return;
+    }
     if (t->n_vocab > 0 && !t->vocab_off) fail(TM_EINVAL, w + ": vocab_off is NULL");
     if (t->n_bytes > 0 && !t->vocab_bytes) fail(TM_EINVAL, w + ": vocab_bytes is NULL");
     if (t->n_tags > 0 && t->tag_idx == nullptr && t->n_tags != t->n_vocab)
@@ -102,6 +128,12 @@ void check_tagsets_shape(const tm_tagsets *t, const char *what) {
     if (!t) fail(TM_EINVAL, w + ": NULL tagsets");
     if (t->n_sets > 0xFFFFFFFFull) fail(TM_ERANGE, w + ": more than 2^32-1 sets");
     if (!t->set_off) fail(TM_EINVAL, w + ": set_off is NULL");
+    if (t->vocab_hash) {
+        check_hashed(t, w);
+        if (t->set_off[0] != 0 || t->set_off[t->n_sets] != t->n_tags)
+            fail(TM_EINVAL, w + ": set_off[0] != 0 or set_off[n_sets] != n_tags");
+        return;
+    }
     if (t->n_vocab > 0 && !t->vocab_off) fail(TM_EINVAL, w + ": vocab_off is NULL");
     if (t->n_bytes > 0 && !t->vocab_bytes) fail(TM_EINVAL, w + ": vocab_bytes is NULL");
     if (t->n_tags > 0 && t->tag_idx == nullptr && t->n_tags != t->n_vocab)
@@ -120,6 +152,10 @@ void check_tagsets_device(const tm_tagsets *t) {
     if (!t) fail(TM_EINVAL, "queries: NULL tagsets");
     if (t->n_sets > 0xFFFFFFFFull) fail(TM_ERANGE, "queries: more than 2^32-1 sets");
     if (t->n_sets > 0 && !t->set_off) fail(TM_EINVAL, "queries: set_off is NULL");
+    if (t->vocab_hash) {
+        check_hashed(t, "queries");
+        return;
+    }
     if (t->n_vocab > 0 && !t->vocab_off) fail(TM_EINVAL, "queries: vocab_off is NULL");
     if (t->n_bytes > 0 && !t->vocab_bytes) fail(TM_EINVAL, "queries: vocab_bytes is NULL");
     if (t->n_tags > 0 && t->tag_idx == nullptr && t->n_tags != t->n_vocab)
@@ -151,6 +187,8 @@ void *cub_tmp(tm_db *db, size_t bytes) {
 // of a replicated multi-GPU database; default: all), with their batch-global indices.
 uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, uint64_t qlo, uint64_t qn) {
     NvtxRange nv_call("tm_match");
+    if (db->cfg.exact && q->vocab_hash)  // the exact check compares tag strings
+        fail(TM_EINVAL, "queries: exact mode needs tag strings, not vocab_hash");
     tm_stats_t &st = db->st;
     const uint64_t Qall = q->n_sets;
     if (qlo > Qall) qlo = Qall;
@@ -189,7 +227,7 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
     // the query CSR is validated by the encoder kernels themselves (input_err, checked below with
     // the scan counters): no O(n) host pass over the batch on the call's critical path
     TMCK(cudaMemsetAsync(&ctr->input_err, 0, sizeof(ctr->input_err), s));
-    TMCK(launch_hash_vocab(q->vocab_bytes, q->vocab_off, q->n_vocab, q->n_bytes, db->vsig.as<uint64_t>(),
+    TMCK(launch_hash_vocab(q->vocab_bytes, q->vocab_off, q->vocab_hash, q->n_vocab, q->n_bytes, db->vsig.as<uint64_t>(),
                            &ctr->input_err, s));
     TMCK(launch_encode_sets(db->vsig.as<uint64_t>(), q->tag_idx, q->set_off, Q, q->n_tags, q->n_vocab, q0, q1, q2,
                             &ctr->input_err, s));
@@ -494,7 +532,7 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
         d_vsig.ensure(std::max<uint64_t>(sets->n_vocab, 1) * 24);
         d_planes.ensure(N * 24);
         uint64_t *w0 = d_planes.as<uint64_t>(), *w1 = w0 + N, *w2 = w1 + N;
-        TMCK(launch_hash_vocab(d_bytes.as<uint8_t>(), d_voff.as<uint64_t>(), sets->n_vocab, sets->n_bytes,
+        TMCK(launch_hash_vocab(d_bytes.as<uint8_t>(), d_voff.as<uint64_t>(), nullptr, sets->n_vocab, sets->n_bytes,
                                d_vsig.as<uint64_t>(), nullptr, s));
         TMCK(launch_encode_sets(d_vsig.as<uint64_t>(), (sets->tag_idx && sets->n_tags) ? d_tidx.as<uint32_t>() : nullptr,
                                 d_soff.as<uint64_t>(), N, sets->n_tags, sets->n_vocab, w0, w1, w2, nullptr, s));
@@ -765,12 +803,17 @@ tm_tagsets upload_queries(tm_db *db, const tm_tagsets *q, cudaStream_t s) {
     db->in_soff.ensure((q->n_sets + 1) * 8);
     TMCK(cudaMemcpyAsync(db->in_soff.p, q->set_off, (q->n_sets + 1) * 8, cudaMemcpyHostToDevice, s));
     dq.set_off = db->in_soff.as<uint64_t>();
+    if (q->vocab_hash && q->n_vocab) {  // pre-hashed vocabulary: the hashes instead of the strings
+        db->in_vhash.ensure(q->n_vocab * 8);
+        TMCK(cudaMemcpyAsync(db->in_vhash.p, q->vocab_hash, q->n_vocab * 8, cudaMemcpyHostToDevice, s));
+        dq.vocab_hash = db->in_vhash.as<uint64_t>();
+    }
     if (q->n_bytes) {
         db->in_bytes.ensure(q->n_bytes);
         TMCK(cudaMemcpyAsync(db->in_bytes.p, q->vocab_bytes, q->n_bytes, cudaMemcpyHostToDevice, s));
         dq.vocab_bytes = db->in_bytes.as<uint8_t>();
     }
-    if (q->n_vocab) {
+    if (q->n_vocab && !q->vocab_hash) {
         db->in_voff.ensure((q->n_vocab + 1) * 8);
         TMCK(cudaMemcpyAsync(db->in_voff.p, q->vocab_off, (q->n_vocab + 1) * 8, cudaMemcpyHostToDevice, s));
         dq.vocab_off = db->in_voff.as<uint64_t>();
@@ -823,6 +866,7 @@ tm_status tm_build(const tm_tagsets *sets, const uint64_t *key_off, const uint32
     TM_API_BEGIN
     if (!out) fail(TM_EINVAL, "out is NULL");
     check_tagsets_host(sets, "sets");
+    require_strings(sets, "sets");
     if (cfg && cfg->n_gpus > 1) {  // in-process multi-GPU database (tm_group.cu)
         tm_db *top = new_db(cfg);
         try {
@@ -969,7 +1013,7 @@ tm_status tm_encode(const tm_tagsets *sets, uint64_t *sig_out, int device) {
     if (!N) return TM_OK;
     cudaStream_t s;
     TMCK(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
-    DevBuf b, vo, ti, so, vs, pl;
+    DevBuf b, vo, ti, so, vs, pl, vh;
     struct Rel {
         std::vector<DevBuf *> v;
         cudaStream_t s;
@@ -978,14 +1022,23 @@ tm_status tm_encode(const tm_tagsets *sets, uint64_t *sig_out, int device) {
             for (auto *x : v) x->release();
             cudaStreamDestroy(s);
         }
-    } rel{{&b, &vo, &ti, &so, &vs, &pl}, s};
+    } rel{{&b, &vo, &ti, &so, &vs, &pl, &vh}, s};
     b.ensure(std::max<uint64_t>(sets->n_bytes, 1));
     vo.ensure((sets->n_vocab + 1) * 8);
     so.ensure((N + 1) * 8);
     vs.ensure(std::max<uint64_t>(sets->n_vocab, 1) * 24);
     pl.ensure(N * 24);
     if (sets->n_bytes) TMCK(cudaMemcpyAsync(b.p, sets->vocab_bytes, sets->n_bytes, cudaMemcpyHostToDevice, s));
-    if (sets->n_vocab) TMCK(cudaMemcpyAsync(vo.p, sets->vocab_off, (sets->n_vocab + 1) * 8, cudaMemcpyHostToDevice, s));
+    const uint64_t *dvh = nullptr;
+    if (sets->vocab_hash) {
+        if (sets->n_vocab) {
+            vh.ensure(sets->n_vocab * 8);
+            TMCK(cudaMemcpyAsync(vh.p, sets->vocab_hash, sets->n_vocab * 8, cudaMemcpyHostToDevice, s));
+        }
+        dvh = vh.as<uint64_t>();
+    } else if (sets->n_vocab) {
+        TMCK(cudaMemcpyAsync(vo.p, sets->vocab_off, (sets->n_vocab + 1) * 8, cudaMemcpyHostToDevice, s));
+    }
     TMCK(cudaMemcpyAsync(so.p, sets->set_off, (N + 1) * 8, cudaMemcpyHostToDevice, s));
     const uint32_t *dti = nullptr;
     if (sets->tag_idx && sets->n_tags) {
@@ -994,7 +1047,7 @@ tm_status tm_encode(const tm_tagsets *sets, uint64_t *sig_out, int device) {
         dti = ti.as<uint32_t>();
     }
     uint64_t *w0 = pl.as<uint64_t>(), *w1 = w0 + N, *w2 = w1 + N;
-    TMCK(launch_hash_vocab(b.as<uint8_t>(), vo.as<uint64_t>(), sets->n_vocab, sets->n_bytes, vs.as<uint64_t>(),
+    TMCK(launch_hash_vocab(b.as<uint8_t>(), vo.as<uint64_t>(), dvh, sets->n_vocab, sets->n_bytes, vs.as<uint64_t>(),
                            nullptr, s));
     TMCK(launch_encode_sets(vs.as<uint64_t>(), dti, so.as<uint64_t>(), N, sets->n_tags, sets->n_vocab, w0, w1, w2,
                             nullptr, s));

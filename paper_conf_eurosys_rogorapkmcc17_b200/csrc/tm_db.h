@@ -150,7 +150,7 @@ struct tm_db {
     std::vector<uint32_t> h_part_row;
     double build_ms = 0;
     // per-call workspace
-    DevBuf in_bytes, in_voff, in_tidx, in_soff;  // host-API staging of the queries
+    DevBuf in_bytes, in_voff, in_tidx, in_soff, in_vhash;  // host-API staging of the queries
     DevBuf vsig, qplanes, bm, word_off, qidx, qoff, item_cnt, item_off, out, out_alt, res_q, res_k, res_off, tmp, ctr;
     DevCounters *h_ctr = nullptr;  // pinned
     unsigned long long *h_nuniq = nullptr;
@@ -198,6 +198,7 @@ tm_status translate(const CudaFail &f);
 int check_device(int dev);
 void check_tagsets_device(const tm_tagsets *t);
 void check_tagsets_host(const tm_tagsets *t, const char *what);
+void require_strings(const tm_tagsets *t, const char *what);  // TM_EINVAL for a pre-hashed vocabulary
 int bits_for(uint64_t n);
 // partition -> shard plan of the handle's config (tm_shard.cu): contiguous ranges of ~equal
 // estimated work; one shard: all 0; replicated: all = this handle's shard (it keeps everything)

@@ -82,8 +82,9 @@ struct ScanParams {
 
 // ------------------------------------------------------------ launchers --
 // All launchers are asynchronous on `s` and return the launch error.
-cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_t n_vocab, uint64_t n_bytes,
-                              uint64_t *vsig, unsigned int *err, cudaStream_t s);
+// hashes: NULL, or the pre-hashed vocabulary (tm_tagsets.vocab_hash; bytes / off then unused)
+cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, const uint64_t *hashes, uint64_t n_vocab,
+                              uint64_t n_bytes, uint64_t *vsig, unsigned int *err, cudaStream_t s);
 cudaError_t launch_encode_sets(const uint64_t *vsig, const uint32_t *tag_idx, const uint64_t *set_off,
                                uint64_t n_sets, uint64_t n_tags, uint64_t n_vocab, uint64_t *w0, uint64_t *w1,
                                uint64_t *w2, unsigned int *err, cudaStream_t s);

@@ -42,19 +42,25 @@ inline unsigned grid_for(uint64_t n, unsigned bs) {
 // floor(z*192/2^64) of the first 7 SplitMix64 outputs seeded with it.
 // The CSR is validated on the device (non-decreasing offsets inside [0, n_bytes], end points):
 // a malformed string sets *err and is hashed as empty, so nothing is read out of bounds.
-__global__ void k_hash_vocab(const uint8_t *__restrict__ bytes, const uint64_t *__restrict__ off, uint64_t n,
-                             uint64_t n_bytes, uint64_t *__restrict__ vsig, unsigned int *err) {
+// hashes != NULL: the vocabulary is given pre-hashed (tm_tagsets.vocab_hash): h = hashes[v].
+__global__ void k_hash_vocab(const uint8_t *__restrict__ bytes, const uint64_t *__restrict__ off,
+                             const uint64_t *__restrict__ hashes, uint64_t n, uint64_t n_bytes,
+                             uint64_t *__restrict__ vsig, unsigned int *err) {
     uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (v >= n) return;
-    uint64_t b = off[v], e = off[v + 1];
-    if (e < b || e > n_bytes || (v == 0 && b != 0) || (v == n - 1 && e != n_bytes)) {
-        if (err) atomicOr(err, 1u);
-        e = b = 0;
-    }
     uint64_t h = kFnvOffset;
-    for (uint64_t i = b; i < e; ++i) {
-        h ^= (uint64_t)__ldg(bytes + i);
-        h *= kFnvPrime;
+    if (hashes) {
+        h = __ldg(hashes + v);
+    } else {
+        uint64_t b = off[v], e = off[v + 1];
+        if (e < b || e > n_bytes || (v == 0 && b != 0) || (v == n - 1 && e != n_bytes)) {
+            if (err) atomicOr(err, 1u);
+            e = b = 0;
+        }
+        for (uint64_t i = b; i < e; ++i) {
+            h ^= (uint64_t)__ldg(bytes + i);
+            h *= kFnvPrime;
+        }
     }
     uint64_t s[3] = {0, 0, 0};
     uint64_t state = h;
@@ -1491,10 +1497,10 @@ struct WidenAt {
 }  // namespace
 
 // ------------------------------------------------------------ launchers ---
-cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, uint64_t n_vocab, uint64_t n_bytes,
-                              uint64_t *vsig, unsigned int *err, cudaStream_t s) {
+cudaError_t launch_hash_vocab(const uint8_t *bytes, const uint64_t *off, const uint64_t *hashes, uint64_t n_vocab,
+                              uint64_t n_bytes, uint64_t *vsig, unsigned int *err, cudaStream_t s) {
     if (!n_vocab) return cudaSuccess;
-    k_hash_vocab<<<grid_for(n_vocab, 256), 256, 0, s>>>(bytes, off, n_vocab, n_bytes, vsig, err);
+    k_hash_vocab<<<grid_for(n_vocab, 256), 256, 0, s>>>(bytes, off, hashes, n_vocab, n_bytes, vsig, err);
     return cudaGetLastError();
 }
 

@@ -194,7 +194,7 @@ std::vector<uint64_t> sample_routes(tm_db *db, const std::vector<Partition> &par
     vsig.ensure(std::max<uint64_t>(dq.n_vocab, 1) * 24);
     planes.ensure(Qs * 24);
     uint64_t *q0 = planes.as<uint64_t>(), *q1 = q0 + Qs, *q2 = q1 + Qs;
-    TMCK(launch_hash_vocab(dq.vocab_bytes, dq.vocab_off, dq.n_vocab, dq.n_bytes, vsig.as<uint64_t>(), nullptr, s));
+    TMCK(launch_hash_vocab(dq.vocab_bytes, dq.vocab_off, dq.vocab_hash, dq.n_vocab, dq.n_bytes, vsig.as<uint64_t>(), nullptr, s));
     TMCK(launch_encode_sets(vsig.as<uint64_t>(), dq.n_tags ? dq.tag_idx : nullptr, dq.set_off, Qs, dq.n_tags,
                             dq.n_vocab, q0, q1, q2, nullptr, s));
     std::vector<uint64_t> hm(3 * P);

@@ -161,6 +161,7 @@ tm_status tm_add_sets(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off
     TM_API_BEGIN
     tmb::Store &st = tmb::mutable_store(db);
     tmb::check_tagsets_host(sets, "sets");
+    tmb::require_strings(sets, "sets");
     const uint64_t N = sets->n_sets;
     if (key_off) {
         if (key_off[0] != 0) fail(TM_EINVAL, "key_off[0] != 0");

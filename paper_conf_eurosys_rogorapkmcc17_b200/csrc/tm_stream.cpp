@@ -260,6 +260,7 @@ tm_status tm_stream_replay(tm_stream *st, const tm_tagsets *q, const uint64_t *a
     // the whole batch is validated before the first query is queued (offsets monotone and in
     // range, tag indices < n_vocab): a malformed batch queues nothing
     tmb::check_tagsets_host(q, "queries");
+    tmb::require_strings(q, "queries");
     const uint64_t t0 = tmb::now_ns();
     for (uint64_t i = 0; i < q->n_sets; ++i) {
         tmb::Query one;

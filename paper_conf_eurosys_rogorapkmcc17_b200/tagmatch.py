@@ -33,7 +33,7 @@ class TagMatchError(RuntimeError):
 class tm_tagsets(ctypes.Structure):
     _fields_ = [("vocab_bytes", ctypes.c_void_p), ("vocab_off", ctypes.c_void_p), ("tag_idx", ctypes.c_void_p),
                 ("set_off", ctypes.c_void_p), ("n_bytes", ctypes.c_uint64), ("n_vocab", ctypes.c_uint64),
-                ("n_tags", ctypes.c_uint64), ("n_sets", ctypes.c_uint64)]
+                ("n_tags", ctypes.c_uint64), ("n_sets", ctypes.c_uint64), ("vocab_hash", ctypes.c_void_p)]
 
 
 class tm_config(ctypes.Structure):
@@ -203,11 +203,27 @@ class HostTagSets:
         """From any object with vocab_bytes / vocab_off / tag_idx / set_off (e.g. tmgen.TagSets)."""
         return cls(ts.vocab_bytes, ts.vocab_off, ts.tag_idx, ts.set_off)
 
+    @classmethod
+    def hashed(cls, vocab_hash, tag_idx, set_off):
+        """A pre-hashed vocabulary (tm_tagsets.vocab_hash: FNV-1a-64 of each vocabulary string, the
+        caller's own hashing; no strings are passed)."""
+        self = cls.__new__(cls)
+        self.vh = np.ascontiguousarray(vocab_hash, dtype=np.uint64)
+        self.vb = self.vo = None
+        self.ti = None if tag_idx is None else np.ascontiguousarray(tag_idx, dtype=np.uint32)
+        self.so = np.ascontiguousarray(set_off, dtype=np.uint64)
+        n_tags = int(self.so[-1]) if self.so.size else 0
+        self.c = tm_tagsets(None, None, _ptr(self.ti) if self.ti is not None else None, _ptr(self.so), 0,
+                            self.vh.size, n_tags, max(self.so.size - 1, 0), _ptr(self.vh))
+        return self
 
-def device_tagsets(vocab_bytes_ptr, vocab_off_ptr, tag_idx_ptr, set_off_ptr, n_bytes, n_vocab, n_tags, n_sets):
-    """tm_tagsets of device pointers (ints, e.g. torch tensor data_ptr())."""
+
+def device_tagsets(vocab_bytes_ptr, vocab_off_ptr, tag_idx_ptr, set_off_ptr, n_bytes, n_vocab, n_tags, n_sets,
+                   vocab_hash_ptr=0):
+    """tm_tagsets of device pointers (ints, e.g. torch tensor data_ptr()); vocab_hash_ptr: a
+    pre-hashed vocabulary instead of vocab_bytes / vocab_off."""
     return tm_tagsets(vocab_bytes_ptr or None, vocab_off_ptr or None, tag_idx_ptr or None, set_off_ptr or None,
-                      n_bytes, n_vocab, n_tags, n_sets)
+                      n_bytes, n_vocab, n_tags, n_sets, vocab_hash_ptr or None)
 
 
 def make_config(max_partition=0, device=-1, n_shards=1, shard=0, tile_filter=0, row_order=0,
