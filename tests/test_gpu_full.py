@@ -1,4 +1,5 @@
-"""Parity at BASELINE.json's full sizes in the configuration bench.py times, checked on
+"""Parity at BASELINE.json's full sizes in the configuration bench.py times (auto MAX_P; C3 / C4
+also at the paper's 200K, whose whole output must be identical), checked on
 seeded samples of queries that the oracle (O2, brute force over the WHOLE database, no
 partitioning or pre-filter: the plain definition of SURVEY 8(c)) computes one by one, plus
 size-independent properties of the whole output:
@@ -57,34 +58,45 @@ def full(request):
     t = time.time()
     wl = tmgen.config(name)
     print(f"\n{name}: generated {wl.db.n_sets} sets, {wl.queries.n_sets} queries in {time.time() - t:.1f} s")
-    t = time.time()
-    # the layout bench.py times by default: balanced splits + tile AND masks (R18)
-    db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=1, row_order=1)
-    st = db.stats()
-    print(f"{name}: built in {time.time() - t:.1f} s: {st['n_partitions']} partitions, {st['n_unique']} rows")
+    dbs = []
+    # the layout bench.py times by default: balanced splits + tile AND masks (R18), at the
+    # MAX_P bench.py uses (TM_AUTO_MAX_PARTITION: 5K at C3, 10K at C4) and at the paper's 200K
+    for mp in (tmb.TM_AUTO_MAX_PARTITION, wl.max_partition):
+        t = time.time()
+        db = tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=mp, tile_filter=1, row_order=1)
+        st = db.stats()
+        print(f"{name}: built in {time.time() - t:.1f} s: {st['n_partitions']} partitions, {st['n_unique']} rows")
+        dbs.append(db)
     db_sig = o2.encode(wl.db)
-    yield name, wl, db, db_sig
-    db.close()
+    yield name, wl, dbs, db_sig
+    for db in dbs:
+        db.close()
     del wl, db_sig
     gc.collect()
 
 
 @pytest.mark.parametrize("unique", [False, True])
 def test_full_size_sampled_parity(full, unique):
-    name, wl, db, db_sig = full
-    t = time.time()
-    gq, gk = db.match_batch(wl.queries, unique)
-    st = db.stats()
-    print(f"{name} unique={unique}: {gq.size} pairs in {time.time() - t:.2f} s (scan {st['scan_ms']:.1f} ms, "
-          f"{st['candidate_pairs']:.3e} candidate pairs, {st['pair_checks']:.3e} checks)")
-    # properties of the whole output: sorted, ids in range, every query matches its base
-    _sorted_props(gq, gk, wl.queries.n_sets, unique)
-    assert np.unique(gq).size == wl.queries.n_sets
+    name, wl, dbs, db_sig = full
+    outs = []
+    for db in dbs:
+        t = time.time()
+        gq, gk = db.match_batch(wl.queries, unique)
+        st = db.stats()
+        print(f"{name} unique={unique} ({st['n_partitions']} partitions): {gq.size} pairs in {time.time() - t:.2f} s "
+              f"(scan {st['scan_ms']:.1f} ms, {st['candidate_pairs']:.3e} candidate pairs, "
+              f"{st['pair_checks']:.3e} checks)")
+        # properties of the whole output: sorted, ids in range, every query matches its base
+        _sorted_props(gq, gk, wl.queries.n_sets, unique)
+        assert np.unique(gq).size == wl.queries.n_sets
+        outs.append((gq, gk))
+    # partitioning is lossless (Alg. 1 / Alg. 2): both MAX_P give the same whole output
+    assert np.array_equal(outs[0][0], outs[1][0]) and np.array_equal(outs[0][1], outs[1][1])
     # sampled bit-exact parity against brute force over the whole database
     rng = np.random.default_rng(2024 + unique + (10 if name == "C4" else 0))
     qsel = np.sort(rng.choice(wl.queries.n_sets, SAMPLE[name], replace=False))
     t = time.time()
-    n = _sample_parity(db_sig, wl.key_off, wl.keys, wl.queries, gq, gk, qsel, unique)
+    n = _sample_parity(db_sig, wl.key_off, wl.keys, wl.queries, outs[0][0], outs[0][1], qsel, unique)
     print(f"oracle sample of {qsel.size} queries ({n} pairs): {time.time() - t:.1f} s")
 
 
@@ -99,7 +111,9 @@ def test_c5_query_size_sweep_sampled_parity():
     print(f"\nC5: generated in {time.time() - t:.1f} s")
     db_sig = o2.encode(wl.db)
     rates = []
-    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=200_000, tile_filter=1, row_order=1) as db:
+    # the MAX_P of scripts/sweep_c5.py and bench.py (TM_AUTO_MAX_PARTITION: 5K at 100M sets)
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=tmb.TM_AUTO_MAX_PARTITION, tile_filter=1,
+                      row_order=1) as db:
         for tt in C5_TOTALS:
             q = batches[tt]
             for unique in (False, True):
@@ -121,8 +135,8 @@ def test_crafted_full_size_sampled_parity(name):
     whole-output properties, then bit-exact parity on a 192-query sample against O2 brute force
     over the whole database, for match and match-unique."""
     wl = tmgen.config(name)
-    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=1,
-                      row_order=1) as db:
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=tmb.TM_AUTO_MAX_PARTITION, tile_filter=1,
+                      row_order=1) as db:   # bench.py's MAX_P for these (auto)
         db_sig = o2.encode(wl.db)
         for unique in (False, True):
             gq, gk = db.match_batch(wl.queries, unique)
