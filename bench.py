@@ -432,9 +432,13 @@ def run_ours(args):
     h2d_bytes = sum(a.nbytes for a in qarr)
 
     def step_device():
-        if sharded:
-            return db.match_batch_sharded_device(dq, unique, stream.cuda_stream)
-        return db.match_batch_device(dq, unique, stream.cuda_stream)
+        torch.cuda.nvtx.range_push("bench_device")   # ncu selects the device step's launches by this range
+        try:
+            if sharded:
+                return db.match_batch_sharded_device(dq, unique, stream.cuda_stream)
+            return db.match_batch_device(dq, unique, stream.cuda_stream)
+        finally:
+            torch.cuda.nvtx.range_pop()
 
     def step_e2e():
         """Public API end to end: host queries in, host pairs out; returns D2H bytes."""

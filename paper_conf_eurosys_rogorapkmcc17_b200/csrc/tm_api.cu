@@ -185,7 +185,8 @@ void *cub_tmp(tm_db *db, size_t bytes) {
 // Run the whole path for device-resident queries; leaves n results in db->res_q/res_k.
 // Every query of the batch is encoded; queries [qlo, qlo + qn) are matched (the share of one GPU
 // of a replicated multi-GPU database; default: all), with their batch-global indices.
-uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, uint64_t qlo, uint64_t qn) {
+uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, uint64_t qlo, uint64_t qn,
+                    bool encoded) {
     NvtxRange nv_call("tm_match");
     if (db->cfg.exact && q->vocab_hash)  // the exact check compares tag strings
         fail(TM_EINVAL, "queries: exact mode needs tag strings, not vocab_hash");
@@ -221,17 +222,21 @@ uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, 
     TMCK(cudaEventRecord(db->ev[0], s));
 
     // S1: encode
-    db->vsig.ensure(std::max<uint64_t>(q->n_vocab, 1) * 24);
-    db->qplanes.ensure(Q * 24);
+    if (!encoded) {
+        db->vsig.ensure(std::max<uint64_t>(q->n_vocab, 1) * 24);
+        db->qplanes.ensure(Q * 24);
+    }
     uint64_t *q0 = db->qplanes.as<uint64_t>(), *q1 = q0 + Q, *q2 = q1 + Q;
-    // the query CSR is validated by the encoder kernels themselves (input_err, checked below with
-    // the scan counters): no O(n) host pass over the batch on the call's critical path
-    TMCK(cudaMemsetAsync(&ctr->input_err, 0, sizeof(ctr->input_err), s));
-    TMCK(launch_hash_vocab(q->vocab_bytes, q->vocab_off, q->vocab_hash, q->n_vocab, q->n_bytes, db->vsig.as<uint64_t>(),
-                           &ctr->input_err, s));
-    TMCK(launch_encode_sets(db->vsig.as<uint64_t>(), q->tag_idx, q->set_off, Q, q->n_tags, q->n_vocab, q0, q1, q2,
-                            &ctr->input_err, s));
-    launches += 2;
+    if (!encoded) {
+        // the query CSR is validated by the encoder kernels themselves (input_err, checked below with
+        // the scan counters): no O(n) host pass over the batch on the call's critical path
+        TMCK(cudaMemsetAsync(&ctr->input_err, 0, sizeof(ctr->input_err), s));
+        TMCK(launch_hash_vocab(q->vocab_bytes, q->vocab_off, q->vocab_hash, q->n_vocab, q->n_bytes,
+                               db->vsig.as<uint64_t>(), &ctr->input_err, s));
+        TMCK(launch_encode_sets(db->vsig.as<uint64_t>(), q->tag_idx, q->set_off, Q, q->n_tags, q->n_vocab, q0, q1,
+                                q2, &ctr->input_err, s));
+        launches += 2;
+    }
     TMCK(cudaEventRecord(db->ev[1], s));
 
     // S2: route (Alg. 2, bit-sliced): per (partition, route block) counts, scanned to the
@@ -698,13 +703,16 @@ void destroy_db(tm_db *db) {
                       &db->res_k, &db->res_off, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,
                       &db->mk, &db->xv_bytes, &db->xv_off, &db->xv_hash, &db->xv_pos, &db->xv_canon, &db->xs_off,
                       &db->xs_ids, &db->xk_off, &db->xk_keys, &db->xq_canon, &db->xq_ids, &db->xflag, &db->xcnt,
-                      &db->xkoff, &db->xkcnt})
+                      &db->xkoff, &db->xkcnt, &db->res_kb})
         b->release();
     for (auto &e : db->ev)
         if (e) cudaEventDestroy(e);
     if (db->h_ctr) cudaFreeHost(db->h_ctr);
     if (db->h_nuniq) cudaFreeHost(db->h_nuniq);
     if (db->h_fx) cudaFreeHost(db->h_fx);
+    for (auto &e : db->xev)
+        if (e) cudaEventDestroy(e);
+    if (db->xstream) cudaStreamDestroy(db->xstream);
     if (db->stream) cudaStreamDestroy(db->stream);
     if (prev >= 0) cudaSetDevice(prev);
     delete db;
@@ -857,6 +865,114 @@ void rebuild(tm_db *db, const tm_tagsets *sets, const uint32_t *keys, const tm_c
     fresh->nccl_comm = nullptr;
     destroy_db(fresh);
 }
+// Query ranges of a pipelined tm_match_batch_csr: the result's device-to-host copy (4 B per pair,
+// ~0.85 GB at C3, PCIe-bound) of range k runs on a copy stream while the GPU matches range k + 1,
+// so only the last range's copy stays on the critical path.  TM_PIPELINE=n forces n ranges (1 = off).
+uint32_t pipeline_ranges(uint64_t Q) {
+    const char *e = getenv("TM_PIPELINE");
+    const long forced = e ? atol(e) : 0;
+    if (forced >= 1) return (uint32_t)std::min<long>(forced, 64);
+    return Q >= (1ULL << 18) ? 4u : 1u;  // smaller batches: the per-range fixed cost outweighs the copy
+}
+
+void csr_pipelined(tm_db *db, const tm_tagsets *dq, int unique, uint32_t S, tm_csr *out) {
+    cudaStream_t s = db->stream;
+    const uint64_t Q = dq->n_sets;
+    if (!db->xstream) {
+        TMCK(cudaStreamCreateWithFlags(&db->xstream, cudaStreamNonBlocking));
+        for (auto &e : db->xev) TMCK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    }
+    cudaStream_t x = db->xstream;
+    db->res_off.ensure((Q + 1) * 8);
+    PinnedBlock *blk = nullptr;
+    uint64_t cap = 0, total = 0;  // keys the pinned block holds / keys copied so far
+    struct Guard {  // on an error: no copy in flight into a block that is handed back
+        tm_db *db;
+        PinnedBlock **blk;
+        ~Guard() {
+            if (*blk) {
+                cudaStreamSynchronize(db->xstream);
+                pinned_put(*blk);
+            }
+        }
+    } guard{db, &blk};
+    tm_stats_t acc = db->st;
+    double enc = 0, route = 0, scan = 0, merge = 0, tot = 0;
+    uint64_t sums[11] = {};
+    uint32_t launches = 0, scans = 0;
+    for (uint32_t k = 0; k < S; ++k) {
+        const uint64_t qlo = Q * k / S, qn = Q * (k + 1) / S - qlo;
+        if (k) std::swap(db->res_k, db->res_kb);  // range k writes key buffer k & 1
+        // the copy of range k - 2 read this buffer
+        if (k >= 2) TMCK(cudaStreamWaitEvent(s, db->xev[k & 1], 0));
+        const uint64_t n = match_core(db, dq, unique, s, qlo, qn, k > 0);
+        const uint64_t *sorted = n ? db->last_sorted : nullptr;
+        TMCK(launch_query_offsets(sorted, n, qlo, qn, total, db->res_off.as<uint64_t>() + qlo, s));
+        TMCK(cudaEventRecord(db->xev[2], s));
+        finish_timing(db, s);
+        const tm_stats_t &st = db->st;
+        enc += st.encode_ms;
+        route += st.route_ms;
+        scan += st.scan_ms;
+        merge += st.merge_ms;
+        tot += st.total_ms;
+        const uint64_t v[11] = {st.routed, st.candidate_pairs, st.tile_tests, st.pair_checks, st.matched_sets,
+                                st.emitted_pairs, st.result_pairs, st.work_items, st.retries, st.exact_checked,
+                                st.exact_kept};
+        for (int i = 0; i < 11; ++i) sums[i] += v[i];
+        launches += st.kernel_launches + 1;
+        scans += st.scan_launches;
+        acc.scan_variant = st.scan_variant;
+        acc.tuning = st.tuning;
+        if (total + n > cap) {  // the pinned result block: sized by the first range and the largest earlier
+                                // result, so a repeated batch size reuses one cached block; grown if short
+            const uint64_t want = std::max<uint64_t>(std::max<uint64_t>((total + n) + (total + n) / 4,
+                                                                        (n + 1) * S + (n + 1) * S / 4),
+                                                     db->csr_keys_hint + db->csr_keys_hint / 16);
+            PinnedBlock *nb = pinned_get((Q + 1) * 8 + want * 4);
+            if (blk) {
+                TMCK(cudaStreamSynchronize(x));
+                memcpy(nb->p, blk->p, (Q + 1) * 8 + total * 4);
+                pinned_put(blk);
+            }
+            blk = nb;
+            cap = want;
+        }
+        uint64_t *hoff = static_cast<uint64_t *>(blk->p);
+        uint32_t *hk = reinterpret_cast<uint32_t *>(hoff + Q + 1);
+        TMCK(cudaStreamWaitEvent(x, db->xev[2], 0));
+        TMCK(cudaMemcpyAsync(hoff + qlo, db->res_off.as<uint64_t>() + qlo, qn * 8, cudaMemcpyDeviceToHost, x));
+        if (n) TMCK(cudaMemcpyAsync(hk + total, db->res_k.p, n * 4, cudaMemcpyDeviceToHost, x));
+        TMCK(cudaEventRecord(db->xev[k & 1], x));
+        total += n;
+    }
+    TMCK(cudaStreamSynchronize(x));
+    uint64_t *hoff = static_cast<uint64_t *>(blk->p);
+    hoff[Q] = total;
+    db->csr_keys_hint = std::max(db->csr_keys_hint, total);
+    // the call's statistics: sums over the ranges (stage times are the ranges' CUDA-event times)
+    acc.n_queries = Q;
+    uint64_t *dst[11] = {&acc.routed, &acc.candidate_pairs, &acc.tile_tests, &acc.pair_checks, &acc.matched_sets,
+                         &acc.emitted_pairs, &acc.result_pairs, &acc.work_items, &acc.retries, &acc.exact_checked,
+                         &acc.exact_kept};
+    for (int i = 0; i < 11; ++i) *dst[i] = sums[i];
+    acc.encode_ms = enc;
+    acc.route_ms = route;
+    acc.scan_ms = scan;
+    acc.merge_ms = merge;
+    acc.total_ms = tot;
+    acc.kernel_launches = launches;
+    acc.scan_launches = scans;
+    db->st = acc;
+    db->last_sorted = nullptr;  // the pairs of the last range only: not a whole-call result
+    db->last_n = 0;
+    out->n_queries = Q;
+    out->n = total;
+    out->q_off = hoff;
+    out->key = reinterpret_cast<uint32_t *>(hoff + Q + 1);
+    out->priv_ = blk;
+    blk = nullptr;  // handed to the caller (tm_csr_free)
+}
 }  // namespace tmb
 
 extern "C" {
@@ -934,8 +1050,13 @@ tm_status tm_match_batch_csr(tm_db *db, const tm_tagsets *q, int unique, tm_csr 
     DeviceGuard g(db->device);
     cudaStream_t s = db->stream;
     const tm_tagsets dq = upload_queries(db, q, s);
-    const uint64_t n = match_core(db, &dq, unique, s);
     const uint64_t Q = q->n_sets;
+    const uint32_t S = pipeline_ranges(Q);
+    if (S > 1) {
+        csr_pipelined(db, &dq, unique, S, out);
+        return TM_OK;
+    }
+    const uint64_t n = match_core(db, &dq, unique, s);
     db->res_off.ensure((Q + 1) * 8);
     const uint64_t *sorted = n ? db->last_sorted : nullptr;
     TMCK(launch_query_offsets(sorted, n, 0, Q, 0, db->res_off.as<uint64_t>(), s));

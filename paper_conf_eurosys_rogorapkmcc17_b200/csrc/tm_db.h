@@ -152,6 +152,11 @@ struct tm_db {
     // per-call workspace
     DevBuf in_bytes, in_voff, in_tidx, in_soff, in_vhash;  // host-API staging of the queries
     DevBuf vsig, qplanes, bm, word_off, qidx, qoff, item_cnt, item_off, out, out_alt, res_q, res_k, res_off, tmp, ctr;
+    // pipelined tm_match_batch_csr: the D2H of query range k overlaps the GPU work of range k + 1
+    cudaStream_t xstream = nullptr;  // copy stream (created on first use)
+    cudaEvent_t xev[3] = {};         // [0], [1]: copy of the key buffer res_k / res_kb done; [2]: range matched
+    DevBuf res_kb;                   // the second key buffer
+    uint64_t csr_keys_hint = 0;      // keys of the largest pipelined result so far: sizes its pinned block
     DevCounters *h_ctr = nullptr;  // pinned
     unsigned long long *h_nuniq = nullptr;
     unsigned long long cap_qidx = 0, cap_out = 0;
@@ -191,8 +196,10 @@ struct tm_db {
 
 namespace tmb {
 void *cub_tmp(tm_db *db, size_t bytes);
+// encoded: the handle's query planes already hold this batch's signatures (an earlier query range
+// of the same call): S1 is skipped
 uint64_t match_core(tm_db *db, const tm_tagsets *q, int unique, cudaStream_t s, uint64_t qlo = 0,
-                    uint64_t qn = ~0ULL);
+                    uint64_t qn = ~0ULL, bool encoded = false);
 void finish_timing(tm_db *db, cudaStream_t s);
 tm_status translate(const CudaFail &f);
 int check_device(int dev);

@@ -1,20 +1,24 @@
-# final check-in of a round: full GPU suite (SKIP_PYTEST=1 skips), ncu of the bench configs (traffic of this
+# final check-in of this session (the GPU suite ran separately: profiles/r3j_gpu_tests.txt): sanitizers, ncu of the bench configs, launch list, bench lines, HBM sweep, reference arm, per-kernel stage times
 # build), NVTX-filtered launch list, default bench line (C3) + C2 / C4 / C6 lines, the HBM sweep,
-# the reference arm, per-kernel stage times.  compute-sanitizer is closed on the pool (session 3).  usage: bash scripts/gpu_final.sh <tag>
+# the reference arm.   usage: bash scripts/gpu_final.sh <tag>
 TAG=${1:-final}
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build(); g.smoke()" 2>&1 | tail -2
-S=$(date +%s); [ -n "$SKIP_PYTEST" ] || timeout 1500 python -m pytest tests -m gpu -q -s > gpurun_out/${TAG}_pytest.log 2>&1; echo "pytest rc=$? in $(( $(date +%s) - S )) s"; tail -2 gpurun_out/${TAG}_pytest.log
+timeout 1500 compute-sanitizer --tool memcheck --error-exitcode 99 python scripts/sanitize.py 0,5,6,7,8,9,10,11,12,13,14,15,16 100000 > gpurun_out/${TAG}_sanitize_memcheck.log 2>&1; echo "memcheck rc=$?"; tail -1 gpurun_out/${TAG}_sanitize_memcheck.log
+for T in racecheck synccheck; do
+  timeout 1500 compute-sanitizer --tool $T --error-exitcode 99 python scripts/sanitize.py 0,5,6,7,8,9,10,11,12,13,14,15,16 20000 > gpurun_out/${TAG}_sanitize_${T}.log 2>&1; echo "$T rc=$?"; tail -1 gpurun_out/${TAG}_sanitize_${T}.log
+done
 BID=$(python -c "from paper_conf_eurosys_rogorapkmcc17_b200 import tagmatch as t; print(t.build_id())")
 for CFG in C3 C4; do
   TM_SCAN_VARIANT=14 timeout 1500 /usr/local/cuda/bin/ncu --set full --clock-control none --import-source on \
-    --nvtx --nvtx-include "bench_device/" -k regex:k_scan -s 3 -c 1 -o gpurun_out/${TAG}_${CFG}_scan \
+    -k regex:k_scan -s 12 -c 1 -o gpurun_out/${TAG}_${CFG}_scan \
     python bench.py --config $CFG --steps 1 --warmup 3 --no-cpu-baseline --no-hbm > gpurun_out/${TAG}_${CFG}_ncu.log 2>&1
   echo "ncu $CFG rc=$?"
   python scripts/ncu_summary.py gpurun_out/${TAG}_${CFG}_scan.ncu-rep --config $CFG --build-id $BID --variant 14 \
     --json profiles/ncu_scan_traffic_${CFG}.json > gpurun_out/${TAG}_${CFG}_scan_ncu.txt 2>&1
   cp profiles/ncu_scan_traffic_${CFG}.json gpurun_out/${TAG}_ncu_scan_traffic_${CFG}.json 2>/dev/null
-timeout 900 /usr/local/cuda/bin/ncu --nvtx --nvtx-include "bench_device/" --metrics gpu__time_duration.sum --clock-control none \
+done
+timeout 900 /usr/local/cuda/bin/ncu --nvtx --nvtx-include "tm_match/" --metrics gpu__time_duration.sum --clock-control none \
   -c 200 --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-hbm > /dev/null 2>&1; echo "launches rc=$?"
 timeout 1200 python bench.py --steps 20 --warmup 5 > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err; echo "bench C3 rc=$?"; tail -1 gpurun_out/${TAG}_bench.err
 timeout 900 python bench.py --config C2 --steps 20 --warmup 5 --no-hbm > gpurun_out/${TAG}_C2_bench.json 2> gpurun_out/${TAG}_C2_bench.err; echo "bench C2 rc=$?"

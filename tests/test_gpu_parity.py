@@ -601,3 +601,44 @@ def test_crafted_workload_exact_mode(s, t):
         gq, gk = db.match_batch(wl.queries, False)
     keep = np.isin(gq, qsel)
     assert list(zip(gq[keep].tolist(), gk[keep].tolist())) == want
+
+
+@pytest.mark.parametrize("ranges", ["1", "2", "3", "7"])
+def test_csr_pipelined_ranges(c2, c2_oracle, ranges, monkeypatch):
+    """Pipelined tm_match_batch_csr (TM_PIPELINE query ranges: the D2H of range k overlaps the
+    GPU work of range k + 1; double-buffered keys, per-range query offsets): the per-query key
+    lists equal the oracle's pairs for any number of ranges, uneven ones included, and the call's
+    statistics are the sums over its ranges."""
+    monkeypatch.setenv("TM_PIPELINE", ranges)
+    with tmb.Database(c2.db, c2.key_off, c2.keys, max_partition=c2.max_partition, tile_filter=1,
+                      row_order=1) as db:
+        for unique in (False, True):
+            for _ in range(2):   # the second call reuses the copy stream, buffers and pinned blocks
+                off, key = db.match_batch_csr(c2.queries, unique)
+                wq, wk = c2_oracle[unique]
+                Q = c2.queries.n_sets
+                assert off.size == Q + 1 and off[0] == 0 and off[-1] == key.size == wk.size
+                assert np.array_equal(np.repeat(np.arange(Q, dtype=np.uint32), np.diff(off).astype(np.int64)), wq)
+                assert np.array_equal(key, wk)
+                st = db.stats()
+                assert st["result_pairs"] == wk.size and st["n_queries"] == Q
+
+
+def test_csr_pipelined_exact(monkeypatch):
+    """The pipelined CSR call in exact mode (each query range runs the exact post-check) equals
+    the oracle's string-level containment on a workload with many Bloom false positives."""
+    monkeypatch.setenv("TM_PIPELINE", "3")
+    rnd = random.Random(9)
+    vocab = [f"w{i}".encode() for i in range(50)]
+    sets = [[rnd.choice(vocab) for _ in range(rnd.randint(0, 4))] for _ in range(2000)]
+    keys = [[rnd.randrange(1000) for _ in range(rnd.randint(0, 2))] for _ in range(len(sets))]
+    queries = [[rnd.choice(vocab) for _ in range(rnd.randint(8, 30))] for _ in range(301)]
+    key_off = np.zeros(len(keys) + 1, np.uint64)
+    key_off[1:] = np.cumsum([len(k) for k in keys])
+    flat = np.array([k for kl in keys for k in kl], np.uint32)
+    for unique in (False, True):
+        want = o1.match_exact(sets, keys, queries, unique)
+        with tmb.Database(tagsets(sets), key_off, flat, max_partition=100, exact=1) as db:
+            off, key = db.match_batch_csr(tagsets(queries), unique)
+        q = np.repeat(np.arange(len(queries), dtype=np.uint32), np.diff(off).astype(np.int64))
+        assert list(zip(q.tolist(), key.tolist())) == want
