@@ -703,7 +703,7 @@ void destroy_db(tm_db *db) {
                       &db->res_k, &db->res_off, &db->tmp, &db->ctr, &db->xcounts, &db->xall, &db->xrecv, &db->xalt, &db->mq,
                       &db->mk, &db->xv_bytes, &db->xv_off, &db->xv_hash, &db->xv_pos, &db->xv_canon, &db->xs_off,
                       &db->xs_ids, &db->xk_off, &db->xk_keys, &db->xq_canon, &db->xq_ids, &db->xflag, &db->xcnt,
-                      &db->xkoff, &db->xkcnt, &db->res_kb})
+                      &db->xkoff, &db->xkcnt, &db->res_kb, &db->res_qb})
         b->release();
     for (auto &e : db->ev)
         if (e) cudaEventDestroy(e);
@@ -865,8 +865,8 @@ void rebuild(tm_db *db, const tm_tagsets *sets, const uint32_t *keys, const tm_c
     fresh->nccl_comm = nullptr;
     destroy_db(fresh);
 }
-// Query ranges of a pipelined tm_match_batch_csr: the result's device-to-host copy (4 B per pair,
-// ~0.85 GB at C3, PCIe-bound) of range k runs on a copy stream while the GPU matches range k + 1,
+// Query ranges of a pipelined tm_match_batch_csr / tm_match_batch: the result's device-to-host copy
+// (4 or 8 B per pair, ~0.85 GB at C3, PCIe-bound) of range k runs on a copy stream while the GPU matches range k + 1,
 // so only the last range's copy stays on the critical path.  TM_PIPELINE=n forces n ranges (1 = off).
 uint32_t pipeline_ranges(uint64_t Q) {
     const char *e = getenv("TM_PIPELINE");
@@ -875,17 +875,24 @@ uint32_t pipeline_ranges(uint64_t Q) {
     return Q >= (1ULL << 18) ? 4u : 1u;  // smaller batches: the per-range fixed cost outweighs the copy
 }
 
-void csr_pipelined(tm_db *db, const tm_tagsets *dq, int unique, uint32_t S, tm_csr *out) {
+// Pipelined tm_match_batch_csr (cout) / tm_match_batch (pout): S query ranges matched in order
+// on the handle's stream; range k's result (keys and its slice of the query offsets, or its query
+// and key arrays) is copied to the pinned result block on a copy stream while range k + 1 runs.
+// Result buffers are double-buffered (res_k / res_kb, res_q / res_qb), each reused only after the
+// copy that read it; the pinned block holds [Q + 1 offsets | cap keys] or [cap queries | cap keys].
+void match_pipelined(tm_db *db, const tm_tagsets *dq, int unique, uint32_t S, tm_csr *cout, tm_pairs *pout) {
     cudaStream_t s = db->stream;
     const uint64_t Q = dq->n_sets;
+    const bool csr = cout != nullptr;
     if (!db->xstream) {
         TMCK(cudaStreamCreateWithFlags(&db->xstream, cudaStreamNonBlocking));
         for (auto &e : db->xev) TMCK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     }
     cudaStream_t x = db->xstream;
-    db->res_off.ensure((Q + 1) * 8);
+    if (csr) db->res_off.ensure((Q + 1) * 8);
+    const uint64_t head = csr ? (Q + 1) * 8 : 0;  // bytes before the first result array
     PinnedBlock *blk = nullptr;
-    uint64_t cap = 0, total = 0;  // keys the pinned block holds / keys copied so far
+    uint64_t cap = 0, total = 0;  // pairs the pinned block holds (per array) / pairs copied so far
     struct Guard {  // on an error: no copy in flight into a block that is handed back
         tm_db *db;
         PinnedBlock **blk;
@@ -896,18 +903,25 @@ void csr_pipelined(tm_db *db, const tm_tagsets *dq, int unique, uint32_t S, tm_c
             }
         }
     } guard{db, &blk};
+    auto q_arr = [&](void *base) { return reinterpret_cast<uint32_t *>(static_cast<char *>(base) + head); };
+    auto k_arr = [&](void *base, uint64_t c) { return q_arr(base) + (csr ? 0 : c); };
     tm_stats_t acc = db->st;
     double enc = 0, route = 0, scan = 0, merge = 0, tot = 0;
     uint64_t sums[11] = {};
     uint32_t launches = 0, scans = 0;
     for (uint32_t k = 0; k < S; ++k) {
         const uint64_t qlo = Q * k / S, qn = Q * (k + 1) / S - qlo;
-        if (k) std::swap(db->res_k, db->res_kb);  // range k writes key buffer k & 1
-        // the copy of range k - 2 read this buffer
+        if (k) {  // range k writes result buffers k & 1
+            std::swap(db->res_k, db->res_kb);
+            std::swap(db->res_q, db->res_qb);
+        }
+        // the copy of range k - 2 read these buffers
         if (k >= 2) TMCK(cudaStreamWaitEvent(s, db->xev[k & 1], 0));
         const uint64_t n = match_core(db, dq, unique, s, qlo, qn, k > 0);
-        const uint64_t *sorted = n ? db->last_sorted : nullptr;
-        TMCK(launch_query_offsets(sorted, n, qlo, qn, total, db->res_off.as<uint64_t>() + qlo, s));
+        if (csr) {
+            const uint64_t *sorted = n ? db->last_sorted : nullptr;
+            TMCK(launch_query_offsets(sorted, n, qlo, qn, total, db->res_off.as<uint64_t>() + qlo, s));
+        }
         TMCK(cudaEventRecord(db->xev[2], s));
         finish_timing(db, s);
         const tm_stats_t &st = db->st;
@@ -920,7 +934,7 @@ void csr_pipelined(tm_db *db, const tm_tagsets *dq, int unique, uint32_t S, tm_c
                                 st.emitted_pairs, st.result_pairs, st.work_items, st.retries, st.exact_checked,
                                 st.exact_kept};
         for (int i = 0; i < 11; ++i) sums[i] += v[i];
-        launches += st.kernel_launches + 1;
+        launches += st.kernel_launches + (csr ? 1 : 0);
         scans += st.scan_launches;
         acc.scan_variant = st.scan_variant;
         acc.tuning = st.tuning;
@@ -928,28 +942,29 @@ void csr_pipelined(tm_db *db, const tm_tagsets *dq, int unique, uint32_t S, tm_c
                                 // result, so a repeated batch size reuses one cached block; grown if short
             const uint64_t want = std::max<uint64_t>(std::max<uint64_t>((total + n) + (total + n) / 4,
                                                                         (n + 1) * S + (n + 1) * S / 4),
-                                                     db->csr_keys_hint + db->csr_keys_hint / 16);
-            PinnedBlock *nb = pinned_get((Q + 1) * 8 + want * 4);
+                                                     db->pipe_pairs_hint + db->pipe_pairs_hint / 16);
+            PinnedBlock *nb = pinned_get(head + want * 4 * (csr ? 1 : 2));
             if (blk) {
                 TMCK(cudaStreamSynchronize(x));
-                memcpy(nb->p, blk->p, (Q + 1) * 8 + total * 4);
+                memcpy(nb->p, blk->p, head + total * 4);  // offsets + keys, or the queries
+                if (!csr) memcpy(k_arr(nb->p, want), k_arr(blk->p, cap), total * 4);
                 pinned_put(blk);
             }
             blk = nb;
             cap = want;
         }
-        uint64_t *hoff = static_cast<uint64_t *>(blk->p);
-        uint32_t *hk = reinterpret_cast<uint32_t *>(hoff + Q + 1);
         TMCK(cudaStreamWaitEvent(x, db->xev[2], 0));
-        TMCK(cudaMemcpyAsync(hoff + qlo, db->res_off.as<uint64_t>() + qlo, qn * 8, cudaMemcpyDeviceToHost, x));
-        if (n) TMCK(cudaMemcpyAsync(hk + total, db->res_k.p, n * 4, cudaMemcpyDeviceToHost, x));
+        if (csr)
+            TMCK(cudaMemcpyAsync(static_cast<uint64_t *>(blk->p) + qlo, db->res_off.as<uint64_t>() + qlo, qn * 8,
+                                 cudaMemcpyDeviceToHost, x));
+        else if (n)
+            TMCK(cudaMemcpyAsync(q_arr(blk->p) + total, db->res_q.p, n * 4, cudaMemcpyDeviceToHost, x));
+        if (n) TMCK(cudaMemcpyAsync(k_arr(blk->p, cap) + total, db->res_k.p, n * 4, cudaMemcpyDeviceToHost, x));
         TMCK(cudaEventRecord(db->xev[k & 1], x));
         total += n;
     }
     TMCK(cudaStreamSynchronize(x));
-    uint64_t *hoff = static_cast<uint64_t *>(blk->p);
-    hoff[Q] = total;
-    db->csr_keys_hint = std::max(db->csr_keys_hint, total);
+    db->pipe_pairs_hint = std::max(db->pipe_pairs_hint, total);
     // the call's statistics: sums over the ranges (stage times are the ranges' CUDA-event times)
     acc.n_queries = Q;
     uint64_t *dst[11] = {&acc.routed, &acc.candidate_pairs, &acc.tile_tests, &acc.pair_checks, &acc.matched_sets,
@@ -966,12 +981,21 @@ void csr_pipelined(tm_db *db, const tm_tagsets *dq, int unique, uint32_t S, tm_c
     db->st = acc;
     db->last_sorted = nullptr;  // the pairs of the last range only: not a whole-call result
     db->last_n = 0;
-    out->n_queries = Q;
-    out->n = total;
-    out->q_off = hoff;
-    out->key = reinterpret_cast<uint32_t *>(hoff + Q + 1);
-    out->priv_ = blk;
-    blk = nullptr;  // handed to the caller (tm_csr_free)
+    if (csr) {
+        uint64_t *hoff = static_cast<uint64_t *>(blk->p);
+        hoff[Q] = total;
+        cout->n_queries = Q;
+        cout->n = total;
+        cout->q_off = hoff;
+        cout->key = k_arr(blk->p, cap);
+        cout->priv_ = blk;
+    } else {
+        pout->n = total;
+        pout->query = q_arr(blk->p);
+        pout->key = k_arr(blk->p, cap);
+        pout->priv_ = blk;
+    }
+    blk = nullptr;  // handed to the caller (tm_csr_free / tm_pairs_free)
 }
 }  // namespace tmb
 
@@ -1013,6 +1037,11 @@ tm_status tm_match_batch(tm_db *db, const tm_tagsets *q, int unique, tm_pairs *o
     DeviceGuard g(db->device);
     cudaStream_t s = db->stream;
     const tm_tagsets dq = upload_queries(db, q, s);  // one H2D copy of the query batch
+    const uint32_t S = pipeline_ranges(q->n_sets);
+    if (S > 1) {  // query ranges, each range's D2H under the next range's GPU work
+        match_pipelined(db, &dq, unique, S, nullptr, out);
+        return TM_OK;
+    }
     const uint64_t n = match_core(db, &dq, unique, s);
     PinnedBlock *blk = pinned_get(std::max<uint64_t>(n, 1) * 8);
     uint32_t *hq = static_cast<uint32_t *>(blk->p), *hk = hq + n;
@@ -1053,7 +1082,7 @@ tm_status tm_match_batch_csr(tm_db *db, const tm_tagsets *q, int unique, tm_csr 
     const uint64_t Q = q->n_sets;
     const uint32_t S = pipeline_ranges(Q);
     if (S > 1) {
-        csr_pipelined(db, &dq, unique, S, out);
+        match_pipelined(db, &dq, unique, S, out, nullptr);
         return TM_OK;
     }
     const uint64_t n = match_core(db, &dq, unique, s);

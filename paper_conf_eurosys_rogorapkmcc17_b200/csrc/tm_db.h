@@ -155,8 +155,8 @@ struct tm_db {
     // pipelined tm_match_batch_csr: the D2H of query range k overlaps the GPU work of range k + 1
     cudaStream_t xstream = nullptr;  // copy stream (created on first use)
     cudaEvent_t xev[3] = {};         // [0], [1]: copy of the key buffer res_k / res_kb done; [2]: range matched
-    DevBuf res_kb;                   // the second key buffer
-    uint64_t csr_keys_hint = 0;      // keys of the largest pipelined result so far: sizes its pinned block
+    DevBuf res_kb, res_qb;           // the second key / query buffers
+    uint64_t pipe_pairs_hint = 0;    // pairs of the largest pipelined result so far: sizes its pinned block
     DevCounters *h_ctr = nullptr;  // pinned
     unsigned long long *h_nuniq = nullptr;
     unsigned long long cap_qidx = 0, cap_out = 0;

@@ -14,6 +14,7 @@ for CFG in C3 C4; do
   python scripts/ncu_summary.py gpurun_out/${TAG}_${CFG}_scan.ncu-rep --config $CFG --build-id $BID --variant 14 \
     --json profiles/ncu_scan_traffic_${CFG}.json > gpurun_out/${TAG}_${CFG}_scan_ncu.txt 2>&1
   cp profiles/ncu_scan_traffic_${CFG}.json gpurun_out/${TAG}_ncu_scan_traffic_${CFG}.json 2>/dev/null
+done
 timeout 900 /usr/local/cuda/bin/ncu --nvtx --nvtx-include "bench_device/" --metrics gpu__time_duration.sum --clock-control none \
   -c 200 --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-hbm > /dev/null 2>&1; echo "launches rc=$?"
 timeout 1200 python bench.py --steps 20 --warmup 5 > gpurun_out/${TAG}_bench.json 2> gpurun_out/${TAG}_bench.err; echo "bench C3 rc=$?"; tail -1 gpurun_out/${TAG}_bench.err

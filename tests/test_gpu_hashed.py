@@ -89,3 +89,20 @@ def test_hashed_rejected_where_strings_are_needed(wl):
     with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, exact=1) as db:
         with pytest.raises(tmb.TagMatchError):           # the exact check compares strings
             db.match_batch(hq, False)
+
+
+@pytest.mark.parametrize("mode", [0, 1])   # TM_SHARD_PARTITIONED, TM_SHARD_REPLICATED
+def test_hashed_queries_in_process_group(wl, mode):
+    """An in-process multi-GPU database (2 sub-databases on device 0) takes the hashed batch and
+    a hashed plan sample (partition -> GPU plan by routed counts) and returns the oracle's pairs."""
+    q = wl.queries
+    hq = tmb.HostTagSets.hashed(vocab_hashes(q), q.tag_idx, q.set_off)
+    smp = q.subset(np.arange(500))
+    hs = tmb.HostTagSets.hashed(vocab_hashes(smp), smp.tag_idx, smp.set_off)
+    db_sig, q_sig = o2.encode(wl.db), o2.encode(q)
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, tile_filter=1, row_order=1,
+                      n_gpus=2, shard_mode=mode, device_ids=[0, 0], plan_sample=hs) as db:
+        for unique in (False, True):
+            gq, gk = db.match_batch(hq, unique)
+            wq, wk = o2.match_brute(db_sig, wl.key_off, wl.keys, q_sig, unique)
+            assert np.array_equal(gq, wq) and np.array_equal(gk, wk), f"mode={mode} unique={unique}"

@@ -605,7 +605,7 @@ def test_crafted_workload_exact_mode(s, t):
 
 @pytest.mark.parametrize("ranges", ["1", "2", "3", "7"])
 def test_csr_pipelined_ranges(c2, c2_oracle, ranges, monkeypatch):
-    """Pipelined tm_match_batch_csr (TM_PIPELINE query ranges: the D2H of range k overlaps the
+    """Pipelined tm_match_batch_csr and tm_match_batch (TM_PIPELINE query ranges: the D2H of range k overlaps the
     GPU work of range k + 1; double-buffered keys, per-range query offsets): the per-query key
     lists equal the oracle's pairs for any number of ranges, uneven ones included, and the call's
     statistics are the sums over its ranges."""
@@ -622,6 +622,7 @@ def test_csr_pipelined_ranges(c2, c2_oracle, ranges, monkeypatch):
                 assert np.array_equal(key, wk)
                 st = db.stats()
                 assert st["result_pairs"] == wk.size and st["n_queries"] == Q
+                assert_pairs_equal(db.match_batch(c2.queries, unique), (wq, wk), f"pairs, {ranges} ranges")
 
 
 def test_csr_pipelined_exact(monkeypatch):
