@@ -293,6 +293,9 @@ def ncu_traffic(config: str, variant: int, build_id: str):
     """DRAM traffic of k_scan from the committed ncu capture of this config, only if it was
     taken on the same library build (tm_build_id) and scan variant; else None + why."""
     path = os.path.join(ROOT, "profiles", f"ncu_scan_traffic_{config}.json")
+    vpath = os.path.join(ROOT, "profiles", f"ncu_scan_traffic_{config}_v{variant}.json")
+    if os.path.exists(vpath):   # a capture of this variant (the handle's tuner may settle on either)
+        path = vpath
     try:
         with open(path) as f:
             tr = json.load(f)
