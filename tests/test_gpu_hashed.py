@@ -89,6 +89,20 @@ def test_hashed_rejected_where_strings_are_needed(wl):
     with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition, exact=1) as db:
         with pytest.raises(tmb.TagMatchError):           # the exact check compares strings
             db.match_batch(hq, False)
+    # the mutable store interns tag strings (tm_add_sets), the stream replays strings
+    mdb = tmb.Database.create(max_partition=1000)
+    try:
+        with pytest.raises(tmb.TagMatchError):
+            mdb.add_sets(hq, np.arange(q.n_sets + 1, dtype=np.uint64), np.arange(q.n_sets, dtype=np.uint32))
+    finally:
+        mdb.close()
+    with tmb.Database(wl.db, wl.key_off, wl.keys, max_partition=wl.max_partition) as db:
+        st = tmb.tagmatch.Stream(db, 64, 1000, False)
+        try:
+            with pytest.raises(tmb.TagMatchError):
+                st.replay(hq, np.zeros(q.n_sets, np.uint64))
+        finally:
+            st.close()
 
 
 @pytest.mark.parametrize("mode", [0, 1])   # TM_SHARD_PARTITIONED, TM_SHARD_REPLICATED
