@@ -511,6 +511,7 @@ void build_impl(tm_db *db, const tm_tagsets *sets, const uint64_t *key_off, cons
     db->n_entries = K;
     if (db->cfg.max_partition == TM_AUTO_MAX_PARTITION)  // reading R8b: MAX_P = N / 3*10^4 (measured)
         db->cfg.max_partition = (uint32_t)std::min<uint64_t>(200000, std::max<uint64_t>(5000, N / 30000));
+    if (db->cfg.tile_filter != 2 && db->cfg.max_partition <= kSmallPMax) db->set_tune(kTuneSmallP);
 
     // S0a: encode every set on the GPU
     DevBuf d_bytes, d_voff, d_tidx, d_soff, d_vsig, d_planes, d_sorted, d_idx, d_idx2, d_key, d_key2;

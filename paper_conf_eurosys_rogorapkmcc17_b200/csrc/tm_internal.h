@@ -30,10 +30,15 @@ constexpr int kMaxOwners = 8;       // fused exchange: GPUs of an in-process gro
 constexpr int kChunk = TM_CHUNK;   // queries per work item (per-partition batch); 640 fits 7 CTAs/SM of shared memory and measured 1.3% faster than 512 (profiles/r1v34_ab.txt)
 constexpr int kSmallBatch = 8;     // partition batches up to this size take the unfiltered streaming path
 constexpr int kRangeRows = 8192;    // default rows per work item (multiple of 256; TM_RANGE_ROWS)
-constexpr int kScanVariants = 17;    // k_scan variants (TM_SCAN_VARIANT)
+constexpr int kScanVariants = 19;    // k_scan variants (TM_SCAN_VARIANT)
 constexpr int kTune[] = {14, 8};  // variants the handle times on its first calls (first = default)
 constexpr int kTuneN = 2;
 constexpr int kTuneDense[] = {13, 9};  // tables without a pre-filter (tile_filter = 2): the dense scan
+// partitions of at most kSmallPMax sets (the auto MAX_P of large tables): 128-row level-A blocks
+// (C3 at 5K: scan 190.1 vs 194.3 ms; C4 at 10K 390.1 vs 397.6; C3 at 200K 285.9 vs 276.4: 256 rows
+// stay for large partitions; profiles/r3u_*)
+constexpr int kTuneSmallP[] = {17, 18};
+constexpr uint32_t kSmallPMax = 50000;
 constexpr int kTuneMinQ = 4096;     // smaller calls are not tuned (default variant kTune[0])
 
 struct DevCounters {            // zeroed at the start of every match call

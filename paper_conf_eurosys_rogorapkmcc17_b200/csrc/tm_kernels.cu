@@ -615,8 +615,11 @@ __device__ __forceinline__ uint64_t warp_and(uint64_t v) {
 // set-up (the two pre-check words read from the build-time wwords plane, no per-lane selects).
 __device__ unsigned long long g_scan_dbg[12];  // OPT & 512: pre-check pass statistics (diagnostic variant)
 
-template <bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0>
+// BT: tiles per level-A block (<= kBlockTiles): 8 (256 rows) or 4 (128 rows; the default with small
+// partitions)
+template <bool WORD1 = false, int MINB = 8, bool STREAM = false, int OPT = 0, int BT = kBlockTiles>
 __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams p) {
+    static_assert(BT >= 1 && BT <= kBlockTiles, "level-A block of at most kBlockTiles tiles");
     constexpr bool kImad = (OPT & 1) != 0;
     constexpr bool kLean = WORD1 && !STREAM && (OPT & 16) != 0;
     constexpr bool kFused = (OPT & 64) != 0;  // emission into the owners' regions (in-process group)
@@ -815,7 +818,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
 
         if constexpr (!STREAM) {
         const uint32_t ntile = (rhi - rlo) / kTile;
-        const uint32_t nblock = (ntile + kBlockTiles - 1) / kBlockTiles;
+        const uint32_t nblock = (ntile + BT - 1) / BT;
         // unit = (256-row block, query sub-range), taken dynamically through unit_ctr;
         // few blocks: split the batch so every warp has work
         // (a small item -- few blocks -- is split over query sub-ranges until it has p.unit_target
@@ -833,7 +836,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
             const uint32_t blk = u / nsplit, sub = u % nsplit;
             const uint32_t qs = sub * subsz, qe = min(nq, qs + subsz);
             if (qs >= qe) continue;
-            const uint32_t t_first = blk * kBlockTiles, t_end = min(ntile, t_first + kBlockTiles);
+            const uint32_t t_first = blk * BT, t_end = min(ntile, t_first + BT);
             const uint32_t brow0 = rlo + t_first * kTile;
             const uint32_t bend = min(rlo + t_end * kTile, real_end);  // real rows of the block
             // ---- level A: the block's common mask
@@ -846,7 +849,7 @@ __global__ void __launch_bounds__(kScanWarps * 32, MINB) k_scan(const ScanParams
                 const bool in = (uint32_t)lane < t_end - t_first;
                 const uint64_t m0 = in ? __ldg(p.t0 + t) : ~0ULL, m1 = in ? __ldg(p.t1 + t) : ~0ULL,
                                m2 = in ? __ldg(p.t2 + t) : ~0ULL;
-                if ((uint32_t)lane < (uint32_t)kBlockTiles) {  // the block's tile masks, for level B
+                if ((uint32_t)lane < (uint32_t)BT) {  // the block's tile masks, for level B
                     sm.tmask[warp][0][lane] = m0;
                     sm.tmask[warp][1][lane] = m1;
                     sm.tmask[warp][2][lane] = m2;
@@ -1567,6 +1570,8 @@ ScanFn scan_fn_t(int variant) {
         case 14: return k_scan<true, 7, false, 17 | F>;  // 8 + lean tile set-up (the default)
         case 15: return k_dense<false, 21 | F>;  // 13 + the build-time pre-check words (no selects)
         case 16: return k_scan<true, 7, false, 17 | 512 | F>;  // 14 + pre-check pass statistics (diagnostic)
+        case 17: return k_scan<true, 7, false, 17 | F, 4>;  // 14 with 128-row level-A blocks
+        case 18: return k_scan<true, 7, false, 1 | F, 4>;   // 8 with 128-row level-A blocks
         default: return nullptr;
     }
 }
@@ -1588,7 +1593,7 @@ int scan_variant_env() {
     // <= kSmallBatch queries, else mapped to 0 / 5 by the caller); 9-13, 15 = the dense
     // (unfiltered) scan (9 two rows per lane, 13 four, 10 / 12 bulk-copy staged, 11 / 12 without
     // the FMA accumulate, 15 = 13 with build-time pre-check words; 16 = 14 printing pre-check pass
-    // statistics, a diagnostic).  Unset or unknown (-1): the
+    // statistics, a diagnostic; 17 / 18 = 14 / 8 with 128-row level-A blocks).  Unset or unknown (-1): the
     // handle tunes on its first calls.
     const char *e = getenv("TM_SCAN_VARIANT");
     if (!e) return -1;

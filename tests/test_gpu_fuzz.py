@@ -41,7 +41,7 @@ def test_random_configuration(case, monkeypatch):
     row_order = rnd.choice([0, 1]) if tile_filter else 0
     exact = rnd.random() < 0.35
     unique = rnd.random() < 0.5
-    variant = rnd.choice(["", "0", "5", "5", "6", "7", "8", "9", "10", "11", "12", "13", "14", "14", "15", "16"])
+    variant = rnd.choice(["", "0", "5", "5", "6", "7", "8", "9", "10", "11", "12", "13", "14", "14", "15", "16", "17", "17", "18"])
     if variant:
         monkeypatch.setenv("TM_SCAN_VARIANT", variant)
     else:

@@ -211,7 +211,7 @@ def test_c2_full_parity(c2, c2_oracle, layout):
 
 
 @pytest.mark.parametrize("variant", ["0", "5", "6", "7", "8", "9", "10", "11", "12", "13",
-                                     "14", "15", "16"])
+                                     "14", "15", "16", "17", "18"])
 def test_c2_every_scan_variant(c2, c2_oracle, variant, monkeypatch):
     """Every scan-kernel variant (TM_SCAN_VARIANT) gives the oracle's
     pairs at C2, in the layout bench.py times (balanced splits + AND masks)."""
