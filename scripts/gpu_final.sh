@@ -13,6 +13,7 @@ for CFG in C3 C4; do for V in ${NCU_VARIANTS:-17 18}; do
   echo "ncu $CFG v$V rc=$?"
   python scripts/ncu_summary.py gpurun_out/${TAG}_${CFG}_v${V}_scan.ncu-rep --config $CFG --build-id $BID --variant $V \
     --json gpurun_out/${TAG}_ncu_scan_traffic_${CFG}_v${V}.json > gpurun_out/${TAG}_${CFG}_v${V}_scan_ncu.txt 2>&1
+  cp gpurun_out/${TAG}_ncu_scan_traffic_${CFG}_v${V}.json profiles/ncu_scan_traffic_${CFG}_v${V}.json 2>/dev/null  # the bench lines below read it
 done; done
 timeout 900 /usr/local/cuda/bin/ncu --nvtx --nvtx-include "bench_device/" --metrics gpu__time_duration.sum --clock-control none \
   -c 200 --csv --log-file gpurun_out/${TAG}_launches.csv python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-hbm > /dev/null 2>&1; echo "launches rc=$?"
